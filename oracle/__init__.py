@@ -1,0 +1,268 @@
+"""CPU oracle for the HIPAcc local operators (Membarth et al., IPDPS 2012).
+
+TEST INFRASTRUCTURE ONLY.  Only ``tests/``, ``__graft_entry__.smoke()`` and
+``bench.py``'s ``cpu_baseline`` / ``--impl reference`` legs may import this
+package.  The product package ``paper_conf_ipps_membarthhtke12_b200`` never
+imports it and shares no code with it (see ``oracle/lop_oracle.c`` header).
+
+This module is argument marshalling only: it compiles ``lop_oracle.c`` with
+gcc (-O2, no -ffast-math, OpenMP over output rows) into ``liblop_oracle.so``
+next to this file and wraps each entry point for numpy arrays.  All arithmetic
+lives in the C file, in double precision, in the order of Algorithm 1
+(PAPER.md L169-L186).
+
+Parity status (details in DESIGN.md "Oracle pins"):
+  map_index, read               pinned: Fig. 2 golden cells, np.pad
+  closeness_mask                pinned: Listing 4 printed value 0.018316,
+                                        Listing 1 l.21 product form
+  gaussian_mask / sobel_mask    pinned: binomial coefficients (scipy.special),
+                                        ramp responses
+  convolve_f32 / convolve_u8    pinned: scipy.ndimage.correlate (all modes),
+                                        impulse response, ramps, separability
+  quantize                      pinned: hand-computed cases, numpy floor-div
+  bilateral_f32                 pinned: sigma_r->inf == scipy Gaussian
+                                        correlate, hand-computed 3x3 examples,
+                                        step-edge preservation, constant image,
+                                        convexity, flip symmetry
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+import threading
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "lop_oracle.c")
+_LIB = os.path.join(_HERE, "liblop_oracle.so")
+_lock = threading.Lock()
+_lib = None
+
+UNDEFINED, CLAMP, REPEAT, MIRROR, CONSTANT = 0, 1, 2, 3, 4
+MODES = {"undefined": UNDEFINED, "clamp": CLAMP, "repeat": REPEAT,
+         "mirror": MIRROR, "constant": CONSTANT}
+
+
+def build(force: bool = False) -> str:
+    """Compile the oracle (plain C, gcc -O2 -fopenmp, no fast-math)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        tmp = _LIB + ".tmp%d" % os.getpid()
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-fopenmp",
+                               "-Wall", "-o", tmp, _SRC, "-lm"])
+        os.replace(tmp, _LIB)
+    return _LIB
+
+
+def _load():
+    global _lib
+    with _lock:
+        if _lib is None:
+            lib = ctypes.CDLL(build())
+            i64, i32, dbl, vp = ctypes.c_int64, ctypes.c_int, ctypes.c_double, ctypes.c_void_p
+            lib.oracle_num_threads.restype = i32
+            lib.oracle_map_index.argtypes = [i64, i64, i32]
+            lib.oracle_map_index.restype = i64
+            lib.oracle_read_f32.argtypes = [vp, i64, i64, i64, i64, i64, i32, dbl, vp]
+            lib.oracle_read_f32.restype = dbl
+            lib.oracle_closeness_mask.argtypes = [dbl, i32, i32, vp]
+            lib.oracle_gaussian_mask_int.argtypes = [i32, vp]
+            lib.oracle_gaussian_mask_int.restype = i32
+            lib.oracle_sobel_mask_int.argtypes = [i32, vp]
+            lib.oracle_convolve_f32.argtypes = [vp, i64, i64, i64, vp, i32, i32, i32, dbl,
+                                                i64, i64, vp, vp]
+            lib.oracle_convolve_f32_points.argtypes = [vp, i64, i64, i64, vp, i32, i32, i32,
+                                                       dbl, vp, vp, i64, vp, vp]
+            lib.oracle_convolve_u8_sum.argtypes = [vp, i64, i64, i64, vp, i32, i32, i32, i64,
+                                                   i64, i64, vp, vp]
+            lib.oracle_convolve_u8_sum_points.argtypes = [vp, i64, i64, i64, vp, i32, i32, i32,
+                                                          i64, vp, vp, i64, vp, vp]
+            lib.oracle_quantize.argtypes = [i64, i32, i32]
+            lib.oracle_quantize.restype = i64
+            lib.oracle_bilateral_f32.argtypes = [vp, i64, i64, i64, vp, i32, i32, dbl, dbl,
+                                                 i32, dbl, i64, i64, vp, vp]
+            lib.oracle_bilateral_f32_points.argtypes = [vp, i64, i64, i64, vp, i32, i32, dbl,
+                                                        dbl, i32, dbl, vp, vp, i64, vp, vp]
+            _lib = lib
+    return _lib
+
+
+def _ptr(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+def _mode(mode) -> int:
+    return MODES[mode] if isinstance(mode, str) else int(mode)
+
+
+def _img(img: np.ndarray, dtype):
+    img = np.asarray(img)
+    if img.dtype != dtype:
+        raise TypeError("oracle expects %s image, got %s" % (dtype, img.dtype))
+    if img.ndim != 2:
+        raise ValueError("oracle expects a 2D image")
+    if img.strides[1] != img.itemsize or img.strides[0] % img.itemsize:
+        img = np.ascontiguousarray(img)
+    return img, img.strides[0] // img.itemsize
+
+
+def num_threads() -> int:
+    return _load().oracle_num_threads()
+
+
+def map_index(i: int, n: int, mode) -> int:
+    """Per-axis index adjustment (Fig. 2); -1 = no pixel."""
+    return _load().oracle_map_index(int(i), int(n), _mode(mode))
+
+
+def read(img: np.ndarray, x: int, y: int, mode, cval: float = 0.0):
+    """Read(x, y) of the virtually expanded image; returns (value, undefined)."""
+    img, stride = _img(img, np.float32)
+    und = ctypes.c_int(0)
+    v = _load().oracle_read_f32(_ptr(img), img.shape[1], img.shape[0], stride, int(x), int(y),
+                                _mode(mode), float(cval), ctypes.byref(und))
+    return v, bool(und.value)
+
+
+def closeness_mask(sigma_d: float, size_x: int, size_y: int | None = None) -> np.ndarray:
+    """Eq. (1) closeness mask, row-major (yf outer), float64."""
+    size_y = size_x if size_y is None else size_y
+    out = np.empty((size_y, size_x), np.float64)
+    _load().oracle_closeness_mask(float(sigma_d), size_x, size_y, _ptr(out))
+    return out
+
+
+def gaussian_mask(size: int):
+    """Binomial Gaussian mask (int32, size x size) and its shift k (sum = 2^k)."""
+    out = np.empty((size, size), np.int32)
+    k = _load().oracle_gaussian_mask_int(size, _ptr(out))
+    if k < 0:
+        raise ValueError("bad Gaussian size %d" % size)
+    return out, k
+
+
+def sobel_mask(direction: int) -> np.ndarray:
+    out = np.empty((3, 3), np.int32)
+    _load().oracle_sobel_mask_int(int(direction), _ptr(out))
+    return out
+
+
+def convolve_f32(img, mask, mode, cval=0.0, rows=None):
+    """Correlation of a float32 image with a float64 mask; returns (out f64, valid)."""
+    img, stride = _img(img, np.float32)
+    mask = np.ascontiguousarray(mask, np.float64)
+    H, W = img.shape
+    y0, y1 = (0, H) if rows is None else rows
+    out = np.empty((y1 - y0, W), np.float64)
+    valid = np.empty((y1 - y0, W), np.uint8)
+    _load().oracle_convolve_f32(_ptr(img), W, H, stride, _ptr(mask), mask.shape[1],
+                                mask.shape[0], _mode(mode), float(cval), y0, y1,
+                                _ptr(out), _ptr(valid))
+    return out, valid.astype(bool)
+
+
+def convolve_f32_points(img, mask, mode, xs, ys, cval=0.0):
+    img, stride = _img(img, np.float32)
+    mask = np.ascontiguousarray(mask, np.float64)
+    xs = np.ascontiguousarray(xs, np.int64)
+    ys = np.ascontiguousarray(ys, np.int64)
+    out = np.empty(len(xs), np.float64)
+    valid = np.empty(len(xs), np.uint8)
+    _load().oracle_convolve_f32_points(_ptr(img), img.shape[1], img.shape[0], stride,
+                                       _ptr(mask), mask.shape[1], mask.shape[0], _mode(mode),
+                                       float(cval), _ptr(xs), _ptr(ys), len(xs), _ptr(out),
+                                       _ptr(valid))
+    return out, valid.astype(bool)
+
+
+def convolve_u8_sum(img, mask, mode, cval=0, rows=None):
+    """Exact integer sums S of an uint8 image with an int32 mask; (S int64, valid)."""
+    img, stride = _img(img, np.uint8)
+    mask = np.ascontiguousarray(mask, np.int32)
+    H, W = img.shape
+    y0, y1 = (0, H) if rows is None else rows
+    out = np.empty((y1 - y0, W), np.int64)
+    valid = np.empty((y1 - y0, W), np.uint8)
+    _load().oracle_convolve_u8_sum(_ptr(img), W, H, stride, _ptr(mask), mask.shape[1],
+                                   mask.shape[0], _mode(mode), int(cval), y0, y1,
+                                   _ptr(out), _ptr(valid))
+    return out, valid.astype(bool)
+
+
+def convolve_u8_sum_points(img, mask, mode, xs, ys, cval=0):
+    img, stride = _img(img, np.uint8)
+    mask = np.ascontiguousarray(mask, np.int32)
+    xs = np.ascontiguousarray(xs, np.int64)
+    ys = np.ascontiguousarray(ys, np.int64)
+    out = np.empty(len(xs), np.int64)
+    valid = np.empty(len(xs), np.uint8)
+    _load().oracle_convolve_u8_sum_points(_ptr(img), img.shape[1], img.shape[0], stride,
+                                          _ptr(mask), mask.shape[1], mask.shape[0],
+                                          _mode(mode), int(cval), _ptr(xs), _ptr(ys), len(xs),
+                                          _ptr(out), _ptr(valid))
+    return out, valid.astype(bool)
+
+
+def quantize(S, shift: int, to_u8: bool):
+    """(S + 2^(k-1)) >> k, saturated to [0,255] for u8 outputs (reading c12)."""
+    lib = _load()
+    f = np.vectorize(lambda s: lib.oracle_quantize(int(s), int(shift), int(bool(to_u8))),
+                     otypes=[np.int64])
+    return f(np.asarray(S, np.int64))
+
+
+def convolve_u8(img, mask, shift, mode, cval=0, out_dtype=np.uint8, rows=None):
+    """Full integer local operator: sums, then quantisation to u8 or i32."""
+    S, valid = convolve_u8_sum(img, mask, mode, cval, rows)
+    q = quantize(S, shift, out_dtype == np.uint8)
+    return q.astype(out_dtype), valid
+
+
+def bilateral_f32(img, sigma_d, sigma_r, mode, cval=0.0, size=None, cmask=None, rows=None):
+    """Bilateral filter (Alg. 1) of a float32 image; returns (out f64, valid).
+
+    ``cmask`` None -> closeness from Eq. (1) per tap with window ``size``
+    (default 4*sigma_d+1, PAPER.md L325 / Listing 3); else the given mask
+    (Listing 5: c = CMask(xf, yf)).
+    """
+    img, stride = _img(img, np.float32)
+    H, W = img.shape
+    if cmask is not None:
+        cmask = np.ascontiguousarray(cmask, np.float64)
+        mh, mw = cmask.shape
+        cptr = _ptr(cmask)
+    else:
+        if size is None:
+            size = int(round(4 * sigma_d)) + 1
+        mw, mh = (size, size) if isinstance(size, int) else size
+        cptr = None
+    y0, y1 = (0, H) if rows is None else rows
+    out = np.empty((y1 - y0, W), np.float64)
+    valid = np.empty((y1 - y0, W), np.uint8)
+    _load().oracle_bilateral_f32(_ptr(img), W, H, stride, cptr, mw, mh, float(sigma_d),
+                                 float(sigma_r), _mode(mode), float(cval), y0, y1,
+                                 _ptr(out), _ptr(valid))
+    return out, valid.astype(bool)
+
+
+def bilateral_f32_points(img, sigma_d, sigma_r, mode, xs, ys, cval=0.0, size=None, cmask=None):
+    img, stride = _img(img, np.float32)
+    if cmask is not None:
+        cmask = np.ascontiguousarray(cmask, np.float64)
+        mh, mw = cmask.shape
+        cptr = _ptr(cmask)
+    else:
+        if size is None:
+            size = int(round(4 * sigma_d)) + 1
+        mw, mh = (size, size) if isinstance(size, int) else size
+        cptr = None
+    xs = np.ascontiguousarray(xs, np.int64)
+    ys = np.ascontiguousarray(ys, np.int64)
+    out = np.empty(len(xs), np.float64)
+    valid = np.empty(len(xs), np.uint8)
+    _load().oracle_bilateral_f32_points(_ptr(img), img.shape[1], img.shape[0], stride, cptr,
+                                        mw, mh, float(sigma_d), float(sigma_r), _mode(mode),
+                                        float(cval), _ptr(xs), _ptr(ys), len(xs), _ptr(out),
+                                        _ptr(valid))
+    return out, valid.astype(bool)

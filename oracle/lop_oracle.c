@@ -1,0 +1,327 @@
+/*
+ * lop_oracle.c -- plain, slow, obviously-correct CPU ORACLE for the local
+ * operators of Membarth et al., "Generating Device-specific GPU Code for Local
+ * Operators in Medical Imaging", IPDPS 2012.
+ *
+ *   *** TEST INFRASTRUCTURE ONLY. ***
+ *   Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline /
+ *   --impl reference legs may load this library.  The product path
+ *   (paper_conf_ipps_membarthhtke12_b200/) never calls it, shares no code,
+ *   header, table or constant with it, and neither side includes the other.
+ *
+ * Arithmetic: IEEE double throughout (the paper fixes no precision for the
+ * reference semantics; the GPU path is f32 and is compared within 1e-5).
+ * Integer (u8) operators: exact int64 sums.
+ * No blocking, fusion or reordering: every output is the brute-force double
+ * loop of Algorithm 1 in its stated order (yf outer,
+ * xf inner).  OpenMP only distributes independent output rows over cores.
+ *
+ * Citations are PAPER.md line numbers ("Lnnn"); readings of ambiguous
+ * passages are the ones listed in DESIGN.md section "Readings" (= SURVEY §8(c)).
+ *
+ * Parity pins: see tests/test_oracle_pins.py.  Every function below is pinned
+ * by at least one test against something other than itself (Fig. 2 golden
+ * cells, np.pad / scipy.ndimage library routines, the paper's printed mask
+ * value 0.018316, closed-form invariants, hand-computed worked examples).
+ */
+#include <math.h>
+#include <stdint.h>
+#include <stdlib.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+/* Boundary handling modes, Table I.  Numbering is part
+ * of the test interface only. */
+enum { OR_UNDEFINED = 0, OR_CLAMP = 1, OR_REPEAT = 2, OR_MIRROR = 3, OR_CONSTANT = 4 };
+
+int oracle_num_threads(void)
+{
+#ifdef _OPENMP
+    return omp_get_max_threads();
+#else
+    return 1;
+#endif
+}
+
+/*
+ * Per-axis index adjustment, PAPER.md L340-L357 ("adjusting the index of the
+ * accessed pixel to a pixel that resides within the image"), Table I and
+ * Fig. 2 (L359-L432).  Returns the in-image index, or -1 when the access is
+ * out of bounds and the mode does not remap (Constant, Undefined).
+ *   clamp : last valid pixel within image               (Fig. 2c)
+ *   repeat: image repeated at the border (true modulo)   (Fig. 2b, reading c7)
+ *   mirror: mirrored at the border, edge pixel repeated  (Fig. 2d edges, reading c6)
+ */
+int64_t oracle_map_index(int64_t i, int64_t n, int mode)
+{
+    if (i >= 0 && i < n)
+        return i;
+    switch (mode) {
+    case OR_CLAMP:
+        return i < 0 ? 0 : n - 1;
+    case OR_REPEAT: {
+        int64_t q = i % n;
+        if (q < 0) q += n;
+        return q;
+    }
+    case OR_MIRROR: {
+        int64_t period = 2 * n;
+        int64_t q = i % period;
+        if (q < 0) q += period;
+        return q < n ? q : period - 1 - q;
+    }
+    default: /* OR_CONSTANT, OR_UNDEFINED */
+        return -1;
+    }
+}
+
+/*
+ * Read(x', y') of the virtually expanded image:
+ * in range -> the pixel; out of range -> Constant: the user constant
+ * (Table I; reading c8: if either axis is out of bounds), Clamp/Repeat/
+ * Mirror: the pixel at the per-axis adjusted indices; Undefined: not
+ * specified (L295) -> *undef is set and the value must not be used.
+ */
+static double read_f32(const float *img, int64_t W, int64_t H, int64_t stride,
+                       int64_t x, int64_t y, int mode, double cval, int *undef)
+{
+    if (x >= 0 && x < W && y >= 0 && y < H)
+        return (double)img[y * stride + x];
+    if (mode == OR_CONSTANT)
+        return cval;
+    if (mode == OR_UNDEFINED) {
+        *undef = 1;
+        return 0.0;
+    }
+    int64_t mx = oracle_map_index(x, W, mode);
+    int64_t my = oracle_map_index(y, H, mode);
+    return (double)img[my * stride + mx];
+}
+
+static int64_t read_u8(const uint8_t *img, int64_t W, int64_t H, int64_t stride,
+                       int64_t x, int64_t y, int mode, int64_t cval, int *undef)
+{
+    if (x >= 0 && x < W && y >= 0 && y < H)
+        return (int64_t)img[y * stride + x];
+    if (mode == OR_CONSTANT)
+        return cval;
+    if (mode == OR_UNDEFINED) {
+        *undef = 1;
+        return 0;
+    }
+    int64_t mx = oracle_map_index(x, W, mode);
+    int64_t my = oracle_map_index(y, H, mode);
+    return (int64_t)img[my * stride + mx];
+}
+
+/* The same Read() applied to one output of a 4x4 (or any) test image, exported
+ * so the Fig. 2 golden cells can be checked cell by cell. */
+double oracle_read_f32(const float *img, int64_t W, int64_t H, int64_t stride,
+                       int64_t x, int64_t y, int mode, double cval, int *undef)
+{
+    *undef = 0;
+    return read_f32(img, W, H, stride, x, y, mode, cval, undef);
+}
+
+/*
+ * Closeness, Eq. (1) (reading c2):
+ *   closeness((x,y),(x',y')) = exp(-1/2 * (||(x,y)-(x',y')|| / sigma_d)^2)
+ * Mask layout (reading c4): row-major, yf outer, first element (-m,-n);
+ * Listing 4 (L364-L372) stores it as Mask<float> CMask(4*sigma_d+1, ...).
+ */
+void oracle_closeness_mask(double sigma_d, int mw, int mh, double *mask)
+{
+    int m = mw / 2, n = mh / 2;
+    for (int yf = -n; yf <= n; ++yf)
+        for (int xf = -m; xf <= m; ++xf) {
+            double dist = sqrt((double)(xf * xf + yf * yf));
+            mask[(yf + n) * mw + (xf + m)] = exp(-0.5 * (dist / sigma_d) * (dist / sigma_d));
+        }
+}
+
+/* Binomial Gaussian masks (reading c11): outer product of row n of Pascal's
+ * triangle with itself; returns the normalising shift k (sum = 2^k). */
+int oracle_gaussian_mask_int(int size, int32_t *mask)
+{
+    int64_t row[64];
+    if (size < 1 || size > 63 || (size % 2) == 0)
+        return -1;
+    row[0] = 1;
+    for (int i = 1; i < size; ++i) {          /* Pascal: row_i from row_{i-1} */
+        row[i] = 0;
+        for (int j = i; j >= 1; --j)
+            row[j] = row[j] + row[j - 1];
+    }
+    for (int y = 0; y < size; ++y)
+        for (int x = 0; x < size; ++x)
+            mask[y * size + x] = (int32_t)(row[y] * row[x]);
+    return 2 * (size - 1);
+}
+
+/* Sobel 3x3 (reading c12): dir 0 = x-gradient [[-1,0,1],[-2,0,2],[-1,0,1]]
+ * (correlation, reading c5); dir 1 = its transpose (y-gradient). */
+void oracle_sobel_mask_int(int dir, int32_t *mask)
+{
+    static const int32_t smooth[3] = {1, 2, 1};
+    static const int32_t deriv[3] = {-1, 0, 1};
+    for (int y = 0; y < 3; ++y)
+        for (int x = 0; x < 3; ++x)
+            mask[y * 3 + x] = dir == 0 ? smooth[y] * deriv[x] : deriv[y] * smooth[x];
+}
+
+/* ------------------------------------------------------------------ */
+/* Local operator: convolution with a filter mask (PAPER.md L274-L282:  */
+/* window (2m+1)x(2n+1), mask centred at [0,0]; Listing 5 / Listing 9  */
+/* multiply Mask(xf,yf) by Input(xf,yf): correlation, reading c5).     */
+/* ------------------------------------------------------------------ */
+
+static double conv_px_f32(const float *img, int64_t W, int64_t H, int64_t stride,
+                          const double *mask, int mw, int mh, int mode, double cval,
+                          int64_t x, int64_t y, uint8_t *valid)
+{
+    int m = mw / 2, n = mh / 2, undef = 0;
+    double acc = 0.0;
+    for (int yf = -n; yf <= n; ++yf)
+        for (int xf = -m; xf <= m; ++xf)
+            acc += mask[(yf + n) * mw + (xf + m)] *
+                   read_f32(img, W, H, stride, x + xf, y + yf, mode, cval, &undef);
+    *valid = (uint8_t)!undef;
+    return acc;
+}
+
+void oracle_convolve_f32(const float *img, int64_t W, int64_t H, int64_t stride,
+                         const double *mask, int mw, int mh, int mode, double cval,
+                         int64_t y0, int64_t y1, double *out, uint8_t *valid)
+{
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t y = y0; y < y1; ++y)
+        for (int64_t x = 0; x < W; ++x) {
+            int64_t o = (y - y0) * W + x;
+            out[o] = conv_px_f32(img, W, H, stride, mask, mw, mh, mode, cval, x, y, &valid[o]);
+        }
+}
+
+void oracle_convolve_f32_points(const float *img, int64_t W, int64_t H, int64_t stride,
+                                const double *mask, int mw, int mh, int mode, double cval,
+                                const int64_t *xs, const int64_t *ys, int64_t npts,
+                                double *out, uint8_t *valid)
+{
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < npts; ++i)
+        out[i] = conv_px_f32(img, W, H, stride, mask, mw, mh, mode, cval, xs[i], ys[i], &valid[i]);
+}
+
+/* Integer path: exact sum S = sum M(xf,yf) * Read(x+xf, y+yf). */
+static int64_t conv_px_u8(const uint8_t *img, int64_t W, int64_t H, int64_t stride,
+                          const int32_t *mask, int mw, int mh, int mode, int64_t cval,
+                          int64_t x, int64_t y, uint8_t *valid)
+{
+    int m = mw / 2, n = mh / 2, undef = 0;
+    int64_t acc = 0;
+    for (int yf = -n; yf <= n; ++yf)
+        for (int xf = -m; xf <= m; ++xf)
+            acc += (int64_t)mask[(yf + n) * mw + (xf + m)] *
+                   read_u8(img, W, H, stride, x + xf, y + yf, mode, cval, &undef);
+    *valid = (uint8_t)!undef;
+    return acc;
+}
+
+void oracle_convolve_u8_sum(const uint8_t *img, int64_t W, int64_t H, int64_t stride,
+                            const int32_t *mask, int mw, int mh, int mode, int64_t cval,
+                            int64_t y0, int64_t y1, int64_t *out, uint8_t *valid)
+{
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t y = y0; y < y1; ++y)
+        for (int64_t x = 0; x < W; ++x) {
+            int64_t o = (y - y0) * W + x;
+            out[o] = conv_px_u8(img, W, H, stride, mask, mw, mh, mode, cval, x, y, &valid[o]);
+        }
+}
+
+void oracle_convolve_u8_sum_points(const uint8_t *img, int64_t W, int64_t H, int64_t stride,
+                                   const int32_t *mask, int mw, int mh, int mode, int64_t cval,
+                                   const int64_t *xs, const int64_t *ys, int64_t npts,
+                                   int64_t *out, uint8_t *valid)
+{
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < npts; ++i)
+        out[i] = conv_px_u8(img, W, H, stride, mask, mw, mh, mode, cval, xs[i], ys[i], &valid[i]);
+}
+
+/* Output quantisation of the integer sum (reading c12): rounding half-up by
+ * (S + 2^(k-1)) >> k (arithmetic shift = floor), then for u8 outputs
+ * saturation to [0, 255]; i32 outputs keep the shifted value. */
+int64_t oracle_quantize(int64_t S, int shift, int to_u8)
+{
+    int64_t v = S;
+    if (shift > 0) {
+        int64_t num = S + ((int64_t)1 << (shift - 1));
+        /* floor division by 2^shift, valid for negative numerators too */
+        int64_t d = (int64_t)1 << shift;
+        v = num >= 0 ? num / d : -((-num + d - 1) / d);
+    }
+    if (to_u8) {
+        if (v < 0) v = 0;
+        if (v > 255) v = 255;
+    }
+    return v;
+}
+
+/* ------------------------------------------------------------------ */
+/* Bilateral filter, Algorithm 1, Eq. (1)-(2)     */
+/* (L187-L193), Listings 1 and 5 (L204-L265, L379-L416).                */
+/* ------------------------------------------------------------------ */
+
+static double bilateral_px(const float *img, int64_t W, int64_t H, int64_t stride,
+                           const double *cmask, int mw, int mh, double sigma_d,
+                           double sigma_r, int mode, double cval, int64_t x, int64_t y,
+                           uint8_t *valid)
+{
+    int m = mw / 2, n = mh / 2, undef = 0;
+    double center = (double)img[y * stride + x];   /* input[x, y]: always in range */
+    double p = 0.0, k = 0.0;                        /* Alg. 1 line 5 */
+    for (int yf = -n; yf <= n; ++yf)                /* Alg. 1 line 6 */
+        for (int xf = -m; xf <= m; ++xf) {          /* Alg. 1 line 7 */
+            double v = read_f32(img, W, H, stride, x + xf, y + yf, mode, cval, &undef);
+            double c;                               /* Alg. 1 line 8 */
+            if (cmask) {
+                c = cmask[(yf + n) * mw + (xf + m)];   /* Listing 5 l.10: CMask(xf,yf) */
+            } else {
+                double dist = sqrt((double)(xf * xf + yf * yf));
+                c = exp(-0.5 * (dist / sigma_d) * (dist / sigma_d));   /* Eq. (1) */
+            }
+            double dp = fabs(v - center);
+            double s = exp(-0.5 * (dp / sigma_r) * (dp / sigma_r)); /* Eq. (2), Alg. 1 line 9 */
+            k = k + c * s;                          /* Alg. 1 line 10 */
+            p = p + c * s * v;                      /* Alg. 1 line 11 */
+        }
+    *valid = (uint8_t)!undef;
+    return p / k;                                   /* Alg. 1 line 14 */
+}
+
+void oracle_bilateral_f32(const float *img, int64_t W, int64_t H, int64_t stride,
+                          const double *cmask, int mw, int mh, double sigma_d,
+                          double sigma_r, int mode, double cval, int64_t y0, int64_t y1,
+                          double *out, uint8_t *valid)
+{
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t y = y0; y < y1; ++y)
+        for (int64_t x = 0; x < W; ++x) {
+            int64_t o = (y - y0) * W + x;
+            out[o] = bilateral_px(img, W, H, stride, cmask, mw, mh, sigma_d, sigma_r, mode,
+                                  cval, x, y, &valid[o]);
+        }
+}
+
+void oracle_bilateral_f32_points(const float *img, int64_t W, int64_t H, int64_t stride,
+                                 const double *cmask, int mw, int mh, double sigma_d,
+                                 double sigma_r, int mode, double cval,
+                                 const int64_t *xs, const int64_t *ys, int64_t npts,
+                                 double *out, uint8_t *valid)
+{
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < npts; ++i)
+        out[i] = bilateral_px(img, W, H, stride, cmask, mw, mh, sigma_d, sigma_r, mode, cval,
+                              xs[i], ys[i], &valid[i]);
+}
