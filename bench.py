@@ -1,0 +1,507 @@
+#!/usr/bin/env python
+"""bench.py -- throughput of the local-operator hot path on B200.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl lop|reference]
+                    [--workload bilateral4096|frames|bands] [--mode clamp]
+
+One JSON line on rank 0 (driver contract):
+  metric / unit   BASELINE.json's metric, in Mpixel/s
+  value           whole-job Mpixel/s, inputs resident in HBM, CUDA events on
+                  the launching stream, K steps between barrier+synchronize,
+                  max over ranks
+  e2e             the same metric through the host pipeline API
+                  (lop.Pipeline: pinned host in -> device -> pinned host out,
+                  copies inside the timed region)
+  roofline        the dominant kernel against its bound (SFU for the
+                  bilateral filter: 168 ex2 per pixel = (13*13 - 1))
+  cpu_baseline    the C oracle (double, OpenMP) on a bounded sample, rank 0, N=1
+  clocks          nvidia-smi samples taken during the timed region
+  gpu_launches    lop kernel launches inside the timed region (liblop counter)
+
+A step is one pass of the whole hot path over one batch:
+workload bilateral4096 (default, BASELINE config 2 with clamp): every rank
+filters its own 4096x4096 f32 image (13x13, sigma_d=3, sigma_r=5), i.e.
+frame-parallel weak scaling with no data-path collective.
+workload frames (config 4): 1024 frames of 1024^2 split over the ranks.
+workload bands (config 5): one 32768^2 image in row bands, NCCL halo exchange.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+BASELINE_METRIC = "Mpixel/s per filter at 1/2/4/8 B200; % of HBM GB/s or FP32/SFU roofline"
+SM_COUNT = 148
+MUFU_PER_CLK_PER_SM = 16          # MUFU.EX2 lanes per clock per SM on sm_100
+
+
+def parse(argv=None):
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", choices=["lop", "reference"], default="lop")
+    ap.add_argument("--workload", choices=["bilateral4096", "frames", "bands"],
+                    default="bilateral4096")
+    ap.add_argument("--mode", default="clamp")
+    ap.add_argument("--no-extras", action="store_true", help="skip per-filter side measurements")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=10)
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    return ap.parse_args(argv)
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        d["_source"] = "measured (MEASURED_PEAKS.json)"
+        return d
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "sm_max_mhz": 1965.0,
+            "_source": "fallback (B200_PROFILING.md)"}
+
+
+# ------------------------------------------------------------ distributed ----
+
+class Dist:
+    def __init__(self):
+        self.world = int(os.environ.get("WORLD_SIZE", "1"))
+        self.rank = int(os.environ.get("RANK", "0"))
+        self.local = int(os.environ.get("LOCAL_RANK", "0"))
+        self.pg = None
+
+    def init(self, backend="nccl"):
+        import torch
+        import torch.distributed as dist
+        if self.world > 1 and not dist.is_initialized():
+            if backend == "nccl":
+                torch.cuda.set_device(self.local)
+            dist.init_process_group(backend, device_id=(torch.device("cuda", self.local)
+                                                        if backend == "nccl" else None))
+            self.pg = dist.group.WORLD
+
+    def barrier(self):
+        if self.world > 1:
+            import torch.distributed as dist
+            dist.barrier()
+
+    def max(self, v: float) -> float:
+        if self.world == 1:
+            return v
+        import torch
+        import torch.distributed as dist
+        t = torch.tensor([v], dtype=torch.float64,
+                         device="cuda" if torch.cuda.is_available() else "cpu")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def close(self):
+        if self.world > 1:
+            import torch.distributed as dist
+            if dist.is_initialized():
+                dist.destroy_process_group()
+
+
+# ----------------------------------------------------------------- clocks ----
+
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.proc = None
+        self.path = None
+
+    def start(self):
+        try:
+            fd, self.path = tempfile.mkstemp(suffix=".csv")
+            os.close(fd)
+            self.fh = open(self.path, "w")
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), "--query-gpu=" + self.FIELDS,
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=self.fh, stderr=subprocess.DEVNULL)
+        except (OSError, FileNotFoundError):
+            self.proc = None
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        self.fh.close()
+        sm, smax, power, reasons = [], [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        with open(self.path) as f:
+            for line in f:
+                parts = [p.strip() for p in line.split(",")]
+                if len(parts) < 9:
+                    continue
+                try:
+                    sm.append(float(parts[1]))
+                    smax.append(float(parts[2]))
+                    power.append(float(parts[3]))
+                except ValueError:
+                    continue
+                for n, v in zip(names, parts[5:9]):
+                    if v.lower().startswith("active"):
+                        reasons.add(n)
+        os.unlink(self.path)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(smax) if smax else None,
+                "power_w_max": max(power) if power else None,
+                "samples": len(sm), "reasons": sorted(reasons)}
+
+
+# ------------------------------------------------------------------ timing ----
+
+def time_steps(step, K, W, dist, stream):
+    """W warm-up steps, then K timed steps bracketed by barrier + synchronize;
+    returns (total_ms max over ranks, per-launch ms list on this rank)."""
+    import torch
+    for i in range(W):
+        step(i)
+    torch.cuda.synchronize()
+    dist.barrier()
+    torch.cuda.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(K)]
+    t0 = torch.cuda.Event(enable_timing=True)
+    t1 = torch.cuda.Event(enable_timing=True)
+    t0.record(stream)
+    for i in range(K):
+        ev[i][0].record(stream)
+        step(i)
+        ev[i][1].record(stream)
+    t1.record(stream)
+    torch.cuda.synchronize()
+    dist.barrier()
+    torch.cuda.synchronize()
+    total = t0.elapsed_time(t1)
+    per = [a.elapsed_time(b) for a, b in ev]
+    return dist.max(total), per
+
+
+def flush_l2(buf):
+    buf.add_(1)          # write 512 MiB: evicts the 126 MB L2
+
+
+# --------------------------------------------------------------- workloads ----
+
+def run_lop(args, dist, peaks):
+    import torch
+    import numpy as np
+    import synthetic
+    import paper_conf_ipps_membarthhtke12_b200 as lop
+
+    dev = torch.device("cuda", dist.local)
+    torch.cuda.set_device(dev)
+    stream = torch.cuda.current_stream(dev)
+    K, W = args.steps, max(3, args.warmup)
+    sigma_d, sigma_r, size = 3.0, 5.0, 13
+    taps = size * size - 1                     # algorithmic ex2 per pixel
+    result = {}
+
+    if args.workload == "bilateral4096":
+        H = Wd = 4096
+        n_sets = 3                             # rotating sets: 3 x 128 MiB > 126 MB L2
+        seed = synthetic.config_seed(2) + 7919 * dist.rank
+        base = synthetic.angio(H, Wd, seed=seed, device=dev)
+        ins = [base.clone() for _ in range(n_sets)]
+        outs = [torch.empty_like(base) for _ in range(n_sets)]
+        px_per_step_rank = H * Wd
+
+        def step(i):
+            lop.bilateral(ins[i % n_sets], sigma_d, sigma_r, args.mode, size=size,
+                          out=outs[i % n_sets], stream=stream)
+        config = {"workload": "bilateral 4096x4096 f32, 13x13 (sigma_d=3), sigma_r=5, %s; "
+                              "one image per rank per step (BASELINE config 2)" % args.mode,
+                  "height": H, "width": Wd, "window": size, "sigma_d": sigma_d,
+                  "sigma_r": sigma_r, "boundary": args.mode,
+                  "l2": "rotating %d input/output sets (%d MiB) > 126 MB L2" %
+                        (n_sets, n_sets * 128),
+                  "parallelism": "frame-parallel x%d (independent images)" % dist.world}
+        scaling = "weak"
+    elif args.workload == "frames":
+        F, S = 1024, 1024
+        lo, hi = F * dist.rank // dist.world, F * (dist.rank + 1) // dist.world
+        frames = synthetic.angio_frames(F, S, S, seed=synthetic.config_seed(4), first=lo,
+                                        count=hi - lo, device=dev)
+        out = torch.empty_like(frames)
+        px_per_step_rank = (hi - lo) * S * S
+
+        def step(i):
+            lop.bilateral(frames, sigma_d, sigma_r, args.mode, size=size, out=out, stream=stream)
+        config = {"workload": "1024 frames x 1024^2 f32 bilateral 13x13 %s, frame-parallel "
+                              "(BASELINE config 4)" % args.mode,
+                  "frames": F, "frame_size": S, "window": size, "boundary": args.mode,
+                  "l2": "inputs (4 GiB / N) larger than L2",
+                  "parallelism": "frame-parallel x%d" % dist.world}
+        scaling = "strong"
+    else:
+        from paper_conf_ipps_membarthhtke12_b200 import dist as ldist
+        GHt = GW = 32768
+        band = ldist.Bands(GHt, GW, dist.world, dist.rank, halo=size // 2, device=dev,
+                           mode=args.mode)
+        band.fill(lambda y0, y1: synthetic.angio(GHt, GW, seed=synthetic.config_seed(5),
+                                                 device=dev, row_range=(y0, y1)))
+        out = torch.empty_like(band.owned)
+        px_per_step_rank = band.rows * GW
+
+        def step(i):
+            band.exchange()
+            lop.bilateral(band.owned, sigma_d, sigma_r, args.mode, size=size, out=out,
+                          stream=stream, band=band.band_args())
+        config = {"workload": "32768^2 f32 bilateral 13x13 %s, row bands + NCCL halo exchange "
+                              "(BASELINE config 5)" % args.mode,
+                  "height": GHt, "width": GW, "window": size, "boundary": args.mode,
+                  "l2": "inputs (4 GiB / N) larger than L2",
+                  "parallelism": "row-bands x%d" % dist.world}
+        scaling = "strong"
+
+    clocks = ClockSampler(dist.local)
+    clocks.start()
+    lop.reset_launch_count()
+    total_ms, per = time_steps(step, K, W, dist, stream)
+    launches = lop.launch_count() - W * (1 if args.workload != "bands" else 1)
+    # keep the GPU busy a little longer so the sampler sees the clocks under load
+    t_end = time.time() + max(0.0, 1.0 - total_ms / 1000.0)
+    i = 0
+    while time.time() < t_end:
+        step(i)
+        i += 1
+        if i % 20 == 0:
+            torch.cuda.synchronize()
+    torch.cuda.synchronize()
+    clk = clocks.stop()
+
+    px_total = px_per_step_rank * dist.world * K
+    value = px_total / (total_ms / 1000.0) / 1e6
+    avg_launch_ms = sum(per) / len(per)
+    ex2_per_launch = taps * px_per_step_rank
+    achieved = ex2_per_launch / (avg_launch_ms / 1000.0) / 1e12
+    sm_mhz_peak = float(peaks.get("sm_max_mhz", 1965.0))
+    peak = SM_COUNT * MUFU_PER_CLK_PER_SM * sm_mhz_peak * 1e6 / 1e12
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        with open(tp) as f:
+            traffic = json.load(f).get("bilateral_tiled_13x13_4096", None)
+    roofline = {"bound": "alu", "kernel": "lop::bilateral_tiled_kernel<6>",
+                "achieved": round(achieved, 4), "peak": round(peak, 4), "unit": "Tex2/s",
+                "frac": round(achieved / peak, 4), "traffic": traffic,
+                "work_per_launch": "%d ex2 (= 168 per px x %d px)" % (ex2_per_launch,
+                                                                      px_per_step_rank),
+                "peak_basis": "148 SM x 16 MUFU.EX2/clk x %.0f MHz (sm_max_mhz, %s)" %
+                              (sm_mhz_peak, peaks["_source"]),
+                "avg_launch_ms": round(avg_launch_ms, 5)}
+    result.update(dict(metric=BASELINE_METRIC, value=round(value, 2), unit="Mpixel/s",
+                       n_gpus=dist.world, steps=K, warmup=W,
+                       ms_per_step=round(total_ms / K, 5), higher_is_better=True,
+                       scaling=scaling, vs_baseline=None, dtype="f32", data="synthetic",
+                       config=config, roofline=roofline, clocks=clk, gpu_launches=int(launches)))
+
+    # ---- e2e through the host pipeline API (rank-local, max over ranks)
+    if args.workload == "bilateral4096" and args.e2e_steps > 0:
+        H = Wd = 4096
+        host_in = base.cpu().pin_memory()
+        host_out = torch.empty_like(host_in).pin_memory()
+        pipe = lop.Pipeline(Wd, H, device=dist.local, chunk_rows=256)
+        for _ in range(2):
+            pipe.bilateral(host_in, host_out, sigma_d, sigma_r, args.mode, size=size)
+        dist.barrier()
+        t0 = time.perf_counter()
+        for _ in range(args.e2e_steps):
+            pipe.bilateral(host_in, host_out, sigma_d, sigma_r, args.mode, size=size)
+        t = dist.max(time.perf_counter() - t0)
+        pipe.close()
+        chunks = math.ceil(H / 256)
+        halo_rows = 2 * (size // 2) * (chunks - 1)
+        result["e2e"] = {"value": round(H * Wd * dist.world * args.e2e_steps / t / 1e6, 2),
+                         "unit": "Mpixel/s", "h2d_bytes_per_step": (H + halo_rows) * Wd * 4,
+                         "d2h_bytes_per_step": H * Wd * 4,
+                         "api": "lop.Pipeline.bilateral (lop_pipeline_bilateral), pinned host "
+                                "buffers, 256-row chunks on 3 streams, wall clock"}
+    if not args.no_extras and dist.world == 1 and args.workload == "bilateral4096":
+        result["filters"] = extras(lop, synthetic, dev, stream, peaks)
+    return result
+
+
+def extras(lop, synthetic, dev, stream, peaks):
+    """Per-filter side measurements (L2 flushed between iterations for the
+    memory-bound ones): mode sweep of the bilateral (E5), Gaussian 5x5 and
+    Sobel 3x3 on 4096^2 f32 / u8 (config 3), config 1 (256^2) via CUDA graph."""
+    import torch
+    out = {}
+    H = Wd = 4096
+    img = synthetic.angio(H, Wd, seed=synthetic.config_seed(2), device=dev)
+    res = torch.empty_like(img)
+    flush = torch.empty(128 * 1024 * 1024, dtype=torch.float32, device=dev)
+
+    def timed(fn, n, do_flush):
+        for _ in range(3):
+            fn()
+        ts = []
+        for _ in range(n):
+            if do_flush:
+                flush_l2(flush)
+            a = torch.cuda.Event(enable_timing=True)
+            b = torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            fn()
+            b.record(stream)
+            torch.cuda.synchronize()
+            ts.append(a.elapsed_time(b))
+        return statistics.median(ts)
+
+    modes = {}
+    for mode in ("undefined", "clamp", "repeat", "mirror", "constant"):
+        ms = timed(lambda: lop.bilateral(img, 3.0, 5.0, mode, size=13, out=res, stream=stream),
+                   10, False)
+        modes[mode] = round(H * Wd / ms / 1e3, 1)
+    out["bilateral_13x13_4096_f32_Mpx_s"] = modes
+    v = list(modes.values())
+    out["bilateral_mode_spread"] = round(max(v) / min(v) - 1.0, 4)
+    hbm = float(peaks.get("hbm_gbs", 6650.0))
+    u8 = synthetic.to_u8(img)
+    conv = {}
+    cases = [("gaussian5x5_f32", lambda: lop.gaussian(img, 5, "clamp", out=res, stream=stream), 8),
+             ("sobel3x3_f32", lambda: lop.sobel(img, 0, "clamp", out=res, stream=stream), 8)]
+    u8o = torch.empty_like(u8)
+    i32o = torch.empty(u8.shape, dtype=torch.int32, device=dev)
+    cases += [("gaussian5x5_u8", lambda: lop.gaussian(u8, 5, "clamp", out=u8o, stream=stream), 2),
+              ("sobel3x3_u8_i32", lambda: lop.sobel(u8, 0, "clamp", out=i32o, stream=stream), 5)]
+    for name, fn, bpp in cases:
+        ms = timed(fn, 20, True)
+        gbs = H * Wd * bpp / ms / 1e6
+        conv[name] = {"Mpx_s": round(H * Wd / ms / 1e3, 1), "ms": round(ms, 4),
+                      "GB_s": round(gbs, 1), "hbm_frac": round(gbs / hbm, 3),
+                      "bytes_per_px": bpp}
+    out["conv_4096_l2_flushed"] = conv
+    # config 1: 256^2, 3x3, sigma_d = 1, sigma_r = 5, clamp -- launch-latency bound:
+    # report CUDA-graph replays of 100 launches
+    small = synthetic.angio(256, 256, seed=synthetic.config_seed(1), device=dev)
+    so = torch.empty_like(small)
+    g = torch.cuda.CUDAGraph()
+    s2 = torch.cuda.Stream(dev)
+    s2.wait_stream(stream)
+    with torch.cuda.stream(s2):
+        lop.bilateral(small, 1.0, 5.0, "clamp", size=3, out=so, stream=s2)
+        with torch.cuda.graph(g, stream=s2):
+            for _ in range(100):
+                lop.bilateral(small, 1.0, 5.0, "clamp", size=3, out=so, stream=s2)
+    stream.wait_stream(s2)
+    ms = timed(lambda: g.replay(), 10, False)
+    out["config1_bilateral_256_3x3_graph_Mpx_s"] = round(256 * 256 * 100 / ms / 1e3, 1)
+    return out
+
+
+# ------------------------------------------------------------ CPU oracle ----
+
+def cpu_oracle_rate(H, Wd, seconds, rows_per_chunk=None, mode="clamp"):
+    """Time the C oracle (as it stands) on rows of the config-2 image until
+    `seconds` elapse; returns (Mpixel/s, rows, cores)."""
+    import oracle
+    import synthetic
+    img = synthetic.angio(H, Wd, seed=synthetic.config_seed(2)).numpy()
+    cores = oracle.num_threads()
+    rows_per_chunk = rows_per_chunk or max(1, cores)
+    done, t_used = 0, 0.0
+    while done < H and t_used < seconds:
+        r1 = min(H, done + rows_per_chunk)
+        t0 = time.perf_counter()
+        oracle.bilateral_f32(img, 3.0, 5.0, mode, size=13, rows=(done, r1))
+        t_used += time.perf_counter() - t0
+        done = r1
+    return done * Wd / t_used / 1e6, done, cores, t_used
+
+
+def run_reference(args, dist):
+    """--impl reference: the oracle timed on the host cores (rank 0 only)."""
+    if dist.rank != 0:
+        return None
+    import oracle
+    oracle.build()
+    H = Wd = 4096
+    K, W = args.steps, max(3, args.warmup)
+    per_step = max(0.5, min(5.0, 150.0 / (K + W)))
+    import synthetic
+    img = synthetic.angio(H, Wd, seed=synthetic.config_seed(2)).numpy()
+    cores = oracle.num_threads()
+    t0 = time.perf_counter()
+    oracle.bilateral_f32(img, 3.0, 5.0, args.mode, size=13, rows=(0, 1))
+    t_row = time.perf_counter() - t0
+    rows = max(1, min(H, int(per_step / max(t_row, 1e-6))))
+    y = 0
+
+    def step():
+        nonlocal y
+        y0 = y % (H - rows + 1) if rows < H else 0
+        oracle.bilateral_f32(img, 3.0, 5.0, args.mode, size=13, rows=(y0, y0 + rows))
+        y += rows
+    for _ in range(W):
+        step()
+    t0 = time.perf_counter()
+    for _ in range(K):
+        step()
+    t = time.perf_counter() - t0
+    value = rows * Wd * K / t / 1e6
+    sample = ("%d rows x 4096 px of the config-2 image per step (of 4096 rows), "
+              "13x13, sigma_d=3, sigma_r=5, %s" % (rows, args.mode))
+    return dict(metric=BASELINE_METRIC, value=round(value, 4), unit="Mpixel/s", n_gpus=args.gpus,
+                steps=K, warmup=W, ms_per_step=round(t / K * 1000, 3), higher_is_better=True,
+                scaling="weak", vs_baseline=None, dtype="f64", data="synthetic", impl="reference",
+                config={"workload": "bilateral 4096x4096 f32 input, 13x13 (sigma_d=3), "
+                                    "sigma_r=5, %s (BASELINE config 2), C oracle" % args.mode,
+                        "parallelism": "OpenMP over rows, %d threads" % cores},
+                cpu_baseline={"value": round(value, 4), "unit": "Mpixel/s", "cores": cores,
+                              "kind": "oracle", "sample": sample},
+                e2e={"value": round(value, 4), "unit": "Mpixel/s", "h2d_bytes_per_step": 0,
+                     "d2h_bytes_per_step": 0})
+
+
+def main(argv=None):
+    args = parse(argv)
+    dist = Dist()
+    if args.impl == "reference":
+        if dist.rank == 0:
+            line = run_reference(args, dist)
+            print(json.dumps(line), flush=True)
+        return 0
+    import torch
+    if not torch.cuda.is_available():
+        print(json.dumps({"error": "bench.py needs a CUDA device (no CPU fallback)"}))
+        return 1
+    dist.init("nccl")
+    peaks = load_peaks()
+    res = run_lop(args, dist, peaks)
+    if dist.rank == 0:
+        if dist.world == 1 and not args.no_cpu_baseline:
+            v, rows, cores, t = cpu_oracle_rate(4096, 4096, args.cpu_seconds, mode=args.mode)
+            res["cpu_baseline"] = {"value": round(v, 4), "unit": "Mpixel/s", "cores": cores,
+                                   "kind": "oracle",
+                                   "sample": "first %d rows of the 4096x4096 config-2 image "
+                                             "(%.1f s of CPU time), same filter" % (rows, t)}
+        print(json.dumps(res), flush=True)
+    dist.close()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

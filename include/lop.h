@@ -1,0 +1,215 @@
+/*
+ * lop.h -- C ABI of the B200-native local-operator library ("lop").
+ *
+ * The calls mirror the problem statement of Membarth, Hannig, Teich, Koerner,
+ * Eckert, "Generating Device-specific GPU Code for Local Operators in Medical
+ * Imaging", IPDPS 2012 (cited as PAPER.md line numbers "Lnnn"):
+ *
+ *   Image             lop_image               (§II; Listing 2 l.8-9)
+ *   IterationSpace    lop_iteration_space     (§II; Listing 2 l.15)
+ *   BoundaryCondition lop_boundary_condition  (§III-A; Listing 3)
+ *   Accessor          lop_accessor            (§II; L315-L318)
+ *   Mask              lop_mask                (§III-B; Listing 4)
+ *   Kernel::execute   lop_bilateral_execute / lop_convolve_execute
+ *                                             (Listing 2 l.21-24; Listing 5)
+ *
+ * Conventions (all entry points):
+ *   - Ownership: the caller owns every host and device buffer.  The library
+ *     never allocates on the execute path; mask coefficients are copied into
+ *     the kernel's parameter block at the call, so the caller may free them on
+ *     return (no __constant__ symbol, no global device state).
+ *     The host pipeline (lop_pipeline_*) owns the device staging buffers it
+ *     allocates in lop_pipeline_create and frees in lop_pipeline_destroy.
+ *   - Asynchrony: execute calls enqueue work on `cuda_stream` (a cudaStream_t,
+ *     NULL = legacy default stream) and return without synchronising.
+ *   - Errors: every function returns a lop_status.  Invalid arguments return
+ *     LOP_ERR_INVALID before anything is launched; launch failures return
+ *     LOP_ERR_CUDA.  lop_last_error() returns a thread-local message for the
+ *     last non-OK status of the calling thread.  No C++ exception crosses
+ *     this ABI.
+ *   - Layout: images are row-major; row y of frame b starts at
+ *     (char*)data + b*batch_stride_bytes + y*stride_bytes.  Rows must be
+ *     addressable for y in [-halo_top, height + halo_bottom).
+ *   - Index types: coordinates are int32, byte offsets int64 (a 32768^2 f32
+ *     image is 4 GiB).
+ */
+#ifndef LOP_H
+#define LOP_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define LOP_VERSION 100 /* 1.0.0 */
+
+typedef enum {
+    LOP_OK = 0,
+    LOP_ERR_INVALID = -1,     /* argument validation failed; nothing launched */
+    LOP_ERR_UNSUPPORTED = -2, /* valid request outside what this build supports */
+    LOP_ERR_CUDA = -3         /* CUDA runtime error (message has cudaGetErrorString) */
+} lop_status;
+
+/* Pixel types (Image<T>, L150-L154).  Bilateral: F32 -> F32 (Kernel<float>,
+ * Listing 1).  Convolution: F32 -> F32, U8 -> U8, U8 -> I32 (reading c12). */
+typedef enum { LOP_U8 = 0, LOP_I32 = 1, LOP_F32 = 2 } lop_dtype;
+
+/* Boundary handling modes, Table I (L290-L299), Fig. 2 (L359-L432):
+ *   UNDEFINED  out-of-bounds reads are not specified: outputs whose window
+ *              leaves the image are unspecified, but the library stays
+ *              memory-safe (it never reads outside the image);
+ *   CLAMP      last valid pixel within the image;
+ *   REPEAT     image repeated periodically (true modulo, any distance);
+ *   MIRROR     mirrored at the border with the edge pixel repeated
+ *              (c b a | a b c d | d c b), periodic with period 2N;
+ *   CONSTANT   user-defined constant (lop_boundary_condition.constant) if
+ *              either coordinate is out of bounds.
+ * Index adjustment is per axis (L340-L357). */
+typedef enum {
+    LOP_UNDEFINED = 0,
+    LOP_CLAMP = 1,
+    LOP_REPEAT = 2,
+    LOP_MIRROR = 3,
+    LOP_CONSTANT = 4
+} lop_boundary;
+
+/* Image<T> (L150-L154): non-owning view of device memory.
+ * A single image has batch = 1, halo_top = halo_bottom = 0, global_y0 = 0,
+ * global_height = height (0 is accepted as "= height").
+ * Frame sequences (config C4): batch = F frames, batch_stride_bytes apart.
+ * Row bands (config C5): the view owns global rows
+ *   [global_y0, global_y0 + height) of a global_height-row image and may read
+ *   halo_top rows above / halo_bottom rows below it (filled by the caller,
+ *   e.g. by the NCCL halo exchange).  Boundary modes always use the global
+ *   image extent (reading c10).  A halo row that lies outside the global image
+ *   is read as stored (this is how a REPEAT ring halo is supplied). */
+typedef struct {
+    void *data;                 /* device pointer to pixel (0, 0) of the first owned row */
+    int32_t width, height;      /* owned columns / rows */
+    int64_t stride_bytes;       /* row pitch, >= width * elem_size */
+    int32_t dtype;              /* lop_dtype */
+    int32_t batch;              /* frames, >= 1 */
+    int64_t batch_stride_bytes; /* distance between frames (ignored if batch == 1) */
+    int32_t halo_top, halo_bottom;
+    int32_t global_y0, global_height;
+} lop_image;
+
+/* BoundaryCondition<T>(image, size_x, size_y, mode[, constant]) (Listing 3,
+ * L331-L338; L329-L330).  size_x/size_y: the window of the local operator,
+ * odd (L274-L282). constant: used by LOP_CONSTANT; for U8 images it must be
+ * an integer in [0, 255]. */
+typedef struct {
+    lop_image image;
+    int32_t mode;               /* lop_boundary */
+    int32_t size_x, size_y;
+    double constant;
+} lop_boundary_condition;
+
+/* Accessor<T> (L160-L162, L315-L318): a view of an input through a
+ * BoundaryCondition; allocates nothing.  Input(xf, yf) of output (x, y) reads
+ * input pixel (x + offset_x + xf, y + offset_y + yf). */
+typedef struct {
+    const lop_boundary_condition *bc;
+    int32_t offset_x, offset_y;
+} lop_accessor;
+
+/* Mask<T>(size_x, size_y) (Listing 4): HOST pointer to
+ * size_y * size_x coefficients, row-major, yf outer, first element at
+ * (xf, yf) = (-m, -n) (reading c4).  dtype F32 (float coefficients) or I32
+ * (integer coefficients for U8 images).  shift: for integer masks, the output
+ * is (S + 2^(shift-1)) >> shift (reading c12); 0 for float masks. */
+typedef struct {
+    int32_t size_x, size_y;
+    int32_t dtype;              /* LOP_F32 or LOP_I32 */
+    const void *coeffs;         /* host memory, copied at the call */
+    int32_t shift;
+} lop_mask;
+
+/* IterationSpace<T> (L155-L157): rectangular region of interest of the output
+ * image; every point is one output pixel (1:1 work items, L168-L171).
+ * width/height 0 = the whole output image. */
+typedef struct {
+    lop_image image;
+    int32_t x0, y0, width, height;
+} lop_iteration_space;
+
+/* Bilateral filter (Alg. 1, Eq. 1-2, Listing 5):
+ *   out(x,y) = sum c(xf,yf) s(I(x+xf,y+yf) - I(x,y)) I(x+xf,y+yf)
+ *            / sum c(xf,yf) s(I(x+xf,y+yf) - I(x,y))
+ *   s(d) = exp(-d^2 / (2 sigma_r^2)),
+ *   c = closeness mask (coefficients > 0 required, centre > 0) or, if
+ *       closeness == NULL, c = exp(-(xf^2 + yf^2) / (2 sigma_d^2)) over the
+ *       BoundaryCondition's size_x x size_y window (Eq. 1).
+ * Input and output: LOP_F32, same width/height/batch.
+ * Window: odd, up to 63 x 63 (13 x 13 is the paper's 4*sigma_d+1 for
+ * sigma_d = 3).  sigma_r > 0, sigma_d > 0 when closeness == NULL. */
+lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                 const lop_mask *closeness, float sigma_d, float sigma_r,
+                                 void *cuda_stream);
+
+/* Local operator with a filter mask (L274-L282, Listing 5 / Listing 9):
+ *   S(x,y) = sum_{yf,xf} M(xf,yf) * Read(x+xf, y+yf)   (correlation, reading c5)
+ * F32 -> F32 with an F32 mask: out = S.
+ * U8 -> U8 with an I32 mask: out = clamp((S + 2^(k-1)) >> k, 0, 255), k = shift.
+ * U8 -> I32 with an I32 mask: out = (S + 2^(k-1)) >> k (k = 0: out = S).
+ * Window: odd, up to 63 x 63; mask size must equal the BoundaryCondition's. */
+lop_status lop_convolve_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                const lop_mask *mask, void *cuda_stream);
+
+/* Mask builders (host only).
+ * lop_mask_closeness: Eq. (1), float coefficients (Listing 4's mask[]).
+ * lop_mask_gaussian:  binomial size x size (size odd; 1..11 for LOP_I32, 1..31
+ *                     for LOP_F32); LOP_I32 writes integers and
+ *                     *shift = 2*(size-1); LOP_F32 writes
+ *                     the normalised floats and *shift = 0 (reading c11).
+ * lop_mask_sobel:     3x3 Sobel, dir 0 = d/dx [[-1,0,1],[-2,0,2],[-1,0,1]],
+ *                     dir 1 = d/dy (transpose); dtype LOP_I32 or LOP_F32. */
+lop_status lop_mask_closeness(float sigma_d, int32_t size_x, int32_t size_y, float *out);
+lop_status lop_mask_gaussian(int32_t size, int32_t dtype, void *out, int32_t *shift);
+lop_status lop_mask_sobel(int32_t dir, int32_t dtype, void *out);
+
+/* Kernel selection (process-wide; for tests and the tuning sweep):
+ *   LOP_VARIANT_AUTO    tiled shared-memory kernels where a template instance
+ *                       exists, generic otherwise (default);
+ *   LOP_VARIANT_GENERIC one-thread-per-pixel kernel with per-tap remapping;
+ *   LOP_VARIANT_TILED   force the tiled kernel (LOP_ERR_UNSUPPORTED if none). */
+typedef enum { LOP_VARIANT_AUTO = 0, LOP_VARIANT_GENERIC = 1, LOP_VARIANT_TILED = 2 } lop_variant;
+lop_status lop_set_variant(int32_t variant);
+int32_t lop_get_variant(void);
+
+/* Number of kernel launches issued by this thread since the last reset
+ * (bench.py's "gpu_launches" evidence). */
+int64_t lop_launch_count(void);
+void lop_reset_launch_count(void);
+
+/* Thread-local message for the last non-OK status ("" if none). */
+const char *lop_last_error(void);
+int32_t lop_version(void);
+
+/* ---- Host pipeline (Listing 2 flow: IN = host_in; execute(); getData()) ----
+ * End-to-end execution from pageable or pinned HOST buffers: the image is cut
+ * into row chunks of `chunk_rows` rows; chunk i+1 is copied host->device while
+ * chunk i is filtered and chunk i-1 copied device->host, on separate streams
+ * of `device`.  Halo rows for the window are uploaded with each chunk.  The
+ * pipeline allocates its device staging buffers once at create time (sized
+ * for width x height x max window 63) and frees them at destroy.
+ * The call returns after the result is in host_out (synchronous). */
+typedef struct lop_pipeline lop_pipeline;
+
+lop_status lop_pipeline_create(int32_t device, int32_t width, int32_t height,
+                               int32_t chunk_rows, lop_pipeline **out);
+lop_status lop_pipeline_bilateral(lop_pipeline *p, const float *host_in, int64_t in_stride_bytes,
+                                  float *host_out, int64_t out_stride_bytes, int32_t mode,
+                                  double constant, int32_t size_x, int32_t size_y,
+                                  const lop_mask *closeness, float sigma_d, float sigma_r);
+lop_status lop_pipeline_convolve(lop_pipeline *p, const void *host_in, int32_t in_dtype,
+                                 int64_t in_stride_bytes, void *host_out, int32_t out_dtype,
+                                 int64_t out_stride_bytes, int32_t mode, double constant,
+                                 const lop_mask *mask);
+lop_status lop_pipeline_destroy(lop_pipeline *p);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* LOP_H */

@@ -1,0 +1,287 @@
+"""B200-native local operators (HIPAcc, Membarth et al., IPDPS 2012).
+
+Thin Python binding over the C ABI in ``include/lop.h`` (``liblop.so``):
+argument marshalling only -- every pixel is computed by the sm_100a kernels
+in ``csrc/``.  PyTorch provides device memory, streams and process groups.
+There is no CPU fallback: the functions raise on non-CUDA tensors, and
+importing this package raises if ``liblop.so`` has not been built.
+
+Paper objects -> this API (PAPER.md line numbers):
+  Image (L150-L154)              a CUDA tensor (H, W) or (B, H, W), rows contiguous
+  IterationSpace (L155-L157)     ``roi=(x0, y0, w, h)`` (default: whole image)
+  BoundaryCondition (Listing 3)  ``mode=``, ``constant=``, window ``size=``
+  Accessor (L160-L162)           ``offset=(dx, dy)``
+  Mask (Listing 4)               ``mask=`` (host array), ``closeness_mask()``,
+                                 ``gaussian_mask()``, ``sobel_mask()``
+  Kernel::execute (Listing 2)    ``bilateral()``, ``convolve()``, ``gaussian()``,
+                                 ``sobel()``
+"""
+from __future__ import annotations
+
+import ctypes
+
+import numpy as np
+import torch
+
+from . import _lib
+from ._lib import LopError
+
+lib = _lib.load()
+
+MODES = {"undefined": _lib.LOP_UNDEFINED, "clamp": _lib.LOP_CLAMP, "repeat": _lib.LOP_REPEAT,
+         "mirror": _lib.LOP_MIRROR, "constant": _lib.LOP_CONSTANT}
+_DT = {torch.uint8: _lib.LOP_U8, torch.int32: _lib.LOP_I32, torch.float32: _lib.LOP_F32}
+VARIANTS = {"auto": _lib.LOP_VARIANT_AUTO, "generic": _lib.LOP_VARIANT_GENERIC,
+            "tiled": _lib.LOP_VARIANT_TILED}
+
+__all__ = ["bilateral", "convolve", "gaussian", "sobel", "closeness_mask", "gaussian_mask",
+           "sobel_mask", "set_variant", "get_variant", "launch_count", "reset_launch_count",
+           "Pipeline", "LopError", "image_view", "MODES", "library_path"]
+
+
+def library_path() -> str:
+    return _lib.LIB_PATH
+
+
+def _check(status: int):
+    if status != _lib.LOP_OK:
+        raise LopError(status, lib.lop_last_error().decode())
+
+
+def _mode(mode) -> int:
+    if isinstance(mode, str):
+        return MODES[mode]
+    return int(mode)
+
+
+def image_view(t: torch.Tensor, halo_top: int = 0, halo_bottom: int = 0, global_y0: int = 0,
+               global_height: int = 0) -> _lib.lop_image:
+    """lop_image over a CUDA tensor (H, W) or (B, H, W) whose rows are contiguous.
+
+    For band views, ``t`` covers the OWNED rows; ``halo_top``/``halo_bottom``
+    rows directly above/below in the same storage are readable by the kernel.
+    """
+    if not t.is_cuda:
+        raise TypeError("lop operates on CUDA tensors only (no CPU fallback)")
+    if t.dtype not in _DT:
+        raise TypeError("unsupported dtype %s" % t.dtype)
+    if t.dim() == 2:
+        b, (h, w) = 1, t.shape
+        bstride = 0
+    elif t.dim() == 3:
+        b, h, w = t.shape
+        bstride = t.stride(0) * t.element_size()
+    else:
+        raise ValueError("expected (H, W) or (B, H, W)")
+    if t.stride(-1) != 1:
+        raise ValueError("rows must be contiguous (stride(-1) == 1)")
+    im = _lib.lop_image()
+    im.data = t.data_ptr()
+    im.width, im.height = int(w), int(h)
+    im.stride_bytes = t.stride(-2) * t.element_size()
+    im.dtype = _DT[t.dtype]
+    im.batch = int(b)
+    im.batch_stride_bytes = int(bstride)
+    im.halo_top, im.halo_bottom = int(halo_top), int(halo_bottom)
+    im.global_y0, im.global_height = int(global_y0), int(global_height)
+    return im
+
+
+def _stream_handle(t: torch.Tensor, stream):
+    if stream is None:
+        stream = torch.cuda.current_stream(t.device)
+    return stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream)
+
+
+def _host_mask(mask, dtype) -> tuple[np.ndarray, _lib.lop_mask]:
+    arr = np.ascontiguousarray(np.asarray(mask.cpu() if torch.is_tensor(mask) else mask),
+                               dtype=np.float32 if dtype == _lib.LOP_F32 else np.int32)
+    if arr.ndim != 2:
+        raise ValueError("mask must be 2D (size_y, size_x)")
+    m = _lib.lop_mask()
+    m.size_y, m.size_x = arr.shape
+    m.dtype = dtype
+    m.coeffs = arr.ctypes.data
+    m.shift = 0
+    return arr, m
+
+
+def _execute(kind, x, out, mode, constant, size_xy, roi, offset, stream, band, call):
+    halo_top, halo_bottom, gy0, gh = band
+    in_im = image_view(x, halo_top, halo_bottom, gy0, gh)
+    out_im = image_view(out, 0, 0, gy0, gh)
+    bc = _lib.lop_boundary_condition()
+    bc.image = in_im
+    bc.mode = _mode(mode)
+    bc.size_x, bc.size_y = size_xy
+    bc.constant = float(constant)
+    acc = _lib.lop_accessor(ctypes.pointer(bc), int(offset[0]), int(offset[1]))
+    is_ = _lib.lop_iteration_space()
+    is_.image = out_im
+    if roi is not None:
+        is_.x0, is_.y0, is_.width, is_.height = (int(v) for v in roi)
+    with torch.cuda.device(x.device):
+        _check(call(ctypes.byref(is_), ctypes.byref(acc), _stream_handle(x, stream)))
+    return out
+
+
+def bilateral(x: torch.Tensor, sigma_d: float, sigma_r: float, mode="clamp", constant=0.0,
+              size=None, mask=None, out=None, roi=None, offset=(0, 0), stream=None,
+              band=(0, 0, 0, 0)) -> torch.Tensor:
+    """Bilateral filter (Alg. 1, Listing 5) of a float32 CUDA image.
+
+    size: window (odd int or (sx, sy)); default 4*sigma_d+1.
+    mask: optional host closeness mask (size_y, size_x); default Eq. (1).
+    band: (halo_top, halo_bottom, global_y0, global_height) for row-band views.
+    """
+    if mask is not None:
+        marr, m = _host_mask(mask, _lib.LOP_F32)
+        size_xy = (m.size_x, m.size_y)
+        mptr = ctypes.byref(m)
+    else:
+        marr, mptr = None, None
+        if size is None:
+            size = int(round(4 * sigma_d)) + 1
+        size_xy = (size, size) if isinstance(size, int) else tuple(size)
+    if out is None:
+        out = torch.empty_like(x)
+    return _execute("bilateral", x, out, mode, constant, size_xy, roi, offset, stream, band,
+                    lambda is_, acc, s: lib.lop_bilateral_execute(is_, acc, mptr, float(sigma_d),
+                                                                  float(sigma_r), s))
+
+
+def convolve(x: torch.Tensor, mask, mode="clamp", constant=0.0, shift=0, out=None,
+             out_dtype=None, roi=None, offset=(0, 0), stream=None,
+             band=(0, 0, 0, 0)) -> torch.Tensor:
+    """Local operator with a filter mask (correlation, Listing 5 / Listing 9).
+
+    float32 image: float mask, out float32.  uint8 image: integer mask,
+    out uint8 (default, rounded (S + 2^(k-1)) >> k, saturated) or int32.
+    """
+    mdt = _lib.LOP_F32 if x.dtype == torch.float32 else _lib.LOP_I32
+    marr, m = _host_mask(mask, mdt)
+    m.shift = int(shift)
+    if out is None:
+        out = torch.empty(x.shape, dtype=out_dtype or x.dtype, device=x.device)
+    return _execute("convolve", x, out, mode, constant, (m.size_x, m.size_y), roi, offset,
+                    stream, band,
+                    lambda is_, acc, s: lib.lop_convolve_execute(is_, acc, ctypes.byref(m), s))
+
+
+def gaussian(x: torch.Tensor, size: int = 5, mode="clamp", constant=0.0, **kw) -> torch.Tensor:
+    """Binomial Gaussian (Tables VIII-IX; reading c11): f32 -> f32, u8 -> u8."""
+    if x.dtype == torch.float32:
+        m, _ = gaussian_mask(size, np.float32)
+        return convolve(x, m, mode, constant, **kw)
+    m, k = gaussian_mask(size, np.int32)
+    return convolve(x, m, mode, constant, shift=k, **kw)
+
+
+def sobel(x: torch.Tensor, direction: int = 0, mode="clamp", constant=0.0, **kw) -> torch.Tensor:
+    """Sobel 3x3 (L847-L849): f32 -> f32, u8 -> int32 (reading c12)."""
+    if x.dtype == torch.float32:
+        return convolve(x, sobel_mask(direction, np.float32), mode, constant, **kw)
+    kw.setdefault("out_dtype", torch.int32)
+    return convolve(x, sobel_mask(direction, np.int32), mode, constant, **kw)
+
+
+# --------------------------------------------------------------- masks ----
+
+def closeness_mask(sigma_d: float, size_x: int | None = None, size_y: int | None = None):
+    """Eq. (1) closeness coefficients as Listing 4's float mask[] (yf outer)."""
+    size_x = int(round(4 * sigma_d)) + 1 if size_x is None else size_x
+    size_y = size_x if size_y is None else size_y
+    out = np.empty((size_y, size_x), np.float32)
+    _check(lib.lop_mask_closeness(float(sigma_d), size_x, size_y, out.ctypes.data))
+    return out
+
+
+def gaussian_mask(size: int, dtype=np.int32):
+    out = np.empty((size, size), dtype)
+    k = ctypes.c_int32(0)
+    _check(lib.lop_mask_gaussian(size, _lib.LOP_I32 if dtype == np.int32 else _lib.LOP_F32,
+                                 out.ctypes.data, ctypes.byref(k)))
+    return out, k.value
+
+
+def sobel_mask(direction: int = 0, dtype=np.int32):
+    out = np.empty((3, 3), dtype)
+    _check(lib.lop_mask_sobel(direction, _lib.LOP_I32 if dtype == np.int32 else _lib.LOP_F32,
+                              out.ctypes.data))
+    return out
+
+
+# ------------------------------------------------------------ runtime ----
+
+def set_variant(name: str):
+    _check(lib.lop_set_variant(VARIANTS[name]))
+
+
+def get_variant() -> str:
+    v = lib.lop_get_variant()
+    return {k: n for n, k in VARIANTS.items()}[v]
+
+
+def launch_count() -> int:
+    return int(lib.lop_launch_count())
+
+
+def reset_launch_count():
+    lib.lop_reset_launch_count()
+
+
+class Pipeline:
+    """End-to-end filtering of HOST images (Listing 2 flow) with overlapped
+    chunked H2D / kernel / D2H on three CUDA streams (csrc/pipeline.cpp)."""
+
+    def __init__(self, width: int, height: int, device: int = 0, chunk_rows: int = 512):
+        h = ctypes.c_void_p()
+        _check(lib.lop_pipeline_create(int(device), int(width), int(height), int(chunk_rows),
+                                       ctypes.byref(h)))
+        self._h = h
+        self.width, self.height = width, height
+
+    def close(self):
+        if self._h:
+            lib.lop_pipeline_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    @staticmethod
+    def _host(t: torch.Tensor):
+        if t.is_cuda or t.stride(-1) != 1 or t.dim() != 2:
+            raise ValueError("pipeline needs a 2D host tensor with contiguous rows")
+        return t.data_ptr(), t.stride(0) * t.element_size()
+
+    def bilateral(self, host_in: torch.Tensor, host_out: torch.Tensor, sigma_d: float,
+                  sigma_r: float, mode="clamp", constant=0.0, size=None, mask=None):
+        ip, istr = self._host(host_in)
+        op, ostr = self._host(host_out)
+        if mask is not None:
+            marr, m = _host_mask(mask, _lib.LOP_F32)
+            sx, sy, mptr = m.size_x, m.size_y, ctypes.byref(m)
+        else:
+            size = int(round(4 * sigma_d)) + 1 if size is None else size
+            sx, sy = (size, size) if isinstance(size, int) else size
+            mptr = None
+        _check(lib.lop_pipeline_bilateral(self._h, ip, istr, op, ostr, _mode(mode),
+                                          float(constant), sx, sy, mptr, float(sigma_d),
+                                          float(sigma_r)))
+        return host_out
+
+    def convolve(self, host_in: torch.Tensor, host_out: torch.Tensor, mask, mode="clamp",
+                 constant=0.0, shift=0):
+        ip, istr = self._host(host_in)
+        op, ostr = self._host(host_out)
+        mdt = _lib.LOP_F32 if host_in.dtype == torch.float32 else _lib.LOP_I32
+        marr, m = _host_mask(mask, mdt)
+        m.shift = int(shift)
+        _check(lib.lop_pipeline_convolve(self._h, ip, _DT[host_in.dtype], istr, op,
+                                         _DT[host_out.dtype], ostr, _mode(mode),
+                                         float(constant), ctypes.byref(m)))
+        return host_out

@@ -1,0 +1,91 @@
+"""ctypes declarations of include/lop.h (argument marshalling only).
+
+Loads the in-tree ``liblop.so`` built by ``build.py``.  There is no fallback:
+if the library is missing or cannot be loaded, importing the package raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(PKG, "liblop.so")
+
+LOP_OK, LOP_ERR_INVALID, LOP_ERR_UNSUPPORTED, LOP_ERR_CUDA = 0, -1, -2, -3
+LOP_U8, LOP_I32, LOP_F32 = 0, 1, 2
+LOP_UNDEFINED, LOP_CLAMP, LOP_REPEAT, LOP_MIRROR, LOP_CONSTANT = 0, 1, 2, 3, 4
+LOP_VARIANT_AUTO, LOP_VARIANT_GENERIC, LOP_VARIANT_TILED = 0, 1, 2
+
+c_i32, c_i64, c_dbl, c_flt, c_vp = (ctypes.c_int32, ctypes.c_int64, ctypes.c_double,
+                                    ctypes.c_float, ctypes.c_void_p)
+
+
+class lop_image(ctypes.Structure):
+    _fields_ = [("data", c_vp), ("width", c_i32), ("height", c_i32),
+                ("stride_bytes", c_i64), ("dtype", c_i32), ("batch", c_i32),
+                ("batch_stride_bytes", c_i64), ("halo_top", c_i32), ("halo_bottom", c_i32),
+                ("global_y0", c_i32), ("global_height", c_i32)]
+
+
+class lop_boundary_condition(ctypes.Structure):
+    _fields_ = [("image", lop_image), ("mode", c_i32), ("size_x", c_i32), ("size_y", c_i32),
+                ("constant", c_dbl)]
+
+
+class lop_accessor(ctypes.Structure):
+    _fields_ = [("bc", ctypes.POINTER(lop_boundary_condition)), ("offset_x", c_i32),
+                ("offset_y", c_i32)]
+
+
+class lop_mask(ctypes.Structure):
+    _fields_ = [("size_x", c_i32), ("size_y", c_i32), ("dtype", c_i32), ("coeffs", c_vp),
+                ("shift", c_i32)]
+
+
+class lop_iteration_space(ctypes.Structure):
+    _fields_ = [("image", lop_image), ("x0", c_i32), ("y0", c_i32), ("width", c_i32),
+                ("height", c_i32)]
+
+
+# name -> (restype, argtypes); every symbol include/lop.h declares
+SIGNATURES = {
+    "lop_bilateral_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
+                                      ctypes.POINTER(lop_accessor), ctypes.POINTER(lop_mask),
+                                      c_flt, c_flt, c_vp]),
+    "lop_convolve_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
+                                     ctypes.POINTER(lop_accessor), ctypes.POINTER(lop_mask),
+                                     c_vp]),
+    "lop_mask_closeness": (c_i32, [c_flt, c_i32, c_i32, c_vp]),
+    "lop_mask_gaussian": (c_i32, [c_i32, c_i32, c_vp, ctypes.POINTER(c_i32)]),
+    "lop_mask_sobel": (c_i32, [c_i32, c_i32, c_vp]),
+    "lop_set_variant": (c_i32, [c_i32]),
+    "lop_get_variant": (c_i32, []),
+    "lop_launch_count": (c_i64, []),
+    "lop_reset_launch_count": (None, []),
+    "lop_last_error": (ctypes.c_char_p, []),
+    "lop_version": (c_i32, []),
+    "lop_pipeline_create": (c_i32, [c_i32, c_i32, c_i32, c_i32, ctypes.POINTER(c_vp)]),
+    "lop_pipeline_bilateral": (c_i32, [c_vp, c_vp, c_i64, c_vp, c_i64, c_i32, c_dbl, c_i32,
+                                       c_i32, ctypes.POINTER(lop_mask), c_flt, c_flt]),
+    "lop_pipeline_convolve": (c_i32, [c_vp, c_vp, c_i32, c_i64, c_vp, c_i32, c_i64, c_i32,
+                                      c_dbl, ctypes.POINTER(lop_mask)]),
+    "lop_pipeline_destroy": (c_i32, [c_vp]),
+}
+
+
+class LopError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__("lop status %d: %s" % (status, msg))
+        self.status = status
+
+
+def load(path: str = LIB_PATH) -> ctypes.CDLL:
+    if not os.path.exists(path):
+        raise ImportError("liblop.so not built (%s); run "
+                          "`python -m paper_conf_ipps_membarthhtke12_b200.build`" % path)
+    lib = ctypes.CDLL(path)
+    for name, (res, args) in SIGNATURES.items():
+        fn = getattr(lib, name)
+        fn.restype = res
+        fn.argtypes = args
+    return lib

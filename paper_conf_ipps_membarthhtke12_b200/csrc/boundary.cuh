@@ -1,0 +1,112 @@
+// boundary.cuh -- boundary handling by index adjustment (PAPER.md L340-L357,
+// Table I, Fig. 2) and the per-tap arithmetic shared by
+// every kernel variant, so that the generic and tiled kernels produce
+// bit-identical outputs (the same instruction sequence per tap, in the same
+// yf-major / xf-minor order as Algorithm 1).
+#pragma once
+#include <stdint.h>
+
+#include "lop_params.h"
+
+namespace lop {
+
+enum { M_UNDEFINED = 0, M_CLAMP = 1, M_REPEAT = 2, M_MIRROR = 3, M_CONSTANT = 4 };
+
+// Per-axis index adjustment of i into [0, n).  UNDEFINED is served as CLAMP
+// so that the kernels never read outside the image (reading c9).
+__device__ __forceinline__ int map_axis(int i, int n, int mode)
+{
+    if ((unsigned)i < (unsigned)n) return i;
+    if (mode == M_REPEAT) {
+        int q = i % n;
+        return q < 0 ? q + n : q;
+    }
+    if (mode == M_MIRROR) {
+        int period = 2 * n;
+        int q = i % period;
+        if (q < 0) q += period;
+        return q < n ? q : period - 1 - q;
+    }
+    return i < 0 ? 0 : n - 1;
+}
+
+// Resolve a band-local input row iy (global row iy + gy0) to the band-local
+// row that is physically read; returns false for a CONSTANT read.
+//  * rows inside the global image are read where they are stored (own rows
+//    or halo rows, which the host validated to be present);
+//  * out-of-image rows under REPEAT that are physically present are a ring
+//    halo supplied by the neighbour band: read as stored;
+//  * otherwise the global row is adjusted per mode (Table I).
+__device__ __forceinline__ bool resolve_row(int iy, const Geom &g, int mode, int &row)
+{
+    const int gy = iy + g.gy0;
+    if ((unsigned)gy < (unsigned)g.GH) { row = iy; return true; }
+    if (mode == M_CONSTANT) return false;
+    if (mode == M_REPEAT && iy >= -g.halo_top && iy < g.H + g.halo_bottom) { row = iy; return true; }
+    row = map_axis(gy, g.GH, mode) - g.gy0;
+    return true;
+}
+
+__device__ __forceinline__ bool resolve_col(int ix, const Geom &g, int mode, int &col)
+{
+    if ((unsigned)ix < (unsigned)g.W) { col = ix; return true; }
+    if (mode == M_CONSTANT) return false;
+    col = map_axis(ix, g.W, mode);
+    return true;
+}
+
+template <typename T>
+__device__ __forceinline__ const T *row_ptr(const Geom &g, int b, int row)
+{
+    return reinterpret_cast<const T *>(g.data + (int64_t)b * g.bstride + (int64_t)row * g.stride);
+}
+
+// Read(ix, iy) of frame b with boundary handling (generic, per tap).
+__device__ __forceinline__ float read_f32(const Geom &g, int b, int ix, int iy, int mode, float cval)
+{
+    int row, col;
+    if (!resolve_row(iy, g, mode, row) || !resolve_col(ix, g, mode, col)) return cval;
+    return __ldg(row_ptr<float>(g, b, row) + col);
+}
+
+__device__ __forceinline__ int read_u8(const Geom &g, int b, int ix, int iy, int mode, int cval)
+{
+    int row, col;
+    if (!resolve_row(iy, g, mode, row) || !resolve_col(ix, g, mode, col)) return cval;
+    return (int)__ldg(row_ptr<uint8_t>(g, b, row) + col);
+}
+
+__device__ __forceinline__ float ex2_approx(float x)
+{
+    float y;
+    asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+
+// One bilateral tap (Alg. 1 lines 8-11 / Listing 5 l.7-12) in the log2 domain:
+//   w = c(xf,yf) * exp(-(v - centre)^2 / (2 sigma_r^2))
+//     = ex2(lc + nk * (v - centre)^2),  lc = log2 c,  nk = -log2(e)/(2 sigma_r^2)
+//   d += w;  p += w * v
+// Explicit _rn intrinsics: never contracted or reassociated by the compiler.
+__device__ __forceinline__ void bilateral_tap(float v, float centre, float lc, float nk,
+                                              float &d, float &p)
+{
+    const float diff = __fsub_rn(v, centre);
+    const float t = __fmul_rn(diff, diff);
+    const float w = ex2_approx(__fmaf_rn(t, nk, lc));
+    d = __fadd_rn(d, w);
+    p = __fmaf_rn(w, v, p);
+}
+
+__device__ __forceinline__ float bilateral_finish(float d, float p)
+{
+    return __fdiv_rn(p, d);   // Alg. 1 line 14: output = p / k
+}
+
+// Integer output quantisation (reading c12): (S + 2^(k-1)) >> k, arithmetic.
+__device__ __forceinline__ int quantize_shift(int s, int shift)
+{
+    return shift > 0 ? (s + (1 << (shift - 1))) >> shift : s;
+}
+
+}  // namespace lop

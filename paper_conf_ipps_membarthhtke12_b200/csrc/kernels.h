@@ -1,0 +1,17 @@
+// kernels.h -- launchers implemented in the .cu files, called by lop_api.cpp.
+#pragma once
+#include <cuda_runtime.h>
+
+#include "lop_params.h"
+
+namespace lop {
+
+cudaError_t launch_bilateral_generic(const BilateralGeneric &p, cudaStream_t stream);
+cudaError_t launch_bilateral_tiled(const BilateralTiled &p, cudaStream_t stream);
+cudaError_t launch_conv_generic(const ConvGeneric &p, cudaStream_t stream);
+// Tiled convolution; returns cudaErrorNotSupported when no instance matches
+// (the caller then falls back to the generic kernel).
+cudaError_t launch_conv_tiled(const ConvGeneric &p, cudaStream_t stream);
+bool conv_tiled_supported(const ConvGeneric &p);
+
+}  // namespace lop

@@ -1,0 +1,395 @@
+// lop_api.cpp -- the C ABI (include/lop.h): argument validation, mask
+// construction, kernel dispatch.  Host C++ only; every pixel of every step of
+// the path is computed by the CUDA kernels in *.cu.
+#include "lop.h"
+
+#include <cuda_runtime.h>
+
+#include <atomic>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <memory>
+#include <string>
+
+#include "kernels.h"
+#include "lop_params.h"
+
+namespace {
+
+thread_local std::string g_error;
+thread_local int64_t g_launches = 0;
+std::atomic<int32_t> g_variant{LOP_VARIANT_AUTO};
+
+lop_status fail(lop_status st, const char *fmt, ...)
+{
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_error = buf;
+    return st;
+}
+
+lop_status cuda_fail(cudaError_t e, const char *what)
+{
+    return fail(LOP_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+int elem_size(int32_t dt)
+{
+    switch (dt) {
+    case LOP_U8: return 1;
+    case LOP_I32: return 4;
+    case LOP_F32: return 4;
+    default: return 0;
+    }
+}
+
+const double kLog2e = 1.4426950408889634073599246810019;
+
+// ---------------------------------------------------------------- validation
+lop_status check_image(const lop_image &im, const char *name)
+{
+    if (!im.data) return fail(LOP_ERR_INVALID, "%s: data is NULL", name);
+    const int es = elem_size(im.dtype);
+    if (!es) return fail(LOP_ERR_INVALID, "%s: unknown dtype %d", name, im.dtype);
+    if (im.width <= 0 || im.height <= 0)
+        return fail(LOP_ERR_INVALID, "%s: width/height must be > 0 (got %d x %d)", name, im.width,
+                    im.height);
+    if (im.stride_bytes < (int64_t)im.width * es || im.stride_bytes % es)
+        return fail(LOP_ERR_INVALID, "%s: stride_bytes %lld invalid for width %d", name,
+                    (long long)im.stride_bytes, im.width);
+    if (im.batch < 1) return fail(LOP_ERR_INVALID, "%s: batch must be >= 1", name);
+    if (im.halo_top < 0 || im.halo_bottom < 0)
+        return fail(LOP_ERR_INVALID, "%s: negative halo", name);
+    const int64_t rows = (int64_t)im.height + im.halo_top + im.halo_bottom;
+    if (im.batch > 1 && im.batch_stride_bytes < rows * im.stride_bytes)
+        return fail(LOP_ERR_INVALID, "%s: batch_stride_bytes too small", name);
+    const int32_t gh = im.global_height ? im.global_height : im.height;
+    if (im.global_y0 < 0 || (int64_t)im.global_y0 + im.height > gh)
+        return fail(LOP_ERR_INVALID, "%s: band [%d, %d) outside global height %d", name,
+                    im.global_y0, im.global_y0 + im.height, gh);
+    cudaPointerAttributes attr;
+    cudaError_t e = cudaPointerGetAttributes(&attr, im.data);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(LOP_ERR_INVALID, "%s: data is not a CUDA pointer (%s)", name,
+                    cudaGetErrorString(e));
+    }
+    if (attr.type != cudaMemoryTypeDevice && attr.type != cudaMemoryTypeManaged)
+        return fail(LOP_ERR_INVALID, "%s: data must be device memory", name);
+    int dev = -1;
+    cudaGetDevice(&dev);
+    if (attr.device != dev)
+        return fail(LOP_ERR_INVALID, "%s: data lives on device %d, current device is %d", name,
+                    attr.device, dev);
+    return LOP_OK;
+}
+
+lop::Geom make_geom(const lop_image &im)
+{
+    lop::Geom g;
+    g.data = static_cast<const char *>(im.data);
+    g.stride = im.stride_bytes;
+    g.bstride = im.batch > 1 ? im.batch_stride_bytes : 0;
+    g.W = im.width;
+    g.H = im.height;
+    g.halo_top = im.halo_top;
+    g.halo_bottom = im.halo_bottom;
+    g.gy0 = im.global_y0;
+    g.GH = im.global_height ? im.global_height : im.height;
+    return g;
+}
+
+int map_axis_host(int64_t i, int64_t n, int mode)
+{
+    if (i >= 0 && i < n) return (int)i;
+    if (mode == LOP_REPEAT) { int64_t q = i % n; return (int)(q < 0 ? q + n : q); }
+    if (mode == LOP_MIRROR) {
+        int64_t per = 2 * n, q = i % per;
+        if (q < 0) q += per;
+        return (int)(q < n ? q : per - 1 - q);
+    }
+    return i < 0 ? 0 : (int)(n - 1);
+}
+
+// Every input row the launch can touch must be physically addressable in the
+// band view: same resolution rule as lop::resolve_row (boundary.cuh).
+lop_status check_rows(const lop::Geom &g, int mode, int64_t iy_lo, int64_t iy_hi)
+{
+    for (int64_t iy = iy_lo; iy <= iy_hi; ++iy) {
+        if (iy >= 0 && iy < g.H) continue;
+        const int64_t gy = iy + g.gy0;
+        int64_t row;
+        if (gy >= 0 && gy < g.GH) row = iy;
+        else if (mode == LOP_CONSTANT) continue;
+        else if (mode == LOP_REPEAT && iy >= -g.halo_top && iy < g.H + g.halo_bottom) continue;
+        else row = map_axis_host(gy, g.GH, mode) - g.gy0;
+        if (row < -g.halo_top || row >= g.H + g.halo_bottom)
+            return fail(LOP_ERR_INVALID,
+                        "input row %lld (global %lld) resolves to band row %lld outside the "
+                        "view [-%d, %d): halo too small for the window",
+                        (long long)iy, (long long)gy, (long long)row, g.halo_top,
+                        g.H + g.halo_bottom);
+    }
+    return LOP_OK;
+}
+
+struct Prepared {
+    lop::Common c;
+};
+
+lop_status prepare(const lop_iteration_space *is, const lop_accessor *in, Prepared &pp)
+{
+    if (!is) return fail(LOP_ERR_INVALID, "iteration space is NULL");
+    if (!in || !in->bc) return fail(LOP_ERR_INVALID, "accessor / boundary condition is NULL");
+    const lop_boundary_condition &bc = *in->bc;
+    lop_status st = check_image(bc.image, "input");
+    if (st) return st;
+    st = check_image(is->image, "output");
+    if (st) return st;
+    if (bc.mode < LOP_UNDEFINED || bc.mode > LOP_CONSTANT)
+        return fail(LOP_ERR_INVALID, "unknown boundary mode %d", bc.mode);
+    if (bc.size_x < 1 || bc.size_y < 1 || !(bc.size_x & 1) || !(bc.size_y & 1))
+        return fail(LOP_ERR_INVALID, "window %d x %d must be odd and positive (PAPER.md L274-L282)",
+                    bc.size_x, bc.size_y);
+    if (bc.size_x > 2 * lop::kMaxRadius + 1 || bc.size_y > 2 * lop::kMaxRadius + 1)
+        return fail(LOP_ERR_UNSUPPORTED, "window %d x %d larger than 63 x 63", bc.size_x,
+                    bc.size_y);
+    const lop_image &ii = bc.image, &oi = is->image;
+    if (ii.batch != oi.batch) return fail(LOP_ERR_INVALID, "input/output batch differ");
+    if (ii.width != oi.width || ii.height != oi.height)
+        return fail(LOP_ERR_INVALID, "input %d x %d and output %d x %d differ (Listing 2 l.8-9)",
+                    ii.width, ii.height, oi.width, oi.height);
+    if (!std::isfinite(bc.constant)) return fail(LOP_ERR_INVALID, "constant is not finite");
+    if (ii.dtype == LOP_U8 && bc.mode == LOP_CONSTANT &&
+        (bc.constant < 0 || bc.constant > 255 || bc.constant != std::floor(bc.constant)))
+        return fail(LOP_ERR_INVALID, "constant %g is not a u8 value", bc.constant);
+    lop::Common &c = pp.c;
+    std::memset(&c, 0, sizeof c);
+    c.in = make_geom(ii);
+    c.out.data = static_cast<char *>(oi.data);
+    c.out.stride = oi.stride_bytes;
+    c.out.bstride = oi.batch > 1 ? oi.batch_stride_bytes : 0;
+    c.out.W = oi.width;
+    c.out.H = oi.height;
+    c.roi_x0 = is->x0;
+    c.roi_y0 = is->y0;
+    c.roi_w = is->width ? is->width : oi.width - is->x0;
+    c.roi_h = is->height ? is->height : oi.height - is->y0;
+    if (c.roi_x0 < 0 || c.roi_y0 < 0 || c.roi_w <= 0 || c.roi_h <= 0 ||
+        (int64_t)c.roi_x0 + c.roi_w > oi.width || (int64_t)c.roi_y0 + c.roi_h > oi.height)
+        return fail(LOP_ERR_INVALID, "iteration space [%d,%d)+%dx%d outside the %d x %d output",
+                    is->x0, is->y0, c.roi_w, c.roi_h, oi.width, oi.height);
+    c.off_x = in->offset_x;
+    c.off_y = in->offset_y;
+    c.mode = bc.mode;
+    c.rx = bc.size_x / 2;
+    c.ry = bc.size_y / 2;
+    c.batch = ii.batch;
+    c.cval_f = (float)bc.constant;
+    c.cval_i = (int32_t)bc.constant;
+    return check_rows(c.in, c.mode, (int64_t)c.roi_y0 + c.off_y - c.ry,
+                      (int64_t)c.roi_y0 + c.roi_h - 1 + c.off_y + c.ry);
+}
+
+lop_status launched(cudaError_t e, const char *what)
+{
+    if (e != cudaSuccess) return cuda_fail(e, what);
+    ++g_launches;
+    return LOP_OK;
+}
+
+}  // namespace
+
+namespace lop_detail {
+void set_error(const std::string &msg) { g_error = msg; }
+}  // namespace lop_detail
+
+extern "C" {
+
+const char *lop_last_error(void) { return g_error.c_str(); }
+int32_t lop_version(void) { return LOP_VERSION; }
+int64_t lop_launch_count(void) { return g_launches; }
+void lop_reset_launch_count(void) { g_launches = 0; }
+
+lop_status lop_set_variant(int32_t v)
+{
+    if (v < LOP_VARIANT_AUTO || v > LOP_VARIANT_TILED)
+        return fail(LOP_ERR_INVALID, "unknown variant %d", v);
+    g_variant = v;
+    return LOP_OK;
+}
+int32_t lop_get_variant(void) { return g_variant; }
+
+// ------------------------------------------------------------------ masks
+lop_status lop_mask_closeness(float sigma_d, int32_t size_x, int32_t size_y, float *out)
+{
+    if (!out) return fail(LOP_ERR_INVALID, "out is NULL");
+    if (!(sigma_d > 0) || !std::isfinite(sigma_d)) return fail(LOP_ERR_INVALID, "sigma_d must be > 0");
+    if (size_x < 1 || size_y < 1 || !(size_x & 1) || !(size_y & 1))
+        return fail(LOP_ERR_INVALID, "mask size must be odd");
+    const int m = size_x / 2, n = size_y / 2;
+    const double c_d = 1.0 / (2.0 * (double)sigma_d * (double)sigma_d);  // Listing 1 l.13
+    for (int yf = -n; yf <= n; ++yf)
+        for (int xf = -m; xf <= m; ++xf)
+            out[(yf + n) * size_x + (xf + m)] = (float)std::exp(-c_d * (double)(xf * xf + yf * yf));
+    return LOP_OK;
+}
+
+lop_status lop_mask_gaussian(int32_t size, int32_t dtype, void *out, int32_t *shift)
+{
+    if (!out || !shift) return fail(LOP_ERR_INVALID, "out/shift is NULL");
+    if (size < 1 || size > 31 || !(size & 1)) return fail(LOP_ERR_INVALID, "size must be odd in 1..31");
+    if (dtype != LOP_I32 && dtype != LOP_F32) return fail(LOP_ERR_INVALID, "dtype must be I32 or F32");
+    if (dtype == LOP_I32 && size > 11)   // 255 * 2^(2(size-1)) must fit the int32 sums
+        return fail(LOP_ERR_INVALID, "integer Gaussian masks are limited to 11x11");
+    int64_t binom[32];
+    for (int k = 0; k < size; ++k) {                 // C(size-1, k) via the multiplicative formula
+        int64_t v = 1;
+        for (int j = 1; j <= k; ++j) v = v * (size - j) / j;
+        binom[k] = v;
+    }
+    const int k = 2 * (size - 1);
+    for (int y = 0; y < size; ++y)
+        for (int x = 0; x < size; ++x) {
+            const int64_t v = binom[y] * binom[x];
+            if (dtype == LOP_I32) static_cast<int32_t *>(out)[y * size + x] = (int32_t)v;
+            else static_cast<float *>(out)[y * size + x] = (float)std::ldexp((double)v, -k);
+        }
+    *shift = dtype == LOP_I32 ? k : 0;
+    return LOP_OK;
+}
+
+lop_status lop_mask_sobel(int32_t dir, int32_t dtype, void *out)
+{
+    if (!out) return fail(LOP_ERR_INVALID, "out is NULL");
+    if (dir != 0 && dir != 1) return fail(LOP_ERR_INVALID, "dir must be 0 (x) or 1 (y)");
+    if (dtype != LOP_I32 && dtype != LOP_F32) return fail(LOP_ERR_INVALID, "dtype must be I32 or F32");
+    for (int y = -1; y <= 1; ++y)
+        for (int x = -1; x <= 1; ++x) {
+            const int d = dir == 0 ? x : y, o = dir == 0 ? y : x;   // derivative / smoothing axes
+            const int v = d * (2 - o * o);                           // [-1,0,1] x [1,2,1]
+            if (dtype == LOP_I32) static_cast<int32_t *>(out)[(y + 1) * 3 + x + 1] = v;
+            else static_cast<float *>(out)[(y + 1) * 3 + x + 1] = (float)v;
+        }
+    return LOP_OK;
+}
+
+// -------------------------------------------------------------- bilateral
+lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                 const lop_mask *closeness, float sigma_d, float sigma_r,
+                                 void *cuda_stream)
+{
+    Prepared pp;
+    lop_status st = prepare(is, in, pp);
+    if (st) return st;
+    const lop::Common &c = pp.c;
+    if (in->bc->image.dtype != LOP_F32 || is->image.dtype != LOP_F32)
+        return fail(LOP_ERR_INVALID, "bilateral filter is Kernel<float>: F32 in/out (Listing 1)");
+    if (!(sigma_r > 0) || !std::isfinite(sigma_r)) return fail(LOP_ERR_INVALID, "sigma_r must be > 0");
+    const int sx = 2 * c.rx + 1, sy = 2 * c.ry + 1;
+    // log2 of the closeness coefficients (Listing 5 l.10 c = CMask(xf, yf))
+    std::unique_ptr<float[]> lc(new float[sx * sy]);
+    if (closeness) {
+        if (closeness->dtype != LOP_F32 || !closeness->coeffs)
+            return fail(LOP_ERR_INVALID, "closeness mask must be F32 with coefficients");
+        if (closeness->size_x != sx || closeness->size_y != sy)
+            return fail(LOP_ERR_INVALID, "closeness mask %d x %d != window %d x %d",
+                        closeness->size_x, closeness->size_y, sx, sy);
+        const float *cm = static_cast<const float *>(closeness->coeffs);
+        for (int i = 0; i < sx * sy; ++i) {
+            if (!(cm[i] >= 0) || !std::isfinite(cm[i]))
+                return fail(LOP_ERR_INVALID, "closeness coefficient %d = %g must be finite and >= 0",
+                            i, (double)cm[i]);
+            lc[i] = cm[i] > 0 ? (float)std::log2((double)cm[i]) : -INFINITY;
+        }
+        if (!(cm[c.ry * sx + c.rx] > 0))
+            return fail(LOP_ERR_INVALID, "closeness centre must be > 0 (reading c14)");
+    } else {
+        if (!(sigma_d > 0) || !std::isfinite(sigma_d))
+            return fail(LOP_ERR_INVALID, "sigma_d must be > 0");
+        const double c_d = 1.0 / (2.0 * (double)sigma_d * (double)sigma_d);
+        for (int yf = -c.ry; yf <= c.ry; ++yf)
+            for (int xf = -c.rx; xf <= c.rx; ++xf)  // Eq. (1) in the log2 domain
+                lc[(yf + c.ry) * sx + xf + c.rx] = (float)(-c_d * (double)(xf * xf + yf * yf) * kLog2e);
+    }
+    const float nk = (float)(-kLog2e / (2.0 * (double)sigma_r * (double)sigma_r));
+    cudaStream_t stream = static_cast<cudaStream_t>(cuda_stream);
+    const int32_t variant = g_variant;
+    const bool tiled_ok = c.rx <= lop::kTiledMaxRX;
+    if (variant == LOP_VARIANT_TILED && !tiled_ok)
+        return fail(LOP_ERR_UNSUPPORTED, "no tiled bilateral instance for window width %d", sx);
+    if (variant != LOP_VARIANT_GENERIC && tiled_ok) {
+        static thread_local lop::BilateralTiled p;
+        p.c = c;
+        p.nk = nk;
+        for (int r = 0; r < sy; ++r)
+            for (int k = 0; k < lop::kTiledMaskPitch; ++k)
+                p.lc[r * lop::kTiledMaskPitch + k] = k < sx ? lc[r * sx + k] : 0.0f;
+        return launched(lop::launch_bilateral_tiled(p, stream), "bilateral_tiled launch");
+    }
+    static thread_local lop::BilateralGeneric p;
+    p.c = c;
+    p.nk = nk;
+    std::memcpy(p.lc, lc.get(), sizeof(float) * sx * sy);
+    return launched(lop::launch_bilateral_generic(p, stream), "bilateral_generic launch");
+}
+
+// ------------------------------------------------------------ convolution
+lop_status lop_convolve_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                const lop_mask *mask, void *cuda_stream)
+{
+    Prepared pp;
+    lop_status st = prepare(is, in, pp);
+    if (st) return st;
+    const lop::Common &c = pp.c;
+    if (!mask || !mask->coeffs) return fail(LOP_ERR_INVALID, "mask is NULL");
+    const int sx = 2 * c.rx + 1, sy = 2 * c.ry + 1;
+    if (mask->size_x != sx || mask->size_y != sy)
+        return fail(LOP_ERR_INVALID, "mask %d x %d != window %d x %d", mask->size_x, mask->size_y,
+                    sx, sy);
+    const int32_t idt = in->bc->image.dtype, odt = is->image.dtype;
+    static thread_local lop::ConvGeneric p;
+    p.c = c;
+    p.shift = 0;
+    if (idt == LOP_F32 && odt == LOP_F32) {
+        if (mask->dtype != LOP_F32) return fail(LOP_ERR_INVALID, "F32 images need an F32 mask");
+        if (mask->shift != 0) return fail(LOP_ERR_INVALID, "F32 masks take shift 0");
+        p.kind = lop::CONV_F32;
+        const float *m = static_cast<const float *>(mask->coeffs);
+        for (int i = 0; i < sx * sy; ++i) {
+            if (!std::isfinite(m[i])) return fail(LOP_ERR_INVALID, "mask coefficient %d not finite", i);
+            p.m.f[i] = m[i];
+        }
+    } else if (idt == LOP_U8 && (odt == LOP_U8 || odt == LOP_I32)) {
+        if (mask->dtype != LOP_I32) return fail(LOP_ERR_INVALID, "U8 images need an I32 mask");
+        if (mask->shift < 0 || mask->shift > 30) return fail(LOP_ERR_INVALID, "shift must be in 0..30");
+        p.kind = odt == LOP_U8 ? lop::CONV_U8_U8 : lop::CONV_U8_I32;
+        p.shift = mask->shift;
+        const int32_t *m = static_cast<const int32_t *>(mask->coeffs);
+        int64_t l1 = 0;
+        for (int i = 0; i < sx * sy; ++i) {
+            p.m.i[i] = m[i];
+            l1 += m[i] < 0 ? -(int64_t)m[i] : m[i];
+        }
+        if (l1 * 255 + (1ll << 30) >= (1ll << 31))
+            return fail(LOP_ERR_UNSUPPORTED, "integer mask too large: sums may overflow int32");
+    } else {
+        return fail(LOP_ERR_INVALID, "unsupported dtype combination %d -> %d (F32->F32, U8->U8, U8->I32)",
+                    idt, odt);
+    }
+    cudaStream_t stream = static_cast<cudaStream_t>(cuda_stream);
+    const int32_t variant = g_variant;
+    const bool tiled_ok = lop::conv_tiled_supported(p);
+    if (variant == LOP_VARIANT_TILED && !tiled_ok)
+        return fail(LOP_ERR_UNSUPPORTED, "no tiled convolution instance for this mask");
+    if (variant != LOP_VARIANT_GENERIC && tiled_ok)
+        return launched(lop::launch_conv_tiled(p, stream), "conv_tiled launch");
+    return launched(lop::launch_conv_generic(p, stream), "conv_generic launch");
+}
+
+}  // extern "C"

@@ -1,0 +1,71 @@
+// lop_params.h -- kernel parameter blocks shared by the C-ABI host code
+// (lop_api.cpp) and the CUDA kernels (*.cu).  Product code only; the oracle
+// (oracle/) shares nothing with this tree.
+#pragma once
+#include <stdint.h>
+
+namespace lop {
+
+// Device-side view of an Image (lop_image) used for boundary resolution.
+// Row y (band-local, may be negative inside the top halo) of frame b starts at
+// data + b*bstride + y*stride.
+struct Geom {
+    const char *data;
+    int64_t stride;    // bytes
+    int64_t bstride;   // bytes between frames
+    int32_t W, H;      // owned columns / rows
+    int32_t halo_top, halo_bottom;
+    int32_t gy0, GH;   // band origin / global height
+};
+
+struct OutGeom {
+    char *data;
+    int64_t stride, bstride;
+    int32_t W, H;
+};
+
+// Everything a local-operator launch needs besides the mask.
+struct Common {
+    Geom in;
+    OutGeom out;
+    int32_t roi_x0, roi_y0, roi_w, roi_h;  // iteration space (output coords)
+    int32_t off_x, off_y;                  // accessor offset
+    int32_t mode;                          // lop_boundary
+    int32_t rx, ry;                        // window radii (size = 2r+1)
+    int32_t batch;
+    float cval_f;                          // CONSTANT value (f32 images)
+    int32_t cval_i;                        // CONSTANT value (u8 images)
+};
+
+constexpr int kMaxRadius = 31;                                // windows up to 63x63
+constexpr int kMaxTaps = (2 * kMaxRadius + 1) * (2 * kMaxRadius + 1);  // 3969
+constexpr int kTiledMaxRX = 7;                                // tiled kernels: 2*rx+1 <= 15
+constexpr int kTiledMaskPitch = 16;                           // floats per mask row in the tiled kernels
+constexpr int kTiledMaxTaps = (2 * kMaxRadius + 1) * kTiledMaskPitch;
+
+// Bilateral: weight w = ex2(lc[tap] + nk * (v - centre)^2)
+//   lc[tap] = log2 c(xf, yf), nk = -log2(e) / (2 sigma_r^2)
+struct BilateralGeneric {
+    Common c;
+    float nk;
+    float lc[kMaxTaps];
+};
+struct BilateralTiled {
+    Common c;
+    float nk;
+    float lc[kTiledMaxTaps];   // row pitch kTiledMaskPitch
+};
+
+// Convolution (correlation).  kind: 0 = f32->f32, 1 = u8->u8, 2 = u8->i32.
+enum ConvKind { CONV_F32 = 0, CONV_U8_U8 = 1, CONV_U8_I32 = 2 };
+struct ConvGeneric {
+    Common c;
+    int32_t kind;
+    int32_t shift;
+    union {
+        float f[kMaxTaps];     // f32 masks
+        int32_t i[kMaxTaps];   // integer masks (u8 images)
+    } m;
+};
+
+}  // namespace lop

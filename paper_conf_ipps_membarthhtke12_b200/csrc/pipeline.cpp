@@ -1,0 +1,246 @@
+// pipeline.cpp -- host pipeline for end-to-end execution from host buffers
+// (the paper's Listing 2 flow, L201-L253: IN = host_in; BF.execute();
+// host_out = OUT.getData()), overlapped on B200:
+//   stream h2d : chunk k+1 host -> device (rows + window halo)
+//   stream comp: chunk k filtered by the same kernels as lop_*_execute
+//   stream d2h : chunk k-1 device -> host
+// Double-buffered device staging, ordered with events.  The chunk views are
+// row bands of the global image (lop_image.global_y0/global_height), so the
+// boundary handling is exactly that of the whole-image call; REPEAT halo rows
+// outside the image are uploaded as ring rows.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <string>
+
+#include "lop.h"
+
+namespace lop_detail {
+void set_error(const std::string &msg);   // lop_api.cpp
+}
+
+struct lop_pipeline {
+    int device = 0;
+    int W = 0, H = 0, chunk = 0;
+    size_t in_bytes = 0, out_bytes = 0;     // per staging buffer
+    void *d_in[2] = {nullptr, nullptr};
+    void *d_out[2] = {nullptr, nullptr};
+    cudaStream_t s_h2d = nullptr, s_comp = nullptr, s_d2h = nullptr;
+    cudaEvent_t up_done[2] = {}, comp_done[2] = {}, down_done[2] = {};
+};
+
+namespace {
+
+constexpr int kMaxHalo = 31;   // largest window radius (63 x 63)
+
+lop_status perr(cudaError_t e, const char *what)
+{
+    lop_detail::set_error(std::string(what) + ": " + cudaGetErrorString(e));
+    return LOP_ERR_CUDA;
+}
+
+int esize(int32_t dt) { return dt == LOP_U8 ? 1 : 4; }
+
+struct DevGuard {
+    int prev = -1;
+    explicit DevGuard(int dev) { cudaGetDevice(&prev); cudaSetDevice(dev); }
+    ~DevGuard() { if (prev >= 0) cudaSetDevice(prev); }
+};
+
+int64_t wrap_row(int64_t gy, int64_t H)
+{
+    int64_t q = gy % H;
+    return q < 0 ? q + H : q;
+}
+
+// Enqueue the upload of chunk [y0, y1) with `ry` halo rows into buffer `buf`;
+// returns the band view.
+lop_status upload_chunk(lop_pipeline *p, int buf, const char *host, int64_t hstride, int es,
+                        int32_t dtype, int y0, int y1, int ry, int mode, lop_image *view)
+{
+    const int64_t dstride = (int64_t)p->W * es;
+    const int lo_in = std::max(0, y0 - ry), hi_in = std::min(p->H, y1 + ry);
+    int halo_top = y0 - lo_in, halo_bot = hi_in - y1;
+    if (mode == LOP_REPEAT) { halo_top = ry; halo_bot = ry; }   // ring rows always present
+    char *base = static_cast<char *>(p->d_in[buf]);
+    char *own0 = base + (int64_t)halo_top * dstride;         // row y0
+    cudaError_t e;
+    if (mode == LOP_REPEAT) {
+        for (int gy = y0 - ry; gy < y1 + ry; ++gy) {
+            if (gy >= lo_in && gy < hi_in) continue;
+            const int64_t src = wrap_row(gy, p->H);
+            e = cudaMemcpyAsync(own0 + (int64_t)(gy - y0) * dstride, host + src * hstride, dstride,
+                                cudaMemcpyHostToDevice, p->s_h2d);
+            if (e != cudaSuccess) return perr(e, "pipeline ring row upload");
+        }
+    }
+    e = cudaMemcpy2DAsync(own0 + (int64_t)(lo_in - y0) * dstride, dstride,
+                          host + (int64_t)lo_in * hstride, hstride, dstride, hi_in - lo_in,
+                          cudaMemcpyHostToDevice, p->s_h2d);
+    if (e != cudaSuccess) return perr(e, "pipeline upload");
+    std::memset(view, 0, sizeof *view);
+    view->data = own0;
+    view->width = p->W;
+    view->height = y1 - y0;
+    view->stride_bytes = dstride;
+    view->dtype = dtype;
+    view->batch = 1;
+    view->halo_top = halo_top;
+    view->halo_bottom = halo_bot;
+    view->global_y0 = y0;
+    view->global_height = p->H;
+    return LOP_OK;
+}
+
+template <typename Exec>
+lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t in_stride,
+               void *host_out, int32_t out_dtype, int64_t out_stride, int mode, double constant,
+               int size_x, int size_y, Exec exec)
+{
+    if (!p || !host_in || !host_out) return LOP_ERR_INVALID;
+    const int ry = size_y / 2;
+    if (ry > kMaxHalo || size_x / 2 > kMaxHalo) return LOP_ERR_UNSUPPORTED;
+    const int ies = esize(in_dtype), oes = esize(out_dtype);
+    if (in_stride < (int64_t)p->W * ies || out_stride < (int64_t)p->W * oes) return LOP_ERR_INVALID;
+    DevGuard guard(p->device);
+    const char *hin = static_cast<const char *>(host_in);
+    char *hout = static_cast<char *>(host_out);
+    const int nchunks = (p->H + p->chunk - 1) / p->chunk;
+    for (int k = 0; k < nchunks; ++k) {
+        const int buf = k & 1;
+        const int y0 = k * p->chunk, y1 = std::min(p->H, y0 + p->chunk);
+        cudaError_t e;
+        if (k >= 2) {
+            e = cudaStreamWaitEvent(p->s_h2d, p->comp_done[buf], 0);
+            if (e != cudaSuccess) return perr(e, "wait");
+        }
+        lop_image in_view;
+        lop_status st = upload_chunk(p, buf, hin, in_stride, ies, in_dtype, y0, y1, ry, mode, &in_view);
+        if (st) return st;
+        cudaEventRecord(p->up_done[buf], p->s_h2d);
+        cudaStreamWaitEvent(p->s_comp, p->up_done[buf], 0);
+        if (k >= 2) cudaStreamWaitEvent(p->s_comp, p->down_done[buf], 0);
+        lop_image out_view;
+        std::memset(&out_view, 0, sizeof out_view);
+        out_view.data = p->d_out[buf];
+        out_view.width = p->W;
+        out_view.height = y1 - y0;
+        out_view.stride_bytes = (int64_t)p->W * oes;
+        out_view.dtype = out_dtype;
+        out_view.batch = 1;
+        out_view.global_y0 = y0;
+        out_view.global_height = p->H;
+        lop_boundary_condition bc;
+        std::memset(&bc, 0, sizeof bc);
+        bc.image = in_view;
+        bc.mode = mode;
+        bc.size_x = size_x;
+        bc.size_y = size_y;
+        bc.constant = constant;
+        lop_accessor acc = {&bc, 0, 0};
+        lop_iteration_space is;
+        std::memset(&is, 0, sizeof is);
+        is.image = out_view;
+        st = exec(&is, &acc, p->s_comp);
+        if (st) return st;
+        cudaEventRecord(p->comp_done[buf], p->s_comp);
+        cudaStreamWaitEvent(p->s_d2h, p->comp_done[buf], 0);
+        e = cudaMemcpy2DAsync(hout + (int64_t)y0 * out_stride, out_stride, p->d_out[buf],
+                              (int64_t)p->W * oes, (int64_t)p->W * oes, y1 - y0,
+                              cudaMemcpyDeviceToHost, p->s_d2h);
+        if (e != cudaSuccess) return perr(e, "pipeline download");
+        cudaEventRecord(p->down_done[buf], p->s_d2h);
+    }
+    cudaError_t e = cudaStreamSynchronize(p->s_d2h);
+    if (e != cudaSuccess) return perr(e, "pipeline sync");
+    e = cudaStreamSynchronize(p->s_comp);
+    if (e != cudaSuccess) return perr(e, "pipeline sync");
+    return LOP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+lop_status lop_pipeline_create(int32_t device, int32_t width, int32_t height, int32_t chunk_rows,
+                               lop_pipeline **out)
+{
+    if (!out || width <= 0 || height <= 0) return LOP_ERR_INVALID;
+    *out = nullptr;
+    if (chunk_rows <= 0) chunk_rows = 512;
+    chunk_rows = std::min(chunk_rows, height);
+    DevGuard guard(device);
+    lop_pipeline *p = new lop_pipeline;
+    p->device = device;
+    p->W = width;
+    p->H = height;
+    p->chunk = chunk_rows;
+    p->in_bytes = (size_t)(chunk_rows + 2 * kMaxHalo) * width * 4;
+    p->out_bytes = (size_t)chunk_rows * width * 4;
+    cudaError_t e = cudaSuccess;
+    for (int i = 0; i < 2 && e == cudaSuccess; ++i) {
+        e = cudaMalloc(&p->d_in[i], p->in_bytes);
+        if (e == cudaSuccess) e = cudaMalloc(&p->d_out[i], p->out_bytes);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->up_done[i], cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->comp_done[i], cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->down_done[i], cudaEventDisableTiming);
+    }
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&p->s_h2d, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&p->s_comp, cudaStreamNonBlocking);
+    if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&p->s_d2h, cudaStreamNonBlocking);
+    if (e != cudaSuccess) {
+        lop_pipeline_destroy(p);
+        return perr(e, "pipeline create");
+    }
+    *out = p;
+    return LOP_OK;
+}
+
+lop_status lop_pipeline_bilateral(lop_pipeline *p, const float *host_in, int64_t in_stride_bytes,
+                                  float *host_out, int64_t out_stride_bytes, int32_t mode,
+                                  double constant, int32_t size_x, int32_t size_y,
+                                  const lop_mask *closeness, float sigma_d, float sigma_r)
+{
+    return run(p, host_in, LOP_F32, in_stride_bytes, host_out, LOP_F32, out_stride_bytes, mode,
+               constant, size_x, size_y,
+               [&](const lop_iteration_space *is, const lop_accessor *acc, cudaStream_t s) {
+                   return lop_bilateral_execute(is, acc, closeness, sigma_d, sigma_r, s);
+               });
+}
+
+lop_status lop_pipeline_convolve(lop_pipeline *p, const void *host_in, int32_t in_dtype,
+                                 int64_t in_stride_bytes, void *host_out, int32_t out_dtype,
+                                 int64_t out_stride_bytes, int32_t mode, double constant,
+                                 const lop_mask *mask)
+{
+    if (!mask) return LOP_ERR_INVALID;
+    return run(p, host_in, in_dtype, in_stride_bytes, host_out, out_dtype, out_stride_bytes, mode,
+               constant, mask->size_x, mask->size_y,
+               [&](const lop_iteration_space *is, const lop_accessor *acc, cudaStream_t s) {
+                   return lop_convolve_execute(is, acc, mask, s);
+               });
+}
+
+lop_status lop_pipeline_destroy(lop_pipeline *p)
+{
+    if (!p) return LOP_OK;
+    DevGuard guard(p->device);
+    if (p->s_h2d) cudaStreamSynchronize(p->s_h2d);
+    if (p->s_comp) cudaStreamSynchronize(p->s_comp);
+    if (p->s_d2h) cudaStreamSynchronize(p->s_d2h);
+    for (int i = 0; i < 2; ++i) {
+        if (p->d_in[i]) cudaFree(p->d_in[i]);
+        if (p->d_out[i]) cudaFree(p->d_out[i]);
+        if (p->up_done[i]) cudaEventDestroy(p->up_done[i]);
+        if (p->comp_done[i]) cudaEventDestroy(p->comp_done[i]);
+        if (p->down_done[i]) cudaEventDestroy(p->down_done[i]);
+    }
+    if (p->s_h2d) cudaStreamDestroy(p->s_h2d);
+    if (p->s_comp) cudaStreamDestroy(p->s_comp);
+    if (p->s_d2h) cudaStreamDestroy(p->s_d2h);
+    delete p;
+    return LOP_OK;
+}
+
+}  // extern "C"

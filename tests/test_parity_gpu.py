@@ -1,0 +1,351 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle.
+
+Floating point: max |gpu - oracle| <= 1e-5 on images in [0, 1] (BASELINE.json
+north_star).  Integer (u8 -> u8, u8 -> i32) outputs: bit-exact.  Undefined
+mode: only outputs whose window stays inside the image are compared
+(reading c9).  Full-size configs are checked on sampled outputs (all border
+strips + random interior points) computed one by one by the oracle.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synthetic
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-5
+MODES = ["undefined", "clamp", "repeat", "mirror", "constant"]
+
+
+@pytest.fixture(scope="module")
+def lop():
+    import paper_conf_ipps_membarthhtke12_b200 as lop
+    yield lop
+    lop.set_variant("auto")
+
+
+@pytest.fixture(params=["generic", "tiled"])
+def variant(request, lop):
+    lop.set_variant(request.param)
+    yield request.param
+    lop.set_variant("auto")
+
+
+CONV_VARIANTS = ["generic", "auto"]
+
+
+@pytest.fixture(params=CONV_VARIANTS)
+def conv_variant(request, lop):
+    lop.set_variant(request.param)
+    yield request.param
+    lop.set_variant("auto")
+
+
+def _cmp_float(gpu, ref, valid=None, tol=TOL):
+    gpu = np.asarray(gpu, dtype=np.float64)
+    ref = np.asarray(ref)
+    if valid is not None:
+        gpu, ref = gpu[valid], ref[valid]
+    err = np.abs(gpu - ref).max() if gpu.size else 0.0
+    assert err <= tol, "max abs err %.3g > %.1g" % (err, tol)
+    return err
+
+
+def _sample_points(H, W, n_random, r, seed):
+    rng = np.random.default_rng(seed)
+    pts = set()
+    for y in list(range(min(H, r + 2))) + list(range(max(0, H - r - 2), H)):
+        for x in range(0, W, max(1, W // 64)):
+            pts.add((y, x))
+    for x in list(range(min(W, r + 2))) + list(range(max(0, W - r - 2), W)):
+        for y in range(0, H, max(1, H // 64)):
+            pts.add((y, x))
+    for cy in (0, H - 1):
+        for cx in (0, W - 1):
+            for dy in range(-r, r + 1):
+                for dx in range(-r, r + 1):
+                    y, x = cy + dy, cx + dx
+                    if 0 <= y < H and 0 <= x < W:
+                        pts.add((y, x))
+    ys = rng.integers(0, H, n_random)
+    xs = rng.integers(0, W, n_random)
+    pts.update(zip(ys.tolist(), xs.tolist()))
+    pts = np.array(sorted(pts))
+    return pts[:, 0], pts[:, 1]
+
+
+# ------------------------------------------------------------- bilateral ----
+
+SHAPES = [(1, 1), (1, 7), (5, 1), (4, 4), (13, 17), (17, 13), (33, 130), (70, 257), (129, 131)]
+
+
+@pytest.mark.parametrize("shape", SHAPES)
+@pytest.mark.parametrize("mode", MODES)
+def test_bilateral_small_shapes(lop, variant, shape, mode):
+    H, W = shape
+    img = synthetic.uniform(H, W, seed=H * 1000 + W)
+    for sigma_d, size, sigma_r in ((1.0, 3, 5.0), (1.0, 5, 0.1), (3.0, 13, 0.1), (3.0, 13, 0.02)):
+        out = lop.bilateral(img.cuda(), sigma_d, sigma_r, mode, constant=0.5, size=size)
+        ref, valid = oracle.bilateral_f32(img.numpy(), sigma_d, sigma_r, mode, cval=0.5,
+                                          size=size)
+        _cmp_float(out.cpu().numpy(), ref, valid if mode == "undefined" else None)
+
+
+@pytest.mark.parametrize("size", [(5, 3), (3, 9), (15, 1), (1, 1), (9, 9), (7, 13)])
+def test_bilateral_asymmetric_windows(lop, variant, size):
+    img = synthetic.angio(61, 75, seed=77)
+    for mode in MODES:
+        out = lop.bilateral(img.cuda(), 1.5, 0.1, mode, constant=0.25, size=size)
+        ref, valid = oracle.bilateral_f32(img.numpy(), 1.5, 0.1, mode, cval=0.25, size=size)
+        _cmp_float(out.cpu().numpy(), ref, valid if mode == "undefined" else None)
+
+
+def test_bilateral_large_window_generic(lop):
+    img = synthetic.uniform(40, 45, seed=5)
+    out = lop.bilateral(img.cuda(), 6.0, 0.2, "mirror", size=25)       # rx = 12: generic only
+    ref, _ = oracle.bilateral_f32(img.numpy(), 6.0, 0.2, "mirror", size=25)
+    _cmp_float(out.cpu().numpy(), ref)
+
+
+def test_bilateral_user_mask(lop, variant):
+    rng = np.random.default_rng(4)
+    cm = (rng.random((5, 7)) + 0.05).astype(np.float32)
+    img = synthetic.uniform(50, 66, seed=8)
+    out = lop.bilateral(img.cuda(), 0.0, 0.15, "repeat", mask=cm)
+    ref, _ = oracle.bilateral_f32(img.numpy(), 0.0, 0.15, "repeat", cmask=cm.astype(np.float64))
+    _cmp_float(out.cpu().numpy(), ref)
+
+
+def test_bilateral_generic_and_tiled_bit_identical(lop):
+    img = synthetic.angio(300, 517, seed=11).cuda()
+    for mode in MODES:
+        for size in (3, 5, 13, (9, 5)):
+            lop.set_variant("generic")
+            a = lop.bilateral(img, 3.0, 0.05, mode, constant=0.5, size=size)
+            lop.set_variant("tiled")
+            b = lop.bilateral(img, 3.0, 0.05, mode, constant=0.5, size=size)
+            lop.set_variant("auto")
+            assert torch.equal(a, b), (mode, size)
+
+
+def test_config1_bilateral_256_clamp(lop):
+    """BASELINE config 1: 256x256 f32, sigma_d = 1 (3x3), sigma_r = 5, clamp."""
+    img = synthetic.angio(256, 256, seed=synthetic.config_seed(1))
+    out = lop.bilateral(img.cuda(), 1.0, 5.0, "clamp", size=3)
+    ref, _ = oracle.bilateral_f32(img.numpy(), 1.0, 5.0, "clamp", size=3)
+    _cmp_float(out.cpu().numpy(), ref)
+    # and the paper's default window 4*sigma_d+1 (reading c1)
+    out5 = lop.bilateral(img.cuda(), 1.0, 5.0, "clamp")
+    ref5, _ = oracle.bilateral_f32(img.numpy(), 1.0, 5.0, "clamp")
+    _cmp_float(out5.cpu().numpy(), ref5)
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_config2_bilateral_4096_sampled(lop, mode):
+    """BASELINE config 2 at full size, in the launch configuration bench.py
+    times (auto variant): 4096^2 f32, sigma_d = 3 (13x13), sigma_r = 5."""
+    H = W = 4096
+    img = synthetic.angio(H, W, seed=synthetic.config_seed(2), device="cuda")
+    out = lop.bilateral(img, 3.0, 5.0, mode, constant=0.0).cpu().numpy()
+    host = img.cpu().numpy()
+    ys, xs = _sample_points(H, W, 4000, 6, seed=2)
+    ref, valid = oracle.bilateral_f32_points(host, 3.0, 5.0, mode, xs, ys, cval=0.0)
+    _cmp_float(out[ys, xs], ref, valid if mode == "undefined" else None)
+    # small sigma_r exercises the range term (reading c3)
+    out2 = lop.bilateral(img, 3.0, 0.05, mode, constant=0.0).cpu().numpy()
+    ref2, valid2 = oracle.bilateral_f32_points(host, 3.0, 0.05, mode, xs, ys)
+    _cmp_float(out2[ys, xs], ref2, valid2 if mode == "undefined" else None)
+
+
+def test_bilateral_step_edge_bit_exact(lop):
+    """Levels {0, .5, 1}, sigma_r = 0.02: cross-edge weights underflow to 0 in
+    f32, so the output equals the input exactly (SURVEY §8(c) pins)."""
+    img = synthetic.levels(200, 300, seed=3)
+    out = lop.bilateral(img.cuda(), 3.0, 0.02, "clamp").cpu()
+    assert torch.equal(out, img)
+
+
+# ---------------------------------------------------------- convolution ----
+
+def _gauss_f32(size):
+    m, k = oracle.gaussian_mask(size)
+    return m / 2.0 ** k
+
+
+@pytest.mark.parametrize("shape", SHAPES)
+@pytest.mark.parametrize("mode", MODES)
+def test_conv_small_shapes(lop, conv_variant, shape, mode):
+    H, W = shape
+    img = synthetic.uniform(H, W, seed=H * 31 + W)
+    u8 = synthetic.uniform_u8(H, W, seed=H * 37 + W)
+    for size in (3, 5):
+        out = lop.gaussian(img.cuda(), size, mode, constant=0.5).cpu().numpy()
+        ref, valid = oracle.convolve_f32(img.numpy(), _gauss_f32(size), mode, 0.5)
+        _cmp_float(out, ref, valid if mode == "undefined" else None)
+        gm, k = oracle.gaussian_mask(size)
+        q = lop.gaussian(u8.cuda(), size, mode, constant=128).cpu().numpy()
+        refq, valid = oracle.convolve_u8(u8.numpy(), gm, k, mode, cval=128)
+        sel = valid if mode == "undefined" else slice(None)
+        assert (q[sel] == refq[sel]).all()
+    for d in (0, 1):
+        out = lop.sobel(img.cuda(), d, mode, constant=0.5).cpu().numpy()
+        ref, valid = oracle.convolve_f32(img.numpy(), oracle.sobel_mask(d), mode, 0.5)
+        _cmp_float(out, ref, valid if mode == "undefined" else None)
+        s = lop.sobel(u8.cuda(), d, mode, constant=7).cpu().numpy()
+        assert s.dtype == np.int32
+        refs, valid = oracle.convolve_u8(u8.numpy(), oracle.sobel_mask(d), 0, mode, cval=7,
+                                         out_dtype=np.int32)
+        sel = valid if mode == "undefined" else slice(None)
+        assert (s[sel] == refs[sel]).all()
+
+
+@pytest.mark.parametrize("msize", [(3, 5), (7, 1), (1, 9), (11, 11), (15, 3)])
+def test_conv_random_masks(lop, conv_variant, msize):
+    rng = np.random.default_rng(msize[0] * 100 + msize[1])
+    img = synthetic.uniform(45, 77, seed=1)
+    u8 = synthetic.uniform_u8(45, 77, seed=2)
+    mf = rng.standard_normal((msize[1], msize[0])).astype(np.float32)
+    mi = rng.integers(-20, 21, (msize[1], msize[0])).astype(np.int32)
+    for mode in MODES:
+        out = lop.convolve(img.cuda(), mf, mode, constant=0.3).cpu().numpy()
+        ref, valid = oracle.convolve_f32(img.numpy(), mf.astype(np.float64), mode, 0.3)
+        _cmp_float(out, ref, valid if mode == "undefined" else None, tol=1e-4)
+        for odt, npdt in ((torch.uint8, np.uint8), (torch.int32, np.int32)):
+            q = lop.convolve(u8.cuda(), mi, mode, constant=200, shift=3,
+                             out_dtype=odt).cpu().numpy()
+            refq, valid = oracle.convolve_u8(u8.numpy(), mi, 3, mode, cval=200, out_dtype=npdt)
+            sel = valid if mode == "undefined" else slice(None)
+            assert (q[sel] == refq[sel]).all(), (mode, odt)
+
+
+@pytest.mark.parametrize("mode", ["clamp", "repeat", "mirror", "constant"])
+def test_config3_u8_4096_full_bit_exact(lop, mode):
+    """BASELINE config 3, u8: Gaussian 5x5 (u8 -> u8) and Sobel 3x3 (u8 -> i32)
+    at 4096^2, every output compared with the oracle (bit-exact)."""
+    H = W = 4096
+    img = synthetic.to_u8(synthetic.angio(H, W, seed=synthetic.config_seed(3), device="cuda"))
+    host = img.cpu().numpy()
+    gm, k = oracle.gaussian_mask(5)
+    q = lop.gaussian(img, 5, mode, constant=128).cpu().numpy()
+    refq, _ = oracle.convolve_u8(host, gm, k, mode, cval=128)
+    assert (q == refq).all()
+    s = lop.sobel(img, 0, mode, constant=128).cpu().numpy()
+    refs, _ = oracle.convolve_u8(host, oracle.sobel_mask(0), 0, mode, cval=128,
+                                 out_dtype=np.int32)
+    assert (s == refs).all()
+
+
+@pytest.mark.parametrize("mode", ["clamp", "repeat", "mirror", "constant"])
+def test_config3_f32_4096(lop, mode):
+    H = W = 4096
+    img = synthetic.angio(H, W, seed=synthetic.config_seed(3), device="cuda")
+    host = img.cpu().numpy()
+    out = lop.gaussian(img, 5, mode, constant=0.5).cpu().numpy()
+    ref, _ = oracle.convolve_f32(host, _gauss_f32(5), mode, 0.5)
+    _cmp_float(out, ref)
+    s = lop.sobel(img, 0, mode, constant=0.5).cpu().numpy()
+    ys, xs = _sample_points(H, W, 20000, 2, seed=3)
+    refs, _ = oracle.convolve_f32_points(host, oracle.sobel_mask(0), mode, xs, ys, 0.5)
+    _cmp_float(s[ys, xs], refs)
+
+
+# ----------------------------------------------- frames, bands, ROI, misc ----
+
+def test_frames_batch_equals_per_frame_and_oracle(lop):
+    frames = synthetic.angio_frames(1024, 96, 128, seed=synthetic.config_seed(4), first=0,
+                                    count=5).cuda()
+    out = lop.bilateral(frames, 3.0, 5.0, "clamp")
+    for f in range(frames.shape[0]):
+        single = lop.bilateral(frames[f].contiguous(), 3.0, 5.0, "clamp")
+        assert torch.equal(out[f], single)
+    ref, _ = oracle.bilateral_f32(frames[3].cpu().numpy(), 3.0, 5.0, "clamp")
+    _cmp_float(out[3].cpu().numpy(), ref)
+    g = lop.gaussian(frames, 5, "mirror")
+    assert torch.equal(g[2], lop.gaussian(frames[2].contiguous(), 5, "mirror"))
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_band_views_bit_identical_to_whole_image(lop, mode):
+    """Row bands with halo rows (ring rows for REPEAT) reproduce the whole-image
+    output bit for bit (what the NCCL band partition relies on)."""
+    H, W, r = 100, 140, 6
+    img = synthetic.angio(H, W, seed=21).cuda()
+    whole = lop.bilateral(img, 3.0, 0.1, mode, constant=0.5)
+    wg = lop.gaussian(img, 5, mode, constant=0.5)
+    cuts = [0, 7, 40, 41, 93, 100]
+    for y0, y1 in zip(cuts[:-1], cuts[1:]):
+        top = r if (y0 > 0 or mode == "repeat") else 0
+        bot = r if (y1 < H or mode == "repeat") else 0
+        rows = [(y % H) for y in range(y0 - top, y1 + bot)]
+        buf = img[rows].contiguous()
+        band = buf[top:top + (y1 - y0)]
+        out = lop.bilateral(band, 3.0, 0.1, mode, constant=0.5, band=(top, bot, y0, H))
+        assert torch.equal(out, whole[y0:y1]), (y0, y1)
+        og = lop.gaussian(band, 5, mode, constant=0.5, band=(top, bot, y0, H))
+        assert torch.equal(og, wg[y0:y1]), (y0, y1)
+
+
+def test_band_validation_rejects_missing_halo(lop):
+    img = torch.rand(50, 64, device="cuda")
+    with pytest.raises(lop.LopError, match="halo"):
+        lop.bilateral(img[10:20], 3.0, 0.1, "clamp", band=(0, 0, 10, 50))
+
+
+def test_roi_and_unaligned_views(lop, variant):
+    img = synthetic.angio(90, 203, seed=31).cuda()
+    full = lop.bilateral(img, 2.0, 0.1, "mirror", size=9)
+    out = torch.full_like(img, -7.0)
+    lop.bilateral(img, 2.0, 0.1, "mirror", size=9, out=out, roi=(5, 3, 101, 77))
+    assert torch.equal(out[3:80, 5:106], full[3:80, 5:106])
+    out[3:80, 5:106] = -7.0
+    assert (out == -7.0).all()
+    # strided, non-16B-aligned view (column offset 3 of a wider tensor)
+    wide = synthetic.angio(90, 260, seed=32).cuda()
+    view = wide[:, 3:206]
+    a = lop.bilateral(view, 2.0, 0.1, "clamp", size=9)
+    b = lop.bilateral(view.contiguous(), 2.0, 0.1, "clamp", size=9)
+    assert torch.equal(a, b)
+    ref, _ = oracle.bilateral_f32(view.cpu().numpy(), 2.0, 0.1, "clamp", size=9)
+    _cmp_float(a.cpu().numpy(), ref)
+
+
+def test_accessor_offset(lop, variant):
+    img = synthetic.angio(64, 96, seed=41).cuda()
+    out = lop.gaussian(img, 5, "clamp", offset=(3, -2))
+    ref = lop.gaussian(img, 5, "clamp")
+    # interior: out(x, y) = G(I)(x + 3, y - 2)
+    assert torch.equal(out[10:50, 5:80], ref[8:48, 8:83])
+    b = lop.bilateral(img, 1.0, 0.1, "repeat", size=5, offset=(-4, 5))
+    rb = lop.bilateral(torch.roll(img, shifts=(-5, 4), dims=(0, 1)), 1.0, 0.1, "repeat", size=5)
+    assert torch.equal(b, rb)
+
+
+def test_pipeline_host_end_to_end(lop):
+    H, W = 1000, 640
+    img = synthetic.angio(H, W, seed=51).pin_memory()
+    dev = lop.bilateral(img.cuda(), 3.0, 0.1, "repeat").cpu()
+    p = lop.Pipeline(W, H, chunk_rows=128)
+    out = torch.empty_like(img).pin_memory()
+    for mode in MODES:
+        p.bilateral(img, out, 3.0, 0.1, mode, constant=0.5)
+        dev = lop.bilateral(img.cuda(), 3.0, 0.1, mode, constant=0.5).cpu()
+        if mode == "undefined":
+            assert torch.equal(out[6:-6, 6:-6], dev[6:-6, 6:-6])
+        else:
+            assert torch.equal(out, dev), mode
+    u8 = synthetic.to_u8(img)
+    gm, k = lop.gaussian_mask(5)
+    out8 = torch.empty_like(u8)
+    p.convolve(u8, out8, gm, "mirror", shift=k)
+    assert torch.equal(out8, lop.gaussian(u8.cuda(), 5, "mirror").cpu())
+    p.close()
+
+
+def test_launch_count(lop):
+    img = torch.rand(64, 64, device="cuda")
+    lop.reset_launch_count()
+    lop.bilateral(img, 1.0, 0.1)
+    lop.gaussian(img)
+    assert lop.launch_count() == 2
