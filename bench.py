@@ -265,9 +265,8 @@ def run_lop(args, dist, peaks):
         px_per_step_rank = band.rows * GW
 
         def step(i):
-            band.exchange()
-            lop.bilateral(band.owned, sigma_d, sigma_r, args.mode, size=size, out=out,
-                          stream=stream, band=band.band_args())
+            ldist.bilateral_bands(lop, band, sigma_d, sigma_r, args.mode, size=size, out=out,
+                                  stream=stream)
         config = {"workload": "32768^2 f32 bilateral 13x13 %s, row bands + NCCL halo exchange "
                               "(BASELINE config 5)" % args.mode,
                   "height": GHt, "width": GW, "window": size, "boundary": args.mode,

@@ -1,13 +1,397 @@
-// conv_tiled.cu -- HBM-bound tiled convolution kernels (Gaussian / Sobel).
-// First version: no tiled instance yet; the dispatcher uses conv_generic.
+// conv_tiled.cu -- HBM-bound tiled convolution kernels (Gaussian / Sobel and
+// any separable mask up to 9x9): Tables VIII-IX, Sobel
+// "same implementation" (L847-L849).
+//
+// Design:
+//  * the mask is separable (factorised exactly on the host): M = c r^T, so
+//    each output is sum_t c[t] * (sum_xf r[xf] * I(x+xf, y+t-RY)).  The u8
+//    path is exact integer arithmetic, hence bit-identical to the 2D
+//    definition (reading c13); the f32 path is within rounding of it.
+//  * a CTA (128 threads) owns an output tile of 128*PX columns x TS rows
+//    (f32: 512 x 16, u8: 1024 x 16).  Its input footprint, TS + 2RY rows of
+//    128*PX + 2*PAD bytes-aligned columns, is staged into shared memory with
+//    one cp.async.bulk (TMA bulk copy, SASS UBLKCP) per row completing on an
+//    mbarrier -- every row of the tile in flight at once, each input byte read
+//    from DRAM once.  Border tiles (image edge, band edge without halo,
+//    unaligned views) stage element by element with the boundary resolved at
+//    staging time instead (the paper's nine-region idea, Fig. 3 / Listing 8,
+//    reduced to interior vs border CTAs).
+//  * each thread then streams its PX columns down the tile from shared
+//    memory, keeps the horizontal sums of the last 2RY+1 rows in registers and
+//    writes every output row with one 16-B (f32, i32) / 8-B (u8) store.
+//  * coefficients are kernel parameters (constant-bank operands of FFMA/IMAD),
+//    the dynamic constant-memory variant of §IV-C (L563-L605).
 #include <cuda_runtime.h>
+#include <stdint.h>
 
+#include <type_traits>
+
+#include "boundary.cuh"
 #include "kernels.h"
+#include "lop_params.h"
 
 namespace lop {
 
-bool conv_tiled_supported(const ConvGeneric &) { return false; }
+struct ConvSep {
+    Common c;
+    int32_t kind;
+    int32_t shift;
+    float rf[9], cf[9];      // f32 row / column coefficients
+    int32_t ri[9], ci[9];    // integer row / column coefficients
+};
 
-cudaError_t launch_conv_tiled(const ConvGeneric &, cudaStream_t) { return cudaErrorNotSupported; }
+namespace convt {
+constexpr int NT = 128;      // threads per CTA
+constexpr int TS = 16;       // output rows per tile
+}  // namespace convt
+
+template <typename T> struct Px;
+template <> struct Px<float> { static constexpr int N = 4; };
+template <> struct Px<uint8_t> { static constexpr int N = 8; };
+
+template <typename T> struct TileShape {
+    static constexpr int PX = Px<T>::N;
+    static constexpr int TWE = convt::NT * PX;                 // output columns per tile
+    static constexpr int PADE = 16 / sizeof(T);                // left/right pad (elements), 16 B
+    static constexpr int SWE = TWE + 2 * PADE;                 // smem row pitch (elements)
+    static constexpr int ROW_BYTES = SWE * sizeof(T);          // multiple of 16
+};
+
+__device__ __forceinline__ uint32_t smem_addr(const void *p)
+{
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+template <typename T, typename TO, int R>
+__global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_constant__ ConvSep p)
+{
+    constexpr int RX = R, RY = R;
+    using S = TileShape<T>;
+    constexpr int PX = S::PX, TS = convt::TS, SWE = S::SWE, PADE = S::PADE;
+    constexpr bool F = sizeof(T) == 4;
+    using A = typename std::conditional<F, float, int>::type;   // accumulator type
+    static_assert(RX <= 4, "halo must fit the 16-B pad");
+
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ __align__(8) uint64_t bar;
+    T *tile = reinterpret_cast<T *>(smem_raw);                    // (TS+2RY) x SWE
+
+    const Common &c = p.c;
+    const Geom &g = c.in;
+    const int b = blockIdx.z;
+    const int tx0 = c.roi_x0 + blockIdx.x * S::TWE;               // output tile origin
+    const int ty0 = c.roi_y0 + blockIdx.y * TS;
+    const int roi_x1 = c.roi_x0 + c.roi_w, roi_y1 = c.roi_y0 + c.roi_h;
+    const int nrows = min(TS, roi_y1 - ty0);                      // output rows in this tile
+    const int srows = nrows + 2 * RY;                             // staged input rows
+    const int ix0 = tx0 + c.off_x - PADE;                         // input col of smem col 0
+    const int iy0 = ty0 + c.off_y - RY;                           // input row of smem row 0
+    const char *fbase = g.data + (int64_t)b * g.bstride;
+
+    // ---------------------------------------------------------------- stage
+    // Every staged row whose source row exists (in-image, halo, or mapped by
+    // the boundary mode) is copied by one cp.async.bulk of its 16-B aligned
+    // in-image column span; the out-of-image columns (and CONSTANT rows) are
+    // filled element by element with the boundary resolved per column.
+    const A cval = F ? (A)c.cval_f : (A)c.cval_i;
+    const bool aligned = ((reinterpret_cast<uintptr_t>(fbase) | (uintptr_t)g.stride |
+                           (uintptr_t)(ix0 * (int)sizeof(T))) % 16 == 0);
+    constexpr int V16 = 16 / sizeof(T);                            // elements per 16 B
+    // bulk span [xa, xb) in smem columns (same for every row)
+    int xa = max(0, -ix0), xb = min(SWE, g.W - ix0);
+    xa = (xa + V16 - 1) / V16 * V16;
+    xb = xb / V16 * V16;
+    const bool bulk = aligned && xb > xa;
+    if (bulk) {
+        if (threadIdx.x == 0) {
+            asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&bar)));
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int nbytes = 0;
+            for (int r = 0; r < srows; ++r) {
+                int row;
+                if (resolve_row(iy0 + r, g, c.mode, row)) nbytes += (xb - xa) * (int)sizeof(T);
+            }
+            asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;"
+                         ::"r"(smem_addr(&bar)), "r"(nbytes) : "memory");
+        }
+        for (int r = threadIdx.x; r < srows; r += convt::NT) {
+            int row;
+            if (!resolve_row(iy0 + r, g, c.mode, row)) continue;
+            const char *src = fbase + (int64_t)row * g.stride + (int64_t)(ix0 + xa) * sizeof(T);
+            asm volatile(
+                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                ::"r"(smem_addr(tile + r * SWE + xa)), "l"(src), "r"((xb - xa) * (int)sizeof(T)),
+                  "r"(smem_addr(&bar))
+                : "memory");
+        }
+    }
+    // element-wise part: the columns outside the bulk span of every row ...
+    const int side = bulk ? xa + (SWE - xb) : SWE;
+    for (int i = threadIdx.x; i < srows * side; i += convt::NT) {
+        const int r = i / side, k = i - r * side;
+        const int x = !bulk ? k : (k < xa ? k : xb + (k - xa));
+        int row, col;
+        T v;
+        if (resolve_row(iy0 + r, g, c.mode, row) && resolve_col(ix0 + x, g, c.mode, col))
+            v = __ldg(row_ptr<T>(g, b, row) + col);
+        else
+            v = (T)cval;
+        tile[r * SWE + x] = v;
+    }
+    // ... and the bulk span of CONSTANT rows (no source row to copy)
+    if (bulk && c.mode == M_CONSTANT) {
+        for (int r = 0; r < srows; ++r) {
+            int row;
+            if (resolve_row(iy0 + r, g, c.mode, row)) continue;
+            for (int x = xa + threadIdx.x; x < xb; x += convt::NT) tile[r * SWE + x] = (T)cval;
+        }
+    }
+    __syncthreads();
+    if (bulk) {
+        asm volatile(
+            "{\n\t.reg .pred P;\n"
+            "WAIT_%=:\n\t"
+            "mbarrier.try_wait.parity.shared.b64 P, [%0], 0;\n\t"
+            "@!P bra WAIT_%=;\n}" ::"r"(smem_addr(&bar)) : "memory");
+    }
+
+    // -------------------------------------------------------------- compute
+    const int ox0 = tx0 + threadIdx.x * PX;
+    if (ox0 >= roi_x1) return;
+    char *obase = c.out.data + (int64_t)b * c.out.bstride;
+    const bool ovec = (ox0 + PX <= roi_x1) && (ox0 % PX == 0) &&
+                      (((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) %
+                        (sizeof(TO) * PX > 16 ? 16 : sizeof(TO) * PX)) == 0);
+    const T *tcol = tile + PADE + threadIdx.x * PX;              // this thread's centre column
+    A h[2 * RY + 1][PX];                                          // horizontal sums, ring
+#pragma unroll
+    for (int k = 0; k < TS + 2 * RY; ++k) {
+        if (k >= srows) break;
+        // ---- gather PX + 2RX values of staged row k
+        A v[PX + 2 * RX];
+        const T *rp = tcol + k * SWE;
+        if constexpr (F) {
+            const float4 cv = *reinterpret_cast<const float4 *>(rp);
+            v[RX + 0] = cv.x; v[RX + 1] = cv.y; v[RX + 2] = cv.z; v[RX + 3] = cv.w;
+            if constexpr (RX > 0) {
+                const float4 l = *reinterpret_cast<const float4 *>(rp - 4);
+                const float4 r = *reinterpret_cast<const float4 *>(rp + 4);
+                const float lv[4] = {l.x, l.y, l.z, l.w}, rv[4] = {r.x, r.y, r.z, r.w};
+#pragma unroll
+                for (int j = 0; j < RX; ++j) {
+                    v[j] = lv[4 - RX + j];
+                    v[RX + PX + j] = rv[j];
+                }
+            }
+        } else {
+            const uint2 cv = *reinterpret_cast<const uint2 *>(rp);
+            const uint32_t w[2] = {cv.x, cv.y};
+#pragma unroll
+            for (int j = 0; j < 8; ++j) v[RX + j] = (int)((w[j >> 2] >> (8 * (j & 3))) & 0xFF);
+            if constexpr (RX > 0) {
+                const uint32_t l = *reinterpret_cast<const uint32_t *>(rp - 4);
+                const uint32_t r = *reinterpret_cast<const uint32_t *>(rp + 8);
+#pragma unroll
+                for (int j = 0; j < RX; ++j) {
+                    v[j] = (int)((l >> (8 * (4 - RX + j))) & 0xFF);
+                    v[RX + PX + j] = (int)((r >> (8 * j)) & 0xFF);
+                }
+            }
+        }
+        // ---- horizontal pass
+        A *hk = h[k % (2 * RY + 1)];
+#pragma unroll
+        for (int j = 0; j < PX; ++j) {
+            A s;
+            if constexpr (F) {
+                s = __fmul_rn(p.rf[0], v[j]);
+#pragma unroll
+                for (int t = 1; t <= 2 * RX; ++t) s = __fmaf_rn(p.rf[t], v[j + t], s);
+            } else {
+                s = p.ri[0] * v[j];
+#pragma unroll
+                for (int t = 1; t <= 2 * RX; ++t) s += p.ri[t] * v[j + t];
+            }
+            hk[j] = s;
+        }
+        // ---- vertical pass: output row o = k - 2RY is complete
+        const int o = k - 2 * RY;
+        if (o < 0) continue;
+        A out[PX];
+#pragma unroll
+        for (int j = 0; j < PX; ++j) {
+            A s;
+            if constexpr (F) {
+                s = __fmul_rn(p.cf[0], h[o % (2 * RY + 1)][j]);
+#pragma unroll
+                for (int t = 1; t <= 2 * RY; ++t)
+                    s = __fmaf_rn(p.cf[t], h[(o + t) % (2 * RY + 1)][j], s);
+            } else {
+                s = p.ci[0] * h[o % (2 * RY + 1)][j];
+#pragma unroll
+                for (int t = 1; t <= 2 * RY; ++t) s += p.ci[t] * h[(o + t) % (2 * RY + 1)][j];
+            }
+            out[j] = s;
+        }
+        char *orow = obase + (int64_t)(ty0 + o) * c.out.stride;
+        if constexpr (F) {
+            float *op = reinterpret_cast<float *>(orow) + ox0;
+            if (ovec) {
+                *reinterpret_cast<float4 *>(op) = make_float4(out[0], out[1], out[2], out[3]);
+            } else {
+#pragma unroll
+                for (int j = 0; j < PX; ++j)
+                    if (ox0 + j < roi_x1) op[j] = out[j];
+            }
+        } else if constexpr (sizeof(TO) == 1) {
+            uint32_t w[2] = {0u, 0u};
+#pragma unroll
+            for (int j = 0; j < PX; ++j) {
+                const int q = min(max(quantize_shift(out[j], p.shift), 0), 255);
+                w[j >> 2] |= (uint32_t)q << (8 * (j & 3));
+            }
+            uint8_t *op = reinterpret_cast<uint8_t *>(orow) + ox0;
+            if (ovec) {
+                *reinterpret_cast<uint2 *>(op) = make_uint2(w[0], w[1]);
+            } else {
+#pragma unroll
+                for (int j = 0; j < PX; ++j)
+                    if (ox0 + j < roi_x1) op[j] = (uint8_t)(w[j >> 2] >> (8 * (j & 3)));
+            }
+        } else {
+            int32_t *op = reinterpret_cast<int32_t *>(orow) + ox0;
+            int q[PX];
+#pragma unroll
+            for (int j = 0; j < PX; ++j) q[j] = quantize_shift(out[j], p.shift);
+            if (ovec) {
+                *reinterpret_cast<int4 *>(op) = make_int4(q[0], q[1], q[2], q[3]);
+                *reinterpret_cast<int4 *>(op + 4) = make_int4(q[4], q[5], q[6], q[7]);
+            } else {
+#pragma unroll
+                for (int j = 0; j < PX; ++j)
+                    if (ox0 + j < roi_x1) op[j] = q[j];
+            }
+        }
+    }
+}
+
+// -------------------------------------------------------------- host side
+namespace {
+
+int64_t gcd64(int64_t a, int64_t b)
+{
+    a = a < 0 ? -a : a;
+    b = b < 0 ? -b : b;
+    while (b) { int64_t t = a % b; a = b; b = t; }
+    return a;
+}
+
+bool verify_f32(const float *M, int sx, int sy, const float *cf, const float *rf)
+{
+    for (int i = 0; i < sy; ++i)
+        for (int j = 0; j < sx; ++j)
+            if ((double)cf[i] * (double)rf[j] != (double)M[i * sx + j]) return false;
+    return true;
+}
+
+// Exact rank-1 factorisation M = c r^T (integer or float); false if none.
+bool factor(const ConvGeneric &p, ConvSep &s)
+{
+    const int sx = 2 * p.c.rx + 1, sy = 2 * p.c.ry + 1;
+    if (sx > 9 || sy > 9) return false;
+    for (int t = 0; t < 9; ++t) { s.rf[t] = s.cf[t] = 0.f; s.ri[t] = s.ci[t] = 0; }
+    int i0 = -1, j0 = -1;
+    for (int i = 0; i < sy && i0 < 0; ++i)
+        for (int j = 0; j < sx; ++j) {
+            const bool nz = p.kind == CONV_F32 ? p.m.f[i * sx + j] != 0.0f : p.m.i[i * sx + j] != 0;
+            if (nz) { i0 = i; j0 = j; break; }
+        }
+    if (i0 < 0) return true;             // all-zero mask
+    if (p.kind == CONV_F32) {
+        const float *M = p.m.f;
+        // (a) r = row i0, c = column j0 / M[i0][j0];  (b) r = row i0 / M[i0][j0], c = column j0
+        for (int j = 0; j < sx; ++j) s.rf[j] = M[i0 * sx + j];
+        for (int i = 0; i < sy; ++i) s.cf[i] = M[i * sx + j0] / M[i0 * sx + j0];
+        if (verify_f32(M, sx, sy, s.cf, s.rf)) return true;
+        for (int j = 0; j < sx; ++j) s.rf[j] = M[i0 * sx + j] / M[i0 * sx + j0];
+        for (int i = 0; i < sy; ++i) s.cf[i] = M[i * sx + j0];
+        return verify_f32(M, sx, sy, s.cf, s.rf);
+    }
+    const int32_t *M = p.m.i;
+    int64_t g = 0;
+    for (int j = 0; j < sx; ++j) g = gcd64(g, M[i0 * sx + j]);
+    for (int j = 0; j < sx; ++j) s.ri[j] = (int32_t)(M[i0 * sx + j] / g);
+    const int64_t rj0 = s.ri[j0];
+    for (int i = 0; i < sy; ++i) {
+        if (M[i * sx + j0] % rj0) return false;
+        s.ci[i] = (int32_t)(M[i * sx + j0] / rj0);
+    }
+    for (int i = 0; i < sy; ++i)
+        for (int j = 0; j < sx; ++j)
+            if ((int64_t)s.ci[i] * s.ri[j] != (int64_t)M[i * sx + j]) return false;
+    // partial sums must stay exact in int32 (255 * sum|r| * sum|c|)
+    int64_t lr = 0, lc = 0;
+    for (int j = 0; j < sx; ++j) lr += s.ri[j] < 0 ? -(int64_t)s.ri[j] : s.ri[j];
+    for (int i = 0; i < sy; ++i) lc += s.ci[i] < 0 ? -(int64_t)s.ci[i] : s.ci[i];
+    return 255 * lr * lc + (1ll << 30) < (1ll << 31);
+}
+
+template <typename T, typename TO, int R>
+cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
+{
+    using S = TileShape<T>;
+    const size_t smem = (size_t)(convt::TS + 2 * R) * S::ROW_BYTES;
+    dim3 grid((s.c.roi_w + S::TWE - 1) / S::TWE, (s.c.roi_h + convt::TS - 1) / convt::TS,
+              s.c.batch);
+    static bool configured = false;
+    if (!configured && smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(conv_sep_kernel<T, TO, R>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        configured = true;
+    }
+    conv_sep_kernel<T, TO, R><<<grid, convt::NT, smem, stream>>>(s);
+    return cudaGetLastError();
+}
+
+template <typename T, typename TO>
+cudaError_t dispatch_r(const ConvSep &s, cudaStream_t stream)
+{
+    switch (s.c.rx) {
+    case 0: return launch_sep<T, TO, 0>(s, stream);
+    case 1: return launch_sep<T, TO, 1>(s, stream);
+    case 2: return launch_sep<T, TO, 2>(s, stream);
+    case 3: return launch_sep<T, TO, 3>(s, stream);
+    case 4: return launch_sep<T, TO, 4>(s, stream);
+    default: return cudaErrorNotSupported;
+    }
+}
+
+}  // namespace
+
+bool conv_tiled_supported(const ConvGeneric &p)
+{
+    if (p.c.rx != p.c.ry || p.c.rx > 4) return false;
+    static thread_local ConvSep s;
+    return factor(p, s);
+}
+
+cudaError_t launch_conv_tiled(const ConvGeneric &p, cudaStream_t stream)
+{
+    static thread_local ConvSep s;
+    if (p.c.rx != p.c.ry || p.c.rx > 4 || !factor(p, s)) return cudaErrorNotSupported;
+    s.c = p.c;
+    s.kind = p.kind;
+    s.shift = p.shift;
+    switch (p.kind) {
+    case CONV_F32: return dispatch_r<float, float>(s, stream);
+    case CONV_U8_U8: return dispatch_r<uint8_t, uint8_t>(s, stream);
+    case CONV_U8_I32: return dispatch_r<uint8_t, int32_t>(s, stream);
+    default: return cudaErrorNotSupported;
+    }
+}
 
 }  // namespace lop

@@ -43,9 +43,17 @@ def _u(g, lo, hi, n=(), device="cpu"):
     return lo + (hi - lo) * torch.rand(n, generator=g, device=device, dtype=torch.float64)
 
 
+NOISE_BLOCK = 256     # noise is drawn per block of 256 rows, seeded by (seed, frame, block)
+
+
 def angio(height: int, width: int, seed: int, frame: int = 0, n_frames: int = 1,
-          device="cpu", row_chunk: int = 2048) -> torch.Tensor:
-    """One float32 angiography-like frame in [0, 1], shape (height, width)."""
+          device="cpu", row_range=None) -> torch.Tensor:
+    """One float32 angiography-like frame in [0, 1], shape (height, width).
+
+    row_range=(y0, y1) returns only rows [y0, y1) of that same image (used to
+    generate row bands in place on each rank); the pixels do not depend on
+    the range requested.
+    """
     device = torch.device(device)
     H, W = int(height), int(width)
     g = _gen(seed, "cpu")                       # geometry: drawn on CPU (device-independent)
@@ -80,12 +88,15 @@ def angio(height: int, width: int, seed: int, frame: int = 0, n_frames: int = 1,
         sy = round(2.0 * math.cos(2 * math.pi * frame / 23.0))
     else:
         bolus, sx, sy = 1.0, 0, 0
-    gn = _gen(seed ^ (int(frame) * 0x9E3779B9), device)
+    fseed = seed ^ (int(frame) * 0x9E3779B9)
+    y_lo, y_hi = (0, H) if row_range is None else (int(row_range[0]), int(row_range[1]))
 
-    out = torch.empty((H, W), dtype=torch.float32, device=device)
+    out = torch.empty((y_hi - y_lo, W), dtype=torch.float32, device=device)
     xs = torch.arange(W, device=device, dtype=torch.float32) - sx
-    for r0 in range(0, H, row_chunk):
-        r1 = min(H, r0 + row_chunk)
+    for blk in range(y_lo // NOISE_BLOCK, (y_hi + NOISE_BLOCK - 1) // NOISE_BLOCK):
+        r0 = max(y_lo, blk * NOISE_BLOCK)
+        r1 = min(y_hi, (blk + 1) * NOISE_BLOCK, H)
+        gn = _gen(fseed * 1000003 + blk, device)
         ys = (torch.arange(r0, r1, device=device, dtype=torch.float32) - sy)[:, None]
         img = torch.full((r1 - r0, W), 0.55, device=device, dtype=torch.float32)
         for a, fx, fy, ph in waves:
@@ -101,9 +112,11 @@ def angio(height: int, width: int, seed: int, frame: int = 0, n_frames: int = 1,
             prof = torch.exp(-d2 / (2.0 * radius * radius))
             inside = ((along >= start) & (along < stop)).to(torch.float32)
             img -= (depth * bolus) * prof * inside
-        noise = torch.randn((r1 - r0, W), generator=gn, device=device, dtype=torch.float32)
+        b0 = blk * NOISE_BLOCK
+        noise = torch.randn((min(H, b0 + NOISE_BLOCK) - b0, W), generator=gn, device=device,
+                            dtype=torch.float32)[r0 - b0:r1 - b0]
         img += 0.02 * noise
-        out[r0:r1] = img.clamp_(0.0, 1.0)
+        out[r0 - y_lo:r1 - y_lo] = img.clamp_(0.0, 1.0)
     return out
 
 

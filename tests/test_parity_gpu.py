@@ -33,10 +33,7 @@ def variant(request, lop):
     lop.set_variant("auto")
 
 
-CONV_VARIANTS = ["generic", "auto"]
-
-
-@pytest.fixture(params=CONV_VARIANTS)
+@pytest.fixture(params=["generic", "tiled"])
 def conv_variant(request, lop):
     lop.set_variant(request.param)
     yield request.param
@@ -201,8 +198,32 @@ def test_conv_small_shapes(lop, conv_variant, shape, mode):
         assert (s[sel] == refs[sel]).all()
 
 
+@pytest.mark.parametrize("size", [1, 3, 5, 7, 9])
+def test_conv_random_separable_masks(lop, conv_variant, size):
+    """Rank-1 masks take the tiled separable kernel (exact factorisation on the
+    host); u8 stays bit-exact (reading c13)."""
+    rng = np.random.default_rng(size)
+    img = synthetic.uniform(57, 203, seed=3)
+    u8 = synthetic.uniform_u8(57, 203, seed=4)
+    # column factors whose ratios are powers of two: the float factorisation is exact
+    cf = (rng.choice([-4, -2, -1, 1, 2, 4], size)).astype(np.float32)
+    rf = (rng.integers(-8, 9, size) / 8.0).astype(np.float32)
+    mf = np.outer(cf, rf).astype(np.float32)
+    mi = np.outer(rng.integers(-5, 6, size), rng.integers(-5, 6, size)).astype(np.int32)
+    for mode in MODES:
+        out = lop.convolve(img.cuda(), mf, mode, constant=0.7).cpu().numpy()
+        ref, valid = oracle.convolve_f32(img.numpy(), mf.astype(np.float64), mode, 0.7)
+        _cmp_float(out, ref, valid if mode == "undefined" else None, tol=2e-5)
+        for odt, npdt in ((torch.uint8, np.uint8), (torch.int32, np.int32)):
+            q = lop.convolve(u8.cuda(), mi, mode, constant=9, shift=2,
+                             out_dtype=odt).cpu().numpy()
+            refq, valid = oracle.convolve_u8(u8.numpy(), mi, 2, mode, cval=9, out_dtype=npdt)
+            sel = valid if mode == "undefined" else slice(None)
+            assert (q[sel] == refq[sel]).all(), (mode, odt)
+
+
 @pytest.mark.parametrize("msize", [(3, 5), (7, 1), (1, 9), (11, 11), (15, 3)])
-def test_conv_random_masks(lop, conv_variant, msize):
+def test_conv_random_masks(lop, msize):
     rng = np.random.default_rng(msize[0] * 100 + msize[1])
     img = synthetic.uniform(45, 77, seed=1)
     u8 = synthetic.uniform_u8(45, 77, seed=2)
@@ -285,6 +306,19 @@ def test_band_views_bit_identical_to_whole_image(lop, mode):
         assert torch.equal(out, whole[y0:y1]), (y0, y1)
         og = lop.gaussian(band, 5, mode, constant=0.5, band=(top, bot, y0, H))
         assert torch.equal(og, wg[y0:y1]), (y0, y1)
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_bilateral_bands_driver_single_rank(lop, mode):
+    """dist.bilateral_bands (interior rows, then edge rows after the halo
+    exchange; ring self-copy for REPEAT) equals the whole-image call."""
+    from paper_conf_ipps_membarthhtke12_b200 import dist as ldist
+    H, W = 300, 260
+    img = synthetic.angio(H, W, seed=61).cuda()
+    band = ldist.Bands(H, W, 1, 0, 6, device="cuda", mode=mode)
+    band.fill(lambda a, b: img[a:b])
+    out = ldist.bilateral_bands(lop, band, 3.0, 0.1, mode, constant=0.5)
+    assert torch.equal(out, lop.bilateral(img, 3.0, 0.1, mode, constant=0.5))
 
 
 def test_band_validation_rejects_missing_halo(lop):

@@ -23,6 +23,16 @@ for w in $WHAT; do
     bench)
       timeout 900 python bench.py > "$OUT/bench.json" 2> "$OUT/bench.err"
       echo "bench exit $?" >> "$OUT/status.txt" ;;
+    benchalt)
+      timeout 900 python bench.py --workload frames --steps 5 --warmup 3 --no-cpu-baseline \
+        > "$OUT/bench_frames.json" 2> "$OUT/bench_frames.err"
+      echo "bench_frames exit $?" >> "$OUT/status.txt"
+      timeout 900 python bench.py --workload bands --steps 5 --warmup 3 --no-cpu-baseline \
+        > "$OUT/bench_bands.json" 2> "$OUT/bench_bands.err"
+      echo "bench_bands exit $?" >> "$OUT/status.txt"
+      timeout 600 python bench.py --impl reference --steps 3 --warmup 1 \
+        > "$OUT/bench_reference.json" 2> "$OUT/bench_reference.err"
+      echo "bench_reference exit $?" >> "$OUT/status.txt" ;;
     peaks)
       timeout 300 ./tools/peaks > "$OUT/peaks.txt" 2>&1
       echo "peaks exit $?" >> "$OUT/status.txt" ;;
