@@ -302,7 +302,7 @@ def run_lop(args, dist, peaks):
     if os.path.exists(tp):
         with open(tp) as f:
             traffic = json.load(f).get("bilateral_tiled_13x13_4096", None)
-    roofline = {"bound": "alu", "kernel": "lop::bilateral_tiled_kernel<6>",
+    roofline = {"bound": "alu", "kernel": "lop::bilateral_sep_kernel<6>",
                 "achieved": round(achieved, 4), "peak": round(peak, 4), "unit": "Tex2/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic,
                 "work_per_launch": "%d ex2 (= 168 per px x %d px)" % (ex2_per_launch,

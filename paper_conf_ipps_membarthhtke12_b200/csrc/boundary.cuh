@@ -98,6 +98,42 @@ __device__ __forceinline__ void bilateral_tap(float v, float centre, float lc, f
     p = __fmaf_rn(w, v, p);
 }
 
+// Separable-closeness form (Eq. 1 is a product of two 1D Gaussians, Listing 1
+// l.21): c(xf,yf) = cy[yf] * 2^lx[xf].  Per window row the taps accumulate
+//   rd = sum_xf w',  rp = sum_xf w' v,   w' = ex2(lx[xf] + nk * (v - centre)^2)
+// (first tap initialises), then the row is folded in with one FFMA each:
+//   d += cy[yf] * rd,  p += cy[yf] * rp.
+// Same operation count per tap as bilateral_tap, no per-tap mask operand from
+// shared memory, and per-row partial sums (better accuracy).
+__device__ __forceinline__ float bilateral_weight(float v, float centre, float lx, float nk)
+{
+    const float diff = __fsub_rn(v, centre);
+    const float t = __fmul_rn(diff, diff);
+    return ex2_approx(__fmaf_rn(t, nk, lx));
+}
+
+__device__ __forceinline__ void bilateral_row_first(float v, float centre, float lx, float nk,
+                                                    float &rd, float &rp)
+{
+    const float w = bilateral_weight(v, centre, lx, nk);
+    rd = w;
+    rp = __fmul_rn(w, v);
+}
+
+__device__ __forceinline__ void bilateral_row_tap(float v, float centre, float lx, float nk,
+                                                  float &rd, float &rp)
+{
+    const float w = bilateral_weight(v, centre, lx, nk);
+    rd = __fadd_rn(rd, w);
+    rp = __fmaf_rn(w, v, rp);
+}
+
+__device__ __forceinline__ void bilateral_row_fold(float cy, float rd, float rp, float &d, float &p)
+{
+    d = __fmaf_rn(cy, rd, d);
+    p = __fmaf_rn(cy, rp, p);
+}
+
 __device__ __forceinline__ float bilateral_finish(float d, float p)
 {
     return __fdiv_rn(p, d);   // Alg. 1 line 14: output = p / k

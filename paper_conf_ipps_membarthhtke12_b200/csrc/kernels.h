@@ -8,6 +8,7 @@ namespace lop {
 
 cudaError_t launch_bilateral_generic(const BilateralGeneric &p, cudaStream_t stream);
 cudaError_t launch_bilateral_tiled(const BilateralTiled &p, cudaStream_t stream);
+cudaError_t launch_bilateral_sep(const BilateralSep &p, cudaStream_t stream);
 cudaError_t launch_conv_generic(const ConvGeneric &p, cudaStream_t stream);
 // Tiled convolution; returns cudaErrorNotSupported when no instance matches
 // (the caller then falls back to the generic kernel).

@@ -323,6 +323,22 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
     const bool tiled_ok = c.rx <= lop::kTiledMaxRX;
     if (variant == LOP_VARIANT_TILED && !tiled_ok)
         return fail(LOP_ERR_UNSUPPORTED, "no tiled bilateral instance for window width %d", sx);
+    // Closeness from sigma_d (Eq. 1) is separable: c = cy[yf] * 2^lx[xf]
+    // (Listing 1 l.21: exp(-c_d xf^2) * exp(-c_d yf^2)).
+    float lx[2 * lop::kMaxRadius + 1], cy[2 * lop::kMaxRadius + 1];
+    if (!closeness) {
+        const double c_d = 1.0 / (2.0 * (double)sigma_d * (double)sigma_d);
+        for (int xf = -c.rx; xf <= c.rx; ++xf) lx[xf + c.rx] = (float)(-c_d * (double)(xf * xf) * kLog2e);
+        for (int yf = -c.ry; yf <= c.ry; ++yf) cy[yf + c.ry] = (float)std::exp(-c_d * (double)(yf * yf));
+    }
+    if (variant != LOP_VARIANT_GENERIC && tiled_ok && !closeness) {
+        static thread_local lop::BilateralSep p;
+        p.c = c;
+        p.nk = nk;
+        std::memcpy(p.lx, lx, sizeof(float) * sx);
+        std::memcpy(p.cy, cy, sizeof(float) * sy);
+        return launched(lop::launch_bilateral_sep(p, stream), "bilateral_sep launch");
+    }
     if (variant != LOP_VARIANT_GENERIC && tiled_ok) {
         static thread_local lop::BilateralTiled p;
         p.c = c;
@@ -335,7 +351,13 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
     static thread_local lop::BilateralGeneric p;
     p.c = c;
     p.nk = nk;
-    std::memcpy(p.lc, lc.get(), sizeof(float) * sx * sy);
+    p.sep = closeness ? 0 : 1;
+    if (closeness) {
+        std::memcpy(p.lc, lc.get(), sizeof(float) * sx * sy);
+    } else {
+        std::memcpy(p.lx, lx, sizeof(float) * sx);
+        std::memcpy(p.cy, cy, sizeof(float) * sy);
+    }
     return launched(lop::launch_bilateral_generic(p, stream), "bilateral_generic launch");
 }
 

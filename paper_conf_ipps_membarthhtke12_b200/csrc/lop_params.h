@@ -45,10 +45,21 @@ constexpr int kTiledMaxTaps = (2 * kMaxRadius + 1) * kTiledMaskPitch;
 
 // Bilateral: weight w = ex2(lc[tap] + nk * (v - centre)^2)
 //   lc[tap] = log2 c(xf, yf), nk = -log2(e) / (2 sigma_r^2)
+// sep = 1 (closeness from sigma_d, Eq. 1): c(xf,yf) = cy[yf] * 2^lx[xf] and the
+// kernels use the per-row folded form (boundary.cuh bilateral_row_*).
 struct BilateralGeneric {
     Common c;
     float nk;
+    int32_t sep;
+    float lx[2 * kMaxRadius + 1];
+    float cy[2 * kMaxRadius + 1];
     float lc[kMaxTaps];
+};
+struct BilateralSep {
+    Common c;
+    float nk;
+    float lx[2 * kTiledMaxRX + 1];   // log2 of the x factor (compile-time indexed)
+    float cy[2 * kMaxRadius + 1];    // linear y factor
 };
 struct BilateralTiled {
     Common c;

@@ -43,7 +43,7 @@ for w in $WHAT; do
       echo "ncu exit $?" >> "$OUT/status.txt" ;;
     full)
       timeout 900 ncu --set full --clock-control none --import-source on \
-        -k regex:bilateral_tiled -s 3 -c 1 -o "$OUT/prof_bilateral" -f \
+        -k regex:bilateral_ -s 3 -c 1 -o "$OUT/prof_bilateral" -f \
         python bench.py --steps 5 --warmup 3 --no-extras --no-cpu-baseline --e2e-steps 0 \
         > "$OUT/ncu_full.log" 2>&1
       echo "full exit $?" >> "$OUT/status.txt" ;;
