@@ -53,8 +53,15 @@ __global__ void __launch_bounds__(256) bilateral_generic_kernel(const __grid_con
                 int col;
                 float v = c.cval_f;
                 if (row_ok && resolve_col(ix + xf, c.in, c.mode, col)) v = __ldg(rp + col);
-                if (xf == -c.rx) bilateral_row_first(v, centre, p.lx[xf + c.rx], p.nk, rd, rpp);
-                else bilateral_row_tap(v, centre, p.lx[xf + c.rx], p.nk, rd, rpp);
+                const float lx = p.lx[xf + c.rx];
+                const bool poly = xf + c.rx < p.npoly;
+                if (xf == -c.rx) {
+                    if (poly) bilateral_row_first<true>(v, centre, lx, p.nk, rd, rpp);
+                    else bilateral_row_first<false>(v, centre, lx, p.nk, rd, rpp);
+                } else {
+                    if (poly) bilateral_row_tap<true>(v, centre, lx, p.nk, rd, rpp);
+                    else bilateral_row_tap<false>(v, centre, lx, p.nk, rd, rpp);
+                }
             }
             bilateral_row_fold(p.cy[yf + c.ry], rd, rpp, d, pacc);
         } else {
@@ -219,23 +226,28 @@ __global__ void __launch_bounds__(tiled::NT, 4) bilateral_tiled_kernel(const __g
 // -------------------------------------- separable-closeness tiled kernel
 // One window row of taps for the 4 outputs of a thread (lx from the
 // constant bank, compile-time indexed), folded with cy.
-template <int RX, int VOFF>
+template <int RX, int VOFF, int NP>
 __device__ __forceinline__ void sep_row(const float *v, const float cen[4], const float *lx,
                                         float nk, float cy, float d[4], float pp[4])
 {
     float rd[4], rp[4];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) bilateral_row_first(v[VOFF + j], cen[j], lx[0], nk, rd[j], rp[j]);
+    for (int j = 0; j < 4; ++j)
+        bilateral_row_first<(NP > 0)>(v[VOFF + j], cen[j], lx[0], nk, rd[j], rp[j]);
 #pragma unroll
     for (int xf = 1; xf <= 2 * RX; ++xf)
 #pragma unroll
-        for (int j = 0; j < 4; ++j)
-            bilateral_row_tap(v[VOFF + xf + j], cen[j], lx[xf], nk, rd[j], rp[j]);
+        for (int j = 0; j < 4; ++j) {
+            if (xf < NP)   // resolved at compile time after unrolling
+                bilateral_row_tap<true>(v[VOFF + xf + j], cen[j], lx[xf], nk, rd[j], rp[j]);
+            else
+                bilateral_row_tap<false>(v[VOFF + xf + j], cen[j], lx[xf], nk, rd[j], rp[j]);
+        }
 #pragma unroll
     for (int j = 0; j < 4; ++j) bilateral_row_fold(cy, rd[j], rp[j], d[j], pp[j]);
 }
 
-template <int RX>
+template <int RX, int NP>
 __global__ void __launch_bounds__(tiled::NT, 3) bilateral_sep_kernel(const __grid_constant__ BilateralSep p)
 {
     using S = tiled::Shape<RX>;
@@ -276,16 +288,16 @@ __global__ void __launch_bounds__(tiled::NT, 3) bilateral_sep_kernel(const __gri
         float v[4 * NV];
         // staged row 0: window row 0 of output r0 only
         load_row<NV>(rowv, v);
-        sep_row<RX, S::VOFF>(v, cen0, p.lx, nk, scy[0], d0, p0);
+        sep_row<RX, S::VOFF, NP>(v, cen0, p.lx, nk, scy[0], d0, p0);
 #pragma unroll 1
         for (int r = 1; r <= 2 * ry; ++r) {
             load_row<NV>(rowv + r * (SW / 4), v);
-            sep_row<RX, S::VOFF>(v, cen0, p.lx, nk, scy[r], d0, p0);       // output r0, yf = r
-            sep_row<RX, S::VOFF>(v, cen1, p.lx, nk, scy[r - 1], d1, p1);   // output r0+1, yf = r-1
+            sep_row<RX, S::VOFF, NP>(v, cen0, p.lx, nk, scy[r], d0, p0);       // output r0, yf = r
+            sep_row<RX, S::VOFF, NP>(v, cen1, p.lx, nk, scy[r - 1], d1, p1);   // output r0+1, yf = r-1
         }
         // staged row 2ry+1: last window row of output r0+1
         load_row<NV>(rowv + (2 * ry + 1) * (SW / 4), v);
-        sep_row<RX, S::VOFF>(v, cen1, p.lx, nk, scy[2 * ry], d1, p1);
+        sep_row<RX, S::VOFF, NP>(v, cen1, p.lx, nk, scy[2 * ry], d1, p1);
         float res[4];
 #pragma unroll
         for (int j = 0; j < 4; ++j) res[j] = bilateral_finish(d0[j], p0[j]);
@@ -325,15 +337,34 @@ static cudaError_t launch_tiled_rx(const BilateralTiled &p, cudaStream_t stream)
     return launch_tiled(bilateral_tiled_kernel<RX>, p, smem, stream, configured);
 }
 
-template <int RX>
-static cudaError_t launch_sep_rx(const BilateralSep &p, cudaStream_t stream)
+template <int RX, int NP>
+static cudaError_t launch_sep_rx_np(const BilateralSep &p, cudaStream_t stream)
 {
     using S = tiled::Shape<RX>;
     static size_t configured = 0;
     const size_t smem = (size_t)((tiled::TH + 2 * p.c.ry) * S::SW + ((2 * p.c.ry + 1 + 3) & ~3)) *
                         sizeof(float);
-    return launch_tiled(bilateral_sep_kernel<RX>, p, smem, stream, configured);
+    return launch_tiled(bilateral_sep_kernel<RX, NP>, p, smem, stream, configured);
 }
+
+// npoly instances: 0 for every width; 1..3 for windows >= 9 wide, where the
+// FMA pipe has the issue headroom to absorb the emulated exps.
+template <int RX>
+static cudaError_t launch_sep_rx(const BilateralSep &p, cudaStream_t stream)
+{
+    if constexpr (RX >= 4) {
+        switch (p.npoly) {
+        case 0: return launch_sep_rx_np<RX, 0>(p, stream);
+        case 1: return launch_sep_rx_np<RX, 1>(p, stream);
+        case 2: return launch_sep_rx_np<RX, 2>(p, stream);
+        case 3: return launch_sep_rx_np<RX, 3>(p, stream);
+        default: return cudaErrorInvalidValue;
+        }
+    }
+    return p.npoly == 0 ? launch_sep_rx_np<RX, 0>(p, stream) : cudaErrorInvalidValue;
+}
+
+int bilateral_sep_max_npoly(int rx) { return rx >= 4 ? 3 : 0; }
 
 cudaError_t launch_bilateral_tiled(const BilateralTiled &p, cudaStream_t stream)
 {

@@ -98,6 +98,25 @@ __device__ __forceinline__ void bilateral_tap(float v, float centre, float lc, f
     p = __fmaf_rn(w, v, p);
 }
 
+// 2^x on the FMA pipe (Cody-Waite split + degree-5 polynomial), used for a
+// fixed subset of taps to offload the MUFU (SFU) pipe, which bounds the
+// bilateral kernel.  x <= 0 here (log2 of a product of weights <= 1); values
+// below -126 return 2^-126 (weights that small are below f32 resolution of the
+// sums).  Relative error <= 2.1e-7 in f32 (ex2.approx: <= 2^-22 ~ 2.4e-7).
+__device__ __forceinline__ float ex2_poly(float x)
+{
+    x = fmaxf(x, -126.0f);
+    const float t = __fadd_rn(x, 12582912.0f);          // 1.5 * 2^23: j = round(x) in the low bits
+    const float j = __fsub_rn(t, 12582912.0f);
+    const float f = __fsub_rn(x, j);                    // f in [-0.5, 0.5]
+    float p = __fmaf_rn(1.3277444522827864e-3f, f, 9.675883688032627e-3f);
+    p = __fmaf_rn(p, f, 5.550713092088699e-2f);
+    p = __fmaf_rn(p, f, 2.4022112786769867e-1f);
+    p = __fmaf_rn(p, f, 6.931469440460205e-1f);
+    p = __fmaf_rn(p, f, 1.0000001192092896f);
+    return __int_as_float(__float_as_int(p) + (__float_as_int(t) << 23));   // p * 2^j
+}
+
 // Separable-closeness form (Eq. 1 is a product of two 1D Gaussians, Listing 1
 // l.21): c(xf,yf) = cy[yf] * 2^lx[xf].  Per window row the taps accumulate
 //   rd = sum_xf w',  rp = sum_xf w' v,   w' = ex2(lx[xf] + nk * (v - centre)^2)
@@ -105,25 +124,29 @@ __device__ __forceinline__ void bilateral_tap(float v, float centre, float lc, f
 //   d += cy[yf] * rd,  p += cy[yf] * rp.
 // Same operation count per tap as bilateral_tap, no per-tap mask operand from
 // shared memory, and per-row partial sums (better accuracy).
+template <bool POLY = false>
 __device__ __forceinline__ float bilateral_weight(float v, float centre, float lx, float nk)
 {
     const float diff = __fsub_rn(v, centre);
     const float t = __fmul_rn(diff, diff);
-    return ex2_approx(__fmaf_rn(t, nk, lx));
+    const float e = __fmaf_rn(t, nk, lx);
+    return POLY ? ex2_poly(e) : ex2_approx(e);
 }
 
+template <bool POLY = false>
 __device__ __forceinline__ void bilateral_row_first(float v, float centre, float lx, float nk,
                                                     float &rd, float &rp)
 {
-    const float w = bilateral_weight(v, centre, lx, nk);
+    const float w = bilateral_weight<POLY>(v, centre, lx, nk);
     rd = w;
     rp = __fmul_rn(w, v);
 }
 
+template <bool POLY = false>
 __device__ __forceinline__ void bilateral_row_tap(float v, float centre, float lx, float nk,
                                                   float &rd, float &rp)
 {
-    const float w = bilateral_weight(v, centre, lx, nk);
+    const float w = bilateral_weight<POLY>(v, centre, lx, nk);
     rd = __fadd_rn(rd, w);
     rp = __fmaf_rn(w, v, rp);
 }

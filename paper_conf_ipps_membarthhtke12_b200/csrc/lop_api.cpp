@@ -5,10 +5,12 @@
 
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <atomic>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <memory>
 #include <string>
@@ -49,6 +51,7 @@ int elem_size(int32_t dt)
 }
 
 const double kLog2e = 1.4426950408889634073599246810019;
+const int kDefaultNpoly = 1;   // see DESIGN.md §6 (MUFU offload)
 
 // ---------------------------------------------------------------- validation
 lop_status check_image(const lop_image &im, const char *name)
@@ -331,10 +334,19 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
         for (int xf = -c.rx; xf <= c.rx; ++xf) lx[xf + c.rx] = (float)(-c_d * (double)(xf * xf) * kLog2e);
         for (int yf = -c.ry; yf <= c.ry; ++yf) cy[yf + c.ry] = (float)std::exp(-c_d * (double)(yf * yf));
     }
+    // window columns whose exp runs on the FMA pipe (ex2_poly) instead of the
+    // MUFU: tuned on B200; LOP_BILATERAL_NPOLY overrides
+    int npoly = 0;
+    if (!closeness) {
+        npoly = c.rx >= 4 ? kDefaultNpoly : 0;
+        if (const char *env = std::getenv("LOP_BILATERAL_NPOLY")) npoly = std::atoi(env);
+        npoly = std::max(0, std::min(npoly, lop::bilateral_sep_max_npoly(c.rx)));
+    }
     if (variant != LOP_VARIANT_GENERIC && tiled_ok && !closeness) {
         static thread_local lop::BilateralSep p;
         p.c = c;
         p.nk = nk;
+        p.npoly = npoly;
         std::memcpy(p.lx, lx, sizeof(float) * sx);
         std::memcpy(p.cy, cy, sizeof(float) * sy);
         return launched(lop::launch_bilateral_sep(p, stream), "bilateral_sep launch");
@@ -352,6 +364,7 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
     p.c = c;
     p.nk = nk;
     p.sep = closeness ? 0 : 1;
+    p.npoly = npoly;
     if (closeness) {
         std::memcpy(p.lc, lc.get(), sizeof(float) * sx * sy);
     } else {

@@ -51,6 +51,7 @@ struct BilateralGeneric {
     Common c;
     float nk;
     int32_t sep;
+    int32_t npoly;                   // sep form: columns xf = -rx .. -rx+npoly-1 use ex2_poly
     float lx[2 * kMaxRadius + 1];
     float cy[2 * kMaxRadius + 1];
     float lc[kMaxTaps];
@@ -58,6 +59,7 @@ struct BilateralGeneric {
 struct BilateralSep {
     Common c;
     float nk;
+    int32_t npoly;                   // leftmost npoly window columns use ex2_poly (FMA pipe)
     float lx[2 * kTiledMaxRX + 1];   // log2 of the x factor (compile-time indexed)
     float cy[2 * kMaxRadius + 1];    // linear y factor
 };

@@ -127,6 +127,23 @@ def test_bilateral_generic_and_tiled_bit_identical(lop):
             assert torch.equal(a, b), (mode, size)
 
 
+@pytest.mark.parametrize("npoly", ["0", "1", "2", "3"])
+def test_bilateral_mufu_offload_settings(lop, npoly, monkeypatch):
+    """Every MUFU-offload setting (exp of the leftmost window columns on the FMA
+    pipe) stays within tolerance of the oracle and generic == tiled bit for bit."""
+    monkeypatch.setenv("LOP_BILATERAL_NPOLY", npoly)
+    img = synthetic.angio(150, 300, seed=13)
+    for sigma_r in (5.0, 0.1, 0.02):
+        lop.set_variant("generic")
+        a = lop.bilateral(img.cuda(), 3.0, sigma_r, "mirror")
+        lop.set_variant("tiled")
+        b = lop.bilateral(img.cuda(), 3.0, sigma_r, "mirror")
+        lop.set_variant("auto")
+        assert torch.equal(a, b)
+        ref, _ = oracle.bilateral_f32(img.numpy(), 3.0, sigma_r, "mirror")
+        _cmp_float(b.cpu().numpy(), ref)
+
+
 def test_config1_bilateral_256_clamp(lop):
     """BASELINE config 1: 256x256 f32, sigma_d = 1 (3x3), sigma_r = 5, clamp."""
     img = synthetic.angio(256, 256, seed=synthetic.config_seed(1))
