@@ -40,7 +40,9 @@ __global__ void __launch_bounds__(256) bilateral_generic_kernel(const __grid_con
     const int ix = ox + c.off_x, iy = oy + c.off_y;
     // centre Input(): the pixel itself (for offset accessors it is read
     // through the boundary condition like every other tap)
-    const float centre = read_f32(c.in, b, ix, iy, c.mode, c.cval_f);
+    const bool sc = p.sep && p.scaled;
+    float centre = read_f32(c.in, b, ix, iy, c.mode, c.cval_f);
+    if (sc) centre = __fmul_rn(centre, p.alpha);
     const int sx = 2 * c.rx + 1;
     float d = 0.0f, pacc = 0.0f;
     for (int yf = -c.ry; yf <= c.ry; ++yf) {
@@ -55,7 +57,11 @@ __global__ void __launch_bounds__(256) bilateral_generic_kernel(const __grid_con
                 if (row_ok && resolve_col(ix + xf, c.in, c.mode, col)) v = __ldg(rp + col);
                 const float lx = p.lx[xf + c.rx];
                 const bool poly = xf + c.rx < p.npoly;
-                if (xf == -c.rx) {
+                if (sc) {
+                    v = __fmul_rn(v, p.alpha);
+                    if (xf == -c.rx) bilateral_row_first<false, true>(v, centre, lx, p.nk, rd, rpp);
+                    else bilateral_row_tap<false, true>(v, centre, lx, p.nk, rd, rpp);
+                } else if (xf == -c.rx) {
                     if (poly) bilateral_row_first<true>(v, centre, lx, p.nk, rd, rpp);
                     else bilateral_row_first<false>(v, centre, lx, p.nk, rd, rpp);
                 } else {
@@ -76,7 +82,7 @@ __global__ void __launch_bounds__(256) bilateral_generic_kernel(const __grid_con
     }
     float *orow = reinterpret_cast<float *>(c.out.data + (int64_t)b * c.out.bstride +
                                             (int64_t)oy * c.out.stride);
-    orow[ox] = bilateral_finish(d, pacc);
+    orow[ox] = sc ? bilateral_finish_scaled(d, pacc, p.inv_alpha) : bilateral_finish(d, pacc);
 }
 
 cudaError_t launch_bilateral_generic(const BilateralGeneric &p, cudaStream_t stream)
@@ -107,9 +113,11 @@ template <int RX> struct Shape {
 // handling is resolved here, once per staged pixel (§8(a) a2/a3).  Only the
 // rows the tile's outputs need are staged (a partial last tile must not touch
 // rows beyond the validated band + halo).
-template <int SW>
+// SCALE: store alpha * I (the range-scaled values of the scaled-difference
+// form, boundary.cuh bilateral_weight_scaled) instead of I.
+template <int SW, bool SCALE = false>
 __device__ __forceinline__ void stage_tile(const Common &c, int b, int ix0, int iy0, int srows,
-                                           float *tile)
+                                           float *tile, float alpha = 1.0f)
 {
     constexpr int NT = tiled::NT;
     const Geom &g = c.in;
@@ -124,18 +132,25 @@ __device__ __forceinline__ void stage_tile(const Common &c, int b, int ix0, int 
             const int r = i / V, v = i - r * V;
             const float4 *src = reinterpret_cast<const float4 *>(
                 fbase + (int64_t)(iy0 + r) * g.stride) + (ix0 >> 2) + v;
-            t4[r * V + v] = __ldg(src);
+            float4 q = __ldg(src);
+            if (SCALE) {
+                q.x = __fmul_rn(q.x, alpha); q.y = __fmul_rn(q.y, alpha);
+                q.z = __fmul_rn(q.z, alpha); q.w = __fmul_rn(q.w, alpha);
+            }
+            t4[r * V + v] = q;
         }
     } else if (interior) {
         for (int i = threadIdx.x; i < srows * SW; i += NT) {
             const int r = i / SW, x = i - r * SW;
-            tile[i] = __ldg(reinterpret_cast<const float *>(fbase + (int64_t)(iy0 + r) * g.stride) +
-                            ix0 + x);
+            const float q = __ldg(reinterpret_cast<const float *>(fbase + (int64_t)(iy0 + r) * g.stride) +
+                                  ix0 + x);
+            tile[i] = SCALE ? __fmul_rn(q, alpha) : q;
         }
     } else {
         for (int i = threadIdx.x; i < srows * SW; i += NT) {
             const int r = i / SW, x = i - r * SW;
-            tile[i] = read_f32(g, b, ix0 + x, iy0 + r, c.mode, c.cval_f);
+            const float q = read_f32(g, b, ix0 + x, iy0 + r, c.mode, c.cval_f);
+            tile[i] = SCALE ? __fmul_rn(q, alpha) : q;
         }
     }
 }
@@ -226,28 +241,28 @@ __global__ void __launch_bounds__(tiled::NT, 4) bilateral_tiled_kernel(const __g
 // -------------------------------------- separable-closeness tiled kernel
 // One window row of taps for the 4 outputs of a thread (lx from the
 // constant bank, compile-time indexed), folded with cy.
-template <int RX, int VOFF, int NP>
+template <int RX, int VOFF, int NP, bool SC>
 __device__ __forceinline__ void sep_row(const float *v, const float cen[4], const float *lx,
                                         float nk, float cy, float d[4], float pp[4])
 {
     float rd[4], rp[4];
 #pragma unroll
     for (int j = 0; j < 4; ++j)
-        bilateral_row_first<(NP > 0)>(v[VOFF + j], cen[j], lx[0], nk, rd[j], rp[j]);
+        bilateral_row_first<(NP > 0), SC>(v[VOFF + j], cen[j], lx[0], nk, rd[j], rp[j]);
 #pragma unroll
     for (int xf = 1; xf <= 2 * RX; ++xf)
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
             if (xf < NP)   // resolved at compile time after unrolling
-                bilateral_row_tap<true>(v[VOFF + xf + j], cen[j], lx[xf], nk, rd[j], rp[j]);
+                bilateral_row_tap<true, SC>(v[VOFF + xf + j], cen[j], lx[xf], nk, rd[j], rp[j]);
             else
-                bilateral_row_tap<false>(v[VOFF + xf + j], cen[j], lx[xf], nk, rd[j], rp[j]);
+                bilateral_row_tap<false, SC>(v[VOFF + xf + j], cen[j], lx[xf], nk, rd[j], rp[j]);
         }
 #pragma unroll
     for (int j = 0; j < 4; ++j) bilateral_row_fold(cy, rd[j], rp[j], d[j], pp[j]);
 }
 
-template <int RX, int NP>
+template <int RX, int NP, bool SC>
 __global__ void __launch_bounds__(tiled::NT, 3) bilateral_sep_kernel(const __grid_constant__ BilateralSep p)
 {
     using S = tiled::Shape<RX>;
@@ -267,8 +282,8 @@ __global__ void __launch_bounds__(tiled::NT, 3) bilateral_sep_kernel(const __gri
     const int roi_y1 = c.roi_y0 + c.roi_h;
 
     for (int i = threadIdx.x; i <= 2 * ry; i += NT) scy[i] = p.cy[i];
-    stage_tile<SW>(c, b, tx0 + c.off_x - PAD, ty0 + c.off_y - ry, min(TH, roi_y1 - ty0) + 2 * ry,
-                   tile);
+    stage_tile<SW, SC>(c, b, tx0 + c.off_x - PAD, ty0 + c.off_y - ry,
+                       min(TH, roi_y1 - ty0) + 2 * ry, tile, p.alpha);
     __syncthreads();
 
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -288,23 +303,25 @@ __global__ void __launch_bounds__(tiled::NT, 3) bilateral_sep_kernel(const __gri
         float v[4 * NV];
         // staged row 0: window row 0 of output r0 only
         load_row<NV>(rowv, v);
-        sep_row<RX, S::VOFF, NP>(v, cen0, p.lx, nk, scy[0], d0, p0);
+        sep_row<RX, S::VOFF, NP, SC>(v, cen0, p.lx, nk, scy[0], d0, p0);
 #pragma unroll 1
         for (int r = 1; r <= 2 * ry; ++r) {
             load_row<NV>(rowv + r * (SW / 4), v);
-            sep_row<RX, S::VOFF, NP>(v, cen0, p.lx, nk, scy[r], d0, p0);       // output r0, yf = r
-            sep_row<RX, S::VOFF, NP>(v, cen1, p.lx, nk, scy[r - 1], d1, p1);   // output r0+1, yf = r-1
+            sep_row<RX, S::VOFF, NP, SC>(v, cen0, p.lx, nk, scy[r], d0, p0);       // output r0, yf = r
+            sep_row<RX, S::VOFF, NP, SC>(v, cen1, p.lx, nk, scy[r - 1], d1, p1);   // output r0+1, yf = r-1
         }
         // staged row 2ry+1: last window row of output r0+1
         load_row<NV>(rowv + (2 * ry + 1) * (SW / 4), v);
-        sep_row<RX, S::VOFF, NP>(v, cen1, p.lx, nk, scy[2 * ry], d1, p1);
+        sep_row<RX, S::VOFF, NP, SC>(v, cen1, p.lx, nk, scy[2 * ry], d1, p1);
         float res[4];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) res[j] = bilateral_finish(d0[j], p0[j]);
+        for (int j = 0; j < 4; ++j)
+            res[j] = SC ? bilateral_finish_scaled(d0[j], p0[j], p.inv_alpha) : bilateral_finish(d0[j], p0[j]);
         store4(c, b, oy, x_out, res);
         if (oy + 1 < roi_y1) {
 #pragma unroll
-            for (int j = 0; j < 4; ++j) res[j] = bilateral_finish(d1[j], p1[j]);
+            for (int j = 0; j < 4; ++j)
+                res[j] = SC ? bilateral_finish_scaled(d1[j], p1[j], p.inv_alpha) : bilateral_finish(d1[j], p1[j]);
             store4(c, b, oy + 1, x_out, res);
         }
     }
@@ -337,34 +354,31 @@ static cudaError_t launch_tiled_rx(const BilateralTiled &p, cudaStream_t stream)
     return launch_tiled(bilateral_tiled_kernel<RX>, p, smem, stream, configured);
 }
 
-template <int RX, int NP>
+template <int RX, int NP, bool SC>
 static cudaError_t launch_sep_rx_np(const BilateralSep &p, cudaStream_t stream)
 {
     using S = tiled::Shape<RX>;
     static size_t configured = 0;
     const size_t smem = (size_t)((tiled::TH + 2 * p.c.ry) * S::SW + ((2 * p.c.ry + 1 + 3) & ~3)) *
                         sizeof(float);
-    return launch_tiled(bilateral_sep_kernel<RX, NP>, p, smem, stream, configured);
+    return launch_tiled(bilateral_sep_kernel<RX, NP, SC>, p, smem, stream, configured);
 }
 
-// npoly instances: 0 for every width; 1..3 for windows >= 9 wide, where the
-// FMA pipe has the issue headroom to absorb the emulated exps.
+// instances: npoly 0 (scaled or not) for every width; npoly 1 (unscaled) for
+// windows >= 9 wide (kept for the tuning sweep).
 template <int RX>
 static cudaError_t launch_sep_rx(const BilateralSep &p, cudaStream_t stream)
 {
+    if (p.npoly == 0)
+        return p.scaled ? launch_sep_rx_np<RX, 0, true>(p, stream)
+                        : launch_sep_rx_np<RX, 0, false>(p, stream);
     if constexpr (RX >= 4) {
-        switch (p.npoly) {
-        case 0: return launch_sep_rx_np<RX, 0>(p, stream);
-        case 1: return launch_sep_rx_np<RX, 1>(p, stream);
-        case 2: return launch_sep_rx_np<RX, 2>(p, stream);
-        case 3: return launch_sep_rx_np<RX, 3>(p, stream);
-        default: return cudaErrorInvalidValue;
-        }
+        if (p.npoly == 1 && !p.scaled) return launch_sep_rx_np<RX, 1, false>(p, stream);
     }
-    return p.npoly == 0 ? launch_sep_rx_np<RX, 0>(p, stream) : cudaErrorInvalidValue;
+    return cudaErrorInvalidValue;
 }
 
-int bilateral_sep_max_npoly(int rx) { return rx >= 4 ? 3 : 0; }
+int bilateral_sep_max_npoly(int rx) { return rx >= 4 ? 1 : 0; }
 
 cudaError_t launch_bilateral_tiled(const BilateralTiled &p, cudaStream_t stream)
 {

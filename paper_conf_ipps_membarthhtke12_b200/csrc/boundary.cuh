@@ -124,31 +124,45 @@ __device__ __forceinline__ float ex2_poly(float x)
 //   d += cy[yf] * rd,  p += cy[yf] * rp.
 // Same operation count per tap as bilateral_tap, no per-tap mask operand from
 // shared memory, and per-row partial sums (better accuracy).
-template <bool POLY = false>
+// SCALED = scaled-difference form: v and centre are alpha * I with
+// alpha^2 = log2(e) / (2 sigma_r^2), so the exponent is lx - (v - centre)^2
+// (one FFMA with a negated operand, no FMUL); p then accumulates alpha * I and
+// the result is divided by alpha at the end (bilateral_finish_scaled).
+template <bool POLY = false, bool SCALED = false>
 __device__ __forceinline__ float bilateral_weight(float v, float centre, float lx, float nk)
 {
     const float diff = __fsub_rn(v, centre);
-    const float t = __fmul_rn(diff, diff);
-    const float e = __fmaf_rn(t, nk, lx);
+    float e;
+    if (SCALED) {
+        e = __fmaf_rn(-diff, diff, lx);
+    } else {
+        const float t = __fmul_rn(diff, diff);
+        e = __fmaf_rn(t, nk, lx);
+    }
     return POLY ? ex2_poly(e) : ex2_approx(e);
 }
 
-template <bool POLY = false>
+template <bool POLY = false, bool SCALED = false>
 __device__ __forceinline__ void bilateral_row_first(float v, float centre, float lx, float nk,
                                                     float &rd, float &rp)
 {
-    const float w = bilateral_weight<POLY>(v, centre, lx, nk);
+    const float w = bilateral_weight<POLY, SCALED>(v, centre, lx, nk);
     rd = w;
     rp = __fmul_rn(w, v);
 }
 
-template <bool POLY = false>
+template <bool POLY = false, bool SCALED = false>
 __device__ __forceinline__ void bilateral_row_tap(float v, float centre, float lx, float nk,
                                                   float &rd, float &rp)
 {
-    const float w = bilateral_weight<POLY>(v, centre, lx, nk);
+    const float w = bilateral_weight<POLY, SCALED>(v, centre, lx, nk);
     rd = __fadd_rn(rd, w);
     rp = __fmaf_rn(w, v, rp);
+}
+
+__device__ __forceinline__ float bilateral_finish_scaled(float d, float p, float inv_alpha)
+{
+    return __fmul_rn(__fdiv_rn(p, d), inv_alpha);
 }
 
 __device__ __forceinline__ void bilateral_row_fold(float cy, float rd, float rp, float &d, float &p)

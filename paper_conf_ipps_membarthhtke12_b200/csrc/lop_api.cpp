@@ -51,7 +51,8 @@ int elem_size(int32_t dt)
 }
 
 const double kLog2e = 1.4426950408889634073599246810019;
-const int kDefaultNpoly = 1;   // see DESIGN.md §6 (MUFU offload)
+const int kDefaultNpoly = 0;   // MUFU offload: slower on B200, kept for tuning
+const int kDefaultScaled = 0;  // scaled-difference exponent
 
 // ---------------------------------------------------------------- validation
 lop_status check_image(const lop_image &im, const char *name)
@@ -342,11 +343,23 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
         if (const char *env = std::getenv("LOP_BILATERAL_NPOLY")) npoly = std::atoi(env);
         npoly = std::max(0, std::min(npoly, lop::bilateral_sep_max_npoly(c.rx)));
     }
+    // scaled-difference exponent: LOP_BILATERAL_SCALED overrides
+    int scaled = 0;
+    if (!closeness) {
+        scaled = kDefaultScaled;
+        if (const char *env = std::getenv("LOP_BILATERAL_SCALED")) scaled = std::atoi(env) != 0;
+        if (scaled) npoly = 0;
+    }
+    const double alpha_d = std::sqrt(kLog2e / (2.0 * (double)sigma_r * (double)sigma_r));
+    const float alpha = (float)alpha_d, inv_alpha = (float)(1.0 / alpha_d);
     if (variant != LOP_VARIANT_GENERIC && tiled_ok && !closeness) {
         static thread_local lop::BilateralSep p;
         p.c = c;
         p.nk = nk;
         p.npoly = npoly;
+        p.scaled = scaled;
+        p.alpha = alpha;
+        p.inv_alpha = inv_alpha;
         std::memcpy(p.lx, lx, sizeof(float) * sx);
         std::memcpy(p.cy, cy, sizeof(float) * sy);
         return launched(lop::launch_bilateral_sep(p, stream), "bilateral_sep launch");
@@ -365,6 +378,9 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
     p.nk = nk;
     p.sep = closeness ? 0 : 1;
     p.npoly = npoly;
+    p.scaled = scaled;
+    p.alpha = alpha;
+    p.inv_alpha = inv_alpha;
     if (closeness) {
         std::memcpy(p.lc, lc.get(), sizeof(float) * sx * sy);
     } else {

@@ -52,6 +52,8 @@ struct BilateralGeneric {
     float nk;
     int32_t sep;
     int32_t npoly;                   // sep form: columns xf = -rx .. -rx+npoly-1 use ex2_poly
+    int32_t scaled;                  // sep form: scaled-difference exponent (alpha * I)
+    float alpha, inv_alpha;
     float lx[2 * kMaxRadius + 1];
     float cy[2 * kMaxRadius + 1];
     float lc[kMaxTaps];
@@ -60,6 +62,8 @@ struct BilateralSep {
     Common c;
     float nk;
     int32_t npoly;                   // leftmost npoly window columns use ex2_poly (FMA pipe)
+    int32_t scaled;                  // stage alpha * I; exponent lx - (J - J0)^2
+    float alpha, inv_alpha;          // alpha = sqrt(log2(e) / (2 sigma_r^2))
     float lx[2 * kTiledMaxRX + 1];   // log2 of the x factor (compile-time indexed)
     float cy[2 * kMaxRadius + 1];    // linear y factor
 };

@@ -127,21 +127,28 @@ def test_bilateral_generic_and_tiled_bit_identical(lop):
             assert torch.equal(a, b), (mode, size)
 
 
-@pytest.mark.parametrize("npoly", ["0", "1", "2", "3"])
-def test_bilateral_mufu_offload_settings(lop, npoly, monkeypatch):
-    """Every MUFU-offload setting (exp of the leftmost window columns on the FMA
-    pipe) stays within tolerance of the oracle and generic == tiled bit for bit."""
+@pytest.mark.parametrize("npoly,scaled", [("0", "0"), ("1", "0"), ("0", "1")])
+def test_bilateral_kernel_settings(lop, npoly, scaled, monkeypatch):
+    """Every tuning setting of the separable-closeness kernel (MUFU offload of
+    the leftmost window columns; scaled-difference exponent) stays within
+    tolerance of the oracle and generic == tiled bit for bit."""
     monkeypatch.setenv("LOP_BILATERAL_NPOLY", npoly)
-    img = synthetic.angio(150, 300, seed=13)
-    for sigma_r in (5.0, 0.1, 0.02):
-        lop.set_variant("generic")
-        a = lop.bilateral(img.cuda(), 3.0, sigma_r, "mirror")
-        lop.set_variant("tiled")
-        b = lop.bilateral(img.cuda(), 3.0, sigma_r, "mirror")
-        lop.set_variant("auto")
-        assert torch.equal(a, b)
-        ref, _ = oracle.bilateral_f32(img.numpy(), 3.0, sigma_r, "mirror")
-        _cmp_float(b.cpu().numpy(), ref)
+    monkeypatch.setenv("LOP_BILATERAL_SCALED", scaled)
+    images = (synthetic.angio(150, 300, seed=13),
+              synthetic.levels(150, 300, seed=14, values=(0.2, 0.25, 0.3, 0.8)),
+              synthetic.uniform(150, 300, seed=15))
+    worst = 0.0
+    for img in images:
+        for sigma_r in (5.0, 0.1, 0.05, 0.02, 0.01):
+            lop.set_variant("generic")
+            a = lop.bilateral(img.cuda(), 3.0, sigma_r, "mirror")
+            lop.set_variant("tiled")
+            b = lop.bilateral(img.cuda(), 3.0, sigma_r, "mirror")
+            lop.set_variant("auto")
+            assert torch.equal(a, b)
+            ref, _ = oracle.bilateral_f32(img.numpy(), 3.0, sigma_r, "mirror")
+            worst = max(worst, _cmp_float(b.cpu().numpy(), ref))
+    print("max abs err (npoly=%s, scaled=%s): %.3g" % (npoly, scaled, worst))
 
 
 def test_config1_bilateral_256_clamp(lop):
