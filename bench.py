@@ -378,21 +378,11 @@ def extras(lop, synthetic, dev, stream, peaks):
     v = list(modes.values())
     out["bilateral_mode_spread"] = round(max(v) / min(v) - 1.0, 4)
     hbm = float(peaks.get("hbm_gbs", 6650.0))
-    u8 = synthetic.to_u8(img)
-    conv = {}
-    cases = [("gaussian5x5_f32", lambda: lop.gaussian(img, 5, "clamp", out=res, stream=stream), 8),
-             ("sobel3x3_f32", lambda: lop.sobel(img, 0, "clamp", out=res, stream=stream), 8)]
-    u8o = torch.empty_like(u8)
-    i32o = torch.empty(u8.shape, dtype=torch.int32, device=dev)
-    cases += [("gaussian5x5_u8", lambda: lop.gaussian(u8, 5, "clamp", out=u8o, stream=stream), 2),
-              ("sobel3x3_u8_i32", lambda: lop.sobel(u8, 0, "clamp", out=i32o, stream=stream), 5)]
-    for name, fn, bpp in cases:
-        ms = timed(fn, 20, True)
-        gbs = H * Wd * bpp / ms / 1e6
-        conv[name] = {"Mpx_s": round(H * Wd / ms / 1e3, 1), "ms": round(ms, 4),
-                      "GB_s": round(gbs, 1), "hbm_frac": round(gbs / hbm, 3),
-                      "bytes_per_px": bpp}
-    out["conv_4096_l2_flushed"] = conv
+    out["conv_4096"] = conv_extras(lop, synthetic, dev, stream, hbm, img, timed)
+    out["conv_4096"]["method"] = (
+        "CUDA graph of 8 launches over 8 rotating input/output sets (footprint > L2, so every "
+        "launch reads and writes DRAM), replayed; per-launch time = replay time / 8; also the "
+        "median single launch after an L2 flush")
     # config 1: 256^2, 3x3, sigma_d = 1, sigma_r = 5, clamp -- launch-latency bound:
     # report CUDA-graph replays of 100 launches
     small = synthetic.angio(256, 256, seed=synthetic.config_seed(1), device=dev)
@@ -409,6 +399,46 @@ def extras(lop, synthetic, dev, stream, peaks):
     ms = timed(lambda: g.replay(), 10, False)
     out["config1_bilateral_256_3x3_graph_Mpx_s"] = round(256 * 256 * 100 / ms / 1e3, 1)
     return out
+
+
+def conv_extras(lop, synthetic, dev, stream, hbm, img, timed):
+    """Gaussian 5x5 / Sobel 3x3 on 4096^2 f32 and u8 (BASELINE config 3): HBM roofline."""
+    import torch
+    sets = 8
+    u8 = synthetic.to_u8(img)
+    f_in = [img.clone() for _ in range(sets)]
+    f_out = [torch.empty_like(img) for _ in range(sets)]
+    u_in = [u8.clone() for _ in range(sets)]
+    u_out = [torch.empty_like(u8) for _ in range(sets)]
+    i_out = [torch.empty(u8.shape, dtype=torch.int32, device=dev) for _ in range(sets)]
+    cases = [("gaussian5x5_f32", lambda k, s: lop.gaussian(f_in[k], 5, "clamp", out=f_out[k],
+                                                          stream=s), 8),
+             ("sobel3x3_f32", lambda k, s: lop.sobel(f_in[k], 0, "clamp", out=f_out[k],
+                                                     stream=s), 8),
+             ("gaussian5x5_u8", lambda k, s: lop.gaussian(u_in[k], 5, "clamp", out=u_out[k],
+                                                         stream=s), 2),
+             ("sobel3x3_u8_i32", lambda k, s: lop.sobel(u_in[k], 0, "clamp", out=i_out[k],
+                                                        stream=s), 5)]
+    res = {}
+    H, W = img.shape
+    for name, fn, bpp in cases:
+        g = torch.cuda.CUDAGraph()
+        s2 = torch.cuda.Stream(dev)
+        s2.wait_stream(stream)
+        with torch.cuda.stream(s2):
+            for k in range(sets):
+                fn(k, s2)
+            with torch.cuda.graph(g, stream=s2):
+                for k in range(sets):
+                    fn(k, s2)
+        stream.wait_stream(s2)
+        ms = timed(lambda: g.replay(), 10, False) / sets
+        ms_flush = timed(lambda: fn(0, stream), 10, True)
+        gbs = H * W * bpp / ms / 1e6
+        res[name] = {"Mpx_s": round(H * W / ms / 1e3, 1), "ms": round(ms, 5),
+                     "GB_s": round(gbs, 1), "hbm_frac": round(gbs / hbm, 3), "bytes_per_px": bpp,
+                     "single_launch_after_l2_flush_ms": round(ms_flush, 5)}
+    return res
 
 
 # ------------------------------------------------------------ CPU oracle ----
