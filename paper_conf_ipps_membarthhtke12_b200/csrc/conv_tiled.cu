@@ -62,7 +62,68 @@ __device__ __forceinline__ uint32_t smem_addr(const void *p)
     return (uint32_t)__cvta_generic_to_shared(p);
 }
 
-template <typename T, typename TO, int R>
+// u8 -> u8 with non-negative coefficients whose sums fit 16 bits: SWAR on two
+// 16-bit lanes per 32-bit register (pixels q and q+2), so every IMAD does two
+// exact integer MACs.  Sources: funnel shift of the staged words + byte mask;
+// outputs: (S + 2^(k-1)) >> k per lane, two lanes packed back with PRMT.
+// Exactness conditions are checked on the host (launch_conv_tiled).
+template <int R>
+__device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tcol, int srows,
+                                             char *orow0, int64_t ostride, int ox0, int roi_x1,
+                                             bool ovec)
+{
+    constexpr int SWE = TileShape<uint8_t>::SWE, TS = convt::TS;
+    constexpr uint32_t M = 0x00FF00FFu;
+    static_assert(R <= 3, "SWAR sources cover bytes -4..11");
+    const uint32_t rnd = p.shift > 0 ? (1u << (p.shift - 1)) * 0x00010001u : 0u;
+    uint32_t h[2 * R + 1][4];                     // pairs (0,2) (1,3) (4,6) (5,7)
+#pragma unroll
+    for (int k = 0; k < TS + 2 * R; ++k) {
+        if (k >= srows) break;
+        const uint8_t *rp = tcol + k * SWE;
+        const uint2 cv = *reinterpret_cast<const uint2 *>(rp);
+        const uint32_t W[4] = {*reinterpret_cast<const uint32_t *>(rp - 4), cv.x, cv.y,
+                               *reinterpret_cast<const uint32_t *>(rp + 8)};
+        uint32_t S[6 + 2 * R];                    // S[q + R] = lanes (q, q+2), q in [-R, 5+R]
+#pragma unroll
+        for (int q = -R; q <= 5 + R; ++q) {
+            const int wi = (q + 4) >> 2, sh = (q + 4) & 3;
+            const uint32_t x = sh == 0 ? W[wi] : __funnelshift_r(W[wi], W[wi + 1], 8 * sh);
+            S[q + R] = x & M;
+        }
+        uint32_t *hk = h[k % (2 * R + 1)];
+        constexpr int J[4] = {0, 1, 4, 5};
+#pragma unroll
+        for (int jj = 0; jj < 4; ++jj) {
+            uint32_t s = (uint32_t)p.ri[0] * S[J[jj]];
+#pragma unroll
+            for (int t = 1; t <= 2 * R; ++t) s += (uint32_t)p.ri[t] * S[J[jj] + t];
+            hk[jj] = s;
+        }
+        const int o = k - 2 * R;
+        if (o < 0) continue;
+        uint32_t q4[4];
+#pragma unroll
+        for (int jj = 0; jj < 4; ++jj) {
+            uint32_t s = (uint32_t)p.ci[0] * h[o % (2 * R + 1)][jj];
+#pragma unroll
+            for (int t = 1; t <= 2 * R; ++t) s += (uint32_t)p.ci[t] * h[(o + t) % (2 * R + 1)][jj];
+            q4[jj] = ((s + rnd) >> p.shift) & M;
+        }
+        const uint32_t lo = __byte_perm(q4[0], q4[1], 0x6240);
+        const uint32_t hi = __byte_perm(q4[2], q4[3], 0x6240);
+        uint8_t *op = reinterpret_cast<uint8_t *>(orow0 + (int64_t)o * ostride) + ox0;
+        if (ovec) {
+            *reinterpret_cast<uint2 *>(op) = make_uint2(lo, hi);
+        } else {
+#pragma unroll
+            for (int j = 0; j < 8; ++j)
+                if (ox0 + j < roi_x1) op[j] = (uint8_t)((j < 4 ? lo : hi) >> (8 * (j & 3)));
+        }
+    }
+}
+
+template <typename T, typename TO, int R, bool SWAR = false>
 __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_constant__ ConvSep p)
 {
     constexpr int RX = R, RY = R;
@@ -166,6 +227,11 @@ __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_consta
                       (((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) %
                         (sizeof(TO) * PX > 16 ? 16 : sizeof(TO) * PX)) == 0);
     const T *tcol = tile + PADE + threadIdx.x * PX;              // this thread's centre column
+    if constexpr (SWAR) {
+        conv_u8_swar<R>(p, reinterpret_cast<const uint8_t *>(tcol), srows,
+                        obase + (int64_t)ty0 * c.out.stride, c.out.stride, ox0, roi_x1, ovec);
+        return;
+    }
     A h[2 * RY + 1][PX];                                          // horizontal sums, ring
 #pragma unroll
     for (int k = 0; k < TS + 2 * RY; ++k) {
@@ -339,7 +405,7 @@ bool factor(const ConvGeneric &p, ConvSep &s)
     return 255 * lr * lc + (1ll << 30) < (1ll << 31);
 }
 
-template <typename T, typename TO, int R>
+template <typename T, typename TO, int R, bool SWAR = false>
 cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
 {
     using S = TileShape<T>;
@@ -348,12 +414,12 @@ cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
               s.c.batch);
     static bool configured = false;
     if (!configured && smem > 48 * 1024) {
-        cudaError_t e = cudaFuncSetAttribute(conv_sep_kernel<T, TO, R>,
+        cudaError_t e = cudaFuncSetAttribute(conv_sep_kernel<T, TO, R, SWAR>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
         configured = true;
     }
-    conv_sep_kernel<T, TO, R><<<grid, convt::NT, smem, stream>>>(s);
+    conv_sep_kernel<T, TO, R, SWAR><<<grid, convt::NT, smem, stream>>>(s);
     return cudaGetLastError();
 }
 
@@ -366,6 +432,31 @@ cudaError_t dispatch_r(const ConvSep &s, cudaStream_t stream)
     case 2: return launch_sep<T, TO, 2>(s, stream);
     case 3: return launch_sep<T, TO, 3>(s, stream);
     case 4: return launch_sep<T, TO, 4>(s, stream);
+    default: return cudaErrorNotSupported;
+    }
+}
+
+// SWAR eligibility (u8 -> u8): non-negative factors, sum fits a 16-bit lane,
+// no saturation (sum r * sum c <= 2^shift) and the lane shift stays in-lane.
+bool swar_ok(const ConvSep &s)
+{
+    if (s.kind != CONV_U8_U8 || s.c.rx < 1 || s.c.rx > 3 || s.shift > 8) return false;
+    int64_t lr = 0, lc = 0;
+    for (int t = 0; t <= 2 * s.c.rx; ++t) {
+        if (s.ri[t] < 0 || s.ci[t] < 0) return false;
+        lr += s.ri[t];
+        lc += s.ci[t];
+    }
+    const int64_t rnd = s.shift > 0 ? (1ll << (s.shift - 1)) : 0;
+    return lr * lc <= (1ll << s.shift) && 255 * lr * lc + rnd < 65536;
+}
+
+cudaError_t dispatch_swar(const ConvSep &s, cudaStream_t stream)
+{
+    switch (s.c.rx) {
+    case 1: return launch_sep<uint8_t, uint8_t, 1, true>(s, stream);
+    case 2: return launch_sep<uint8_t, uint8_t, 2, true>(s, stream);
+    case 3: return launch_sep<uint8_t, uint8_t, 3, true>(s, stream);
     default: return cudaErrorNotSupported;
     }
 }
@@ -388,7 +479,8 @@ cudaError_t launch_conv_tiled(const ConvGeneric &p, cudaStream_t stream)
     s.shift = p.shift;
     switch (p.kind) {
     case CONV_F32: return dispatch_r<float, float>(s, stream);
-    case CONV_U8_U8: return dispatch_r<uint8_t, uint8_t>(s, stream);
+    case CONV_U8_U8:
+        return swar_ok(s) ? dispatch_swar(s, stream) : dispatch_r<uint8_t, uint8_t>(s, stream);
     case CONV_U8_I32: return dispatch_r<uint8_t, int32_t>(s, stream);
     default: return cudaErrorNotSupported;
     }

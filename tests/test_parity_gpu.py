@@ -246,6 +246,21 @@ def test_conv_random_separable_masks(lop, conv_variant, size):
             assert (q[sel] == refq[sel]).all(), (mode, odt)
 
 
+@pytest.mark.parametrize("rows,cols,shift", [([1, 2, 1], [1, 1, 1], 4), ([3, 0, 2, 1, 1], [1, 4, 6, 4, 1], 8),
+                                             ([1, 1, 1, 1, 1, 1, 1], [2, 1, 0, 1, 2, 1, 1], 6),
+                                             ([0, 1, 0], [0, 0, 1], 0)])
+def test_conv_u8_swar_masks(lop, conv_variant, rows, cols, shift):
+    """Non-negative separable u8 masks that fit 16-bit lanes take the SWAR path
+    (two exact MACs per IMAD); bit-exact against the oracle in every mode."""
+    mi = np.outer(np.array(cols), np.array(rows)).astype(np.int32)
+    u8 = synthetic.uniform_u8(77, 301, seed=sum(rows) * 7 + shift)
+    for mode in MODES:
+        q = lop.convolve(u8.cuda(), mi, mode, constant=250, shift=shift).cpu().numpy()
+        refq, valid = oracle.convolve_u8(u8.numpy(), mi, shift, mode, cval=250)
+        sel = valid if mode == "undefined" else slice(None)
+        assert (q[sel] == refq[sel]).all(), mode
+
+
 @pytest.mark.parametrize("msize", [(3, 5), (7, 1), (1, 9), (11, 11), (15, 3)])
 def test_conv_random_masks(lop, msize):
     rng = np.random.default_rng(msize[0] * 100 + msize[1])
