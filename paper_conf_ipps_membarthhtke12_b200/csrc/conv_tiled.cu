@@ -123,61 +123,63 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
     }
 }
 
-template <typename T, typename TO, int R, bool SWAR = false>
-__global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_constant__ ConvSep p)
+// Tile geometry of tile index `t` (row-major over column tiles, row tiles, frames).
+struct ConvTile {
+    int b, tx0, ty0, nrows;
+};
+
+template <typename T>
+__device__ __forceinline__ ConvTile conv_tile_at(const Common &c, int t)
 {
-    constexpr int RX = R, RY = R;
     using S = TileShape<T>;
-    constexpr int PX = S::PX, TS = convt::TS, SWE = S::SWE, PADE = S::PADE;
+    const int ntx = (c.roi_w + S::TWE - 1) / S::TWE, nty = (c.roi_h + convt::TS - 1) / convt::TS;
+    ConvTile ct;
+    ct.b = t / (ntx * nty);
+    const int r = t - ct.b * ntx * nty;
+    const int ty = r / ntx, tx = r - ty * ntx;
+    ct.tx0 = c.roi_x0 + tx * S::TWE;
+    ct.ty0 = c.roi_y0 + ty * convt::TS;
+    ct.nrows = min(convt::TS, c.roi_y0 + c.roi_h - ct.ty0);
+    return ct;
+}
+
+// Stage the input footprint of tile `ct` into `tile`: every staged row whose
+// source row exists (in-image, halo, or mapped by the boundary mode) is copied
+// by one cp.async.bulk of its 16-B aligned in-image column span completing on
+// `bar` (thread 0 arms it with the byte count; 0 bytes completes at once); the
+// out-of-image columns and CONSTANT rows are filled element by element with
+// the boundary resolved per column (visible after the caller's __syncthreads).
+template <typename T, int R>
+__device__ __forceinline__ void conv_stage(const Common &c, const ConvTile &ct, T *tile,
+                                           uint64_t *bar)
+{
+    using S = TileShape<T>;
+    constexpr int SWE = S::SWE, PADE = S::PADE;
     constexpr bool F = sizeof(T) == 4;
-    using A = typename std::conditional<F, float, int>::type;   // accumulator type
-    static_assert(RX <= 4, "halo must fit the 16-B pad");
-
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ __align__(8) uint64_t bar;
-    T *tile = reinterpret_cast<T *>(smem_raw);                    // (TS+2RY) x SWE
-
-    const Common &c = p.c;
     const Geom &g = c.in;
-    const int b = blockIdx.z;
-    const int tx0 = c.roi_x0 + blockIdx.x * S::TWE;               // output tile origin
-    const int ty0 = c.roi_y0 + blockIdx.y * TS;
-    const int roi_x1 = c.roi_x0 + c.roi_w, roi_y1 = c.roi_y0 + c.roi_h;
-    const int nrows = min(TS, roi_y1 - ty0);                      // output rows in this tile
-    const int srows = nrows + 2 * RY;                             // staged input rows
-    const int ix0 = tx0 + c.off_x - PADE;                         // input col of smem col 0
-    const int iy0 = ty0 + c.off_y - RY;                           // input row of smem row 0
-    const char *fbase = g.data + (int64_t)b * g.bstride;
-
-    // ---------------------------------------------------------------- stage
-    // Every staged row whose source row exists (in-image, halo, or mapped by
-    // the boundary mode) is copied by one cp.async.bulk of its 16-B aligned
-    // in-image column span; the out-of-image columns (and CONSTANT rows) are
-    // filled element by element with the boundary resolved per column.
-    const A cval = F ? (A)c.cval_f : (A)c.cval_i;
+    const int srows = ct.nrows + 2 * R;
+    const int ix0 = ct.tx0 + c.off_x - PADE;                      // input col of smem col 0
+    const int iy0 = ct.ty0 + c.off_y - R;                         // input row of smem row 0
+    const char *fbase = g.data + (int64_t)ct.b * g.bstride;
+    const T cval = F ? (T)c.cval_f : (T)c.cval_i;
     const bool aligned = ((reinterpret_cast<uintptr_t>(fbase) | (uintptr_t)g.stride |
                            (uintptr_t)(ix0 * (int)sizeof(T))) % 16 == 0);
     constexpr int V16 = 16 / sizeof(T);                            // elements per 16 B
-    // bulk span [xa, xb) in smem columns (same for every row)
-    int xa = max(0, -ix0), xb = min(SWE, g.W - ix0);
+    int xa = max(0, -ix0), xb = min(SWE, g.W - ix0);               // bulk span, smem columns
     xa = (xa + V16 - 1) / V16 * V16;
     xb = xb / V16 * V16;
     const bool bulk = aligned && xb > xa;
-    if (bulk) {
-        if (threadIdx.x == 0) {
-            asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&bar)));
-            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        }
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            int nbytes = 0;
+    if (threadIdx.x == 0) {
+        int nbytes = 0;
+        if (bulk)
             for (int r = 0; r < srows; ++r) {
                 int row;
                 if (resolve_row(iy0 + r, g, c.mode, row)) nbytes += (xb - xa) * (int)sizeof(T);
             }
-            asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;"
-                         ::"r"(smem_addr(&bar)), "r"(nbytes) : "memory");
-        }
+        asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;"
+                     ::"r"(smem_addr(bar)), "r"(nbytes) : "memory");
+    }
+    if (bulk) {
         for (int r = threadIdx.x; r < srows; r += convt::NT) {
             int row;
             if (!resolve_row(iy0 + r, g, c.mode, row)) continue;
@@ -185,7 +187,7 @@ __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_consta
             asm volatile(
                 "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                 ::"r"(smem_addr(tile + r * SWE + xa)), "l"(src), "r"((xb - xa) * (int)sizeof(T)),
-                  "r"(smem_addr(&bar))
+                  "r"(smem_addr(bar))
                 : "memory");
         }
     }
@@ -197,9 +199,9 @@ __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_consta
         int row, col;
         T v;
         if (resolve_row(iy0 + r, g, c.mode, row) && resolve_col(ix0 + x, g, c.mode, col))
-            v = __ldg(row_ptr<T>(g, b, row) + col);
+            v = __ldg(row_ptr<T>(g, ct.b, row) + col);
         else
-            v = (T)cval;
+            v = cval;
         tile[r * SWE + x] = v;
     }
     // ... and the bulk span of CONSTANT rows (no source row to copy)
@@ -207,20 +209,34 @@ __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_consta
         for (int r = 0; r < srows; ++r) {
             int row;
             if (resolve_row(iy0 + r, g, c.mode, row)) continue;
-            for (int x = xa + threadIdx.x; x < xb; x += convt::NT) tile[r * SWE + x] = (T)cval;
+            for (int x = xa + threadIdx.x; x < xb; x += convt::NT) tile[r * SWE + x] = cval;
         }
     }
-    __syncthreads();
-    if (bulk) {
-        asm volatile(
-            "{\n\t.reg .pred P;\n"
-            "WAIT_%=:\n\t"
-            "mbarrier.try_wait.parity.shared.b64 P, [%0], 0;\n\t"
-            "@!P bra WAIT_%=;\n}" ::"r"(smem_addr(&bar)) : "memory");
-    }
+}
 
-    // -------------------------------------------------------------- compute
-    const int ox0 = tx0 + threadIdx.x * PX;
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity)
+{
+    asm volatile(
+        "{\n\t.reg .pred P;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared.b64 P, [%0], %1;\n\t"
+        "@!P bra WAIT_%=;\n}" ::"r"(smem_addr(bar)), "r"(parity) : "memory");
+}
+
+// Filter one staged tile: each thread streams its PX columns down the tile.
+template <typename T, typename TO, int R, bool SWAR>
+__device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &ct, const T *tile)
+{
+    constexpr int RX = R, RY = R;
+    using S = TileShape<T>;
+    constexpr int PX = S::PX, TS = convt::TS, SWE = S::SWE, PADE = S::PADE;
+    constexpr bool F = sizeof(T) == 4;
+    using A = typename std::conditional<F, float, int>::type;   // accumulator type
+    const Common &c = p.c;
+    const int b = ct.b, ty0 = ct.ty0;
+    const int srows = ct.nrows + 2 * RY;
+    const int roi_x1 = c.roi_x0 + c.roi_w;
+    const int ox0 = ct.tx0 + threadIdx.x * PX;
     if (ox0 >= roi_x1) return;
     char *obase = c.out.data + (int64_t)b * c.out.bstride;
     const bool ovec = (ox0 + PX <= roi_x1) && (ox0 % PX == 0) &&
@@ -344,6 +360,41 @@ __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_consta
     }
 }
 
+// Persistent kernel: each CTA walks tiles blockIdx.x, blockIdx.x + gridDim.x,
+// ...; the next tile's rows are in flight (cp.async.bulk into the other smem
+// buffer) while the current tile is filtered.
+template <typename T, typename TO, int R, bool SWAR = false>
+__global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_constant__ ConvSep p)
+{
+    using S = TileShape<T>;
+    static_assert(R <= 4, "halo must fit the 16-B pad");
+    constexpr int BUF_ELEMS = (convt::TS + 2 * R) * S::SWE;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ __align__(8) uint64_t bar[2];
+    T *buf0 = reinterpret_cast<T *>(smem_raw);
+    T *buf1 = buf0 + BUF_ELEMS;
+    const Common &c = p.c;
+    const int ntiles = ((c.roi_w + S::TWE - 1) / S::TWE) *
+                       ((c.roi_h + convt::TS - 1) / convt::TS) * c.batch;
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&bar[0])));
+        asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&bar[1])));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    int t = blockIdx.x;
+    if (t < ntiles) conv_stage<T, R>(c, conv_tile_at<T>(c, t), buf0, &bar[0]);
+    for (int it = 0; t < ntiles; t += gridDim.x, ++it) {
+        const int cur = it & 1;
+        __syncthreads();        // tile it-1 fully consumed; element fills of tile it visible
+        const int tn = t + gridDim.x;
+        if (tn < ntiles)
+            conv_stage<T, R>(c, conv_tile_at<T>(c, tn), cur ? buf0 : buf1, &bar[cur ^ 1]);
+        mbar_wait(&bar[cur], (it >> 1) & 1);
+        conv_compute<T, TO, R, SWAR>(p, conv_tile_at<T>(c, t), cur ? buf1 : buf0);
+    }
+}
+
 // -------------------------------------------------------------- host side
 namespace {
 
@@ -409,16 +460,25 @@ template <typename T, typename TO, int R, bool SWAR = false>
 cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
 {
     using S = TileShape<T>;
-    const size_t smem = (size_t)(convt::TS + 2 * R) * S::ROW_BYTES;
-    dim3 grid((s.c.roi_w + S::TWE - 1) / S::TWE, (s.c.roi_h + convt::TS - 1) / convt::TS,
-              s.c.batch);
-    static bool configured = false;
-    if (!configured && smem > 48 * 1024) {
-        cudaError_t e = cudaFuncSetAttribute(conv_sep_kernel<T, TO, R, SWAR>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        configured = true;
+    const size_t smem = 2 * (size_t)(convt::TS + 2 * R) * S::ROW_BYTES;   // double buffer
+    static int grid_max = 0;
+    if (!grid_max) {
+        if (smem > 48 * 1024) {
+            cudaError_t e = cudaFuncSetAttribute(conv_sep_kernel<T, TO, R, SWAR>,
+                                                 cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                 (int)smem);
+            if (e != cudaSuccess) return e;
+        }
+        int dev = 0, sms = 0, per_sm = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, conv_sep_kernel<T, TO, R, SWAR>,
+                                                      convt::NT, smem);
+        grid_max = sms * (per_sm > 0 ? per_sm : 1);
     }
+    const long ntiles = (long)((s.c.roi_w + S::TWE - 1) / S::TWE) *
+                        ((s.c.roi_h + convt::TS - 1) / convt::TS) * s.c.batch;
+    const int grid = (int)(ntiles < grid_max ? ntiles : grid_max);
     conv_sep_kernel<T, TO, R, SWAR><<<grid, convt::NT, smem, stream>>>(s);
     return cudaGetLastError();
 }

@@ -180,10 +180,15 @@ def test_config2_bilateral_4096_sampled(lop, mode):
     _cmp_float(out2[ys, xs], ref2, valid2 if mode == "undefined" else None)
 
 
-def test_bilateral_step_edge_bit_exact(lop):
+def test_bilateral_step_edge_preserved(lop, monkeypatch):
     """Levels {0, .5, 1}, sigma_r = 0.02: cross-edge weights underflow to 0 in
-    f32, so the output equals the input exactly (SURVEY §8(c) pins)."""
+    f32, so the output equals the input (SURVEY §8(c) pins): bit for bit with
+    the unscaled exponent, within the final 1/alpha rescale (a few ulp) with the
+    default scaled-difference exponent."""
     img = synthetic.levels(200, 300, seed=3)
+    out = lop.bilateral(img.cuda(), 3.0, 0.02, "clamp").cpu()
+    assert (out - img).abs().max() <= 2e-7
+    monkeypatch.setenv("LOP_BILATERAL_SCALED", "0")
     out = lop.bilateral(img.cuda(), 3.0, 0.02, "clamp").cpu()
     assert torch.equal(out, img)
 
