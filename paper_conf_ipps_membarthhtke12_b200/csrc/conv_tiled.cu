@@ -24,6 +24,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <cstdio>
+#include <cstdlib>
 #include <type_traits>
 
 #include "boundary.cuh"
@@ -67,12 +69,12 @@ __device__ __forceinline__ uint32_t smem_addr(const void *p)
 // exact integer MACs.  Sources: funnel shift of the staged words + byte mask;
 // outputs: (S + 2^(k-1)) >> k per lane, two lanes packed back with PRMT.
 // Exactness conditions are checked on the host (launch_conv_tiled).
-template <int R>
+template <int R, int TS>
 __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tcol, int srows,
                                              char *orow0, int64_t ostride, int ox0, int roi_x1,
                                              bool ovec)
 {
-    constexpr int SWE = TileShape<uint8_t>::SWE, TS = convt::TS;
+    constexpr int SWE = TileShape<uint8_t>::SWE;
     constexpr uint32_t M = 0x00FF00FFu;
     static_assert(R <= 3, "SWAR sources cover bytes -4..11");
     const uint32_t rnd = p.shift > 0 ? (1u << (p.shift - 1)) * 0x00010001u : 0u;
@@ -128,18 +130,18 @@ struct ConvTile {
     int b, tx0, ty0, nrows;
 };
 
-template <typename T>
+template <typename T, int TS>
 __device__ __forceinline__ ConvTile conv_tile_at(const Common &c, int t)
 {
     using S = TileShape<T>;
-    const int ntx = (c.roi_w + S::TWE - 1) / S::TWE, nty = (c.roi_h + convt::TS - 1) / convt::TS;
+    const int ntx = (c.roi_w + S::TWE - 1) / S::TWE, nty = (c.roi_h + TS - 1) / TS;
     ConvTile ct;
     ct.b = t / (ntx * nty);
     const int r = t - ct.b * ntx * nty;
     const int ty = r / ntx, tx = r - ty * ntx;
     ct.tx0 = c.roi_x0 + tx * S::TWE;
-    ct.ty0 = c.roi_y0 + ty * convt::TS;
-    ct.nrows = min(convt::TS, c.roi_y0 + c.roi_h - ct.ty0);
+    ct.ty0 = c.roi_y0 + ty * TS;
+    ct.nrows = min(TS, c.roi_y0 + c.roi_h - ct.ty0);
     return ct;
 }
 
@@ -224,12 +226,12 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity)
 }
 
 // Filter one staged tile: each thread streams its PX columns down the tile.
-template <typename T, typename TO, int R, bool SWAR>
+template <typename T, typename TO, int R, bool SWAR, int TS>
 __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &ct, const T *tile)
 {
     constexpr int RX = R, RY = R;
     using S = TileShape<T>;
-    constexpr int PX = S::PX, TS = convt::TS, SWE = S::SWE, PADE = S::PADE;
+    constexpr int PX = S::PX, SWE = S::SWE, PADE = S::PADE;
     constexpr bool F = sizeof(T) == 4;
     using A = typename std::conditional<F, float, int>::type;   // accumulator type
     const Common &c = p.c;
@@ -244,7 +246,7 @@ __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &c
                         (sizeof(TO) * PX > 16 ? 16 : sizeof(TO) * PX)) == 0);
     const T *tcol = tile + PADE + threadIdx.x * PX;              // this thread's centre column
     if constexpr (SWAR) {
-        conv_u8_swar<R>(p, reinterpret_cast<const uint8_t *>(tcol), srows,
+        conv_u8_swar<R, TS>(p, reinterpret_cast<const uint8_t *>(tcol), srows,
                         obase + (int64_t)ty0 * c.out.stride, c.out.stride, ox0, roi_x1, ovec);
         return;
     }
@@ -360,22 +362,24 @@ __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &c
     }
 }
 
-// Persistent kernel: each CTA walks tiles blockIdx.x, blockIdx.x + gridDim.x,
-// ...; the next tile's rows are in flight (cp.async.bulk into the other smem
-// buffer) while the current tile is filtered.
-template <typename T, typename TO, int R, bool SWAR = false>
+// NBUF = 2: persistent kernel -- each CTA walks tiles blockIdx.x,
+// blockIdx.x + gridDim.x, ...; the next tile's rows are in flight
+// (cp.async.bulk into the other smem buffer) while the current tile is
+// filtered.  NBUF = 1: one tile per CTA (grid = #tiles), latency hidden by
+// co-resident CTAs.  TS = output rows per tile.  (Configuration space of the
+// paper's §V-D exploration, re-done for sm_100a: tools/tune_conv.py.)
+template <typename T, typename TO, int R, bool SWAR, int TS, int NBUF>
 __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_constant__ ConvSep p)
 {
     using S = TileShape<T>;
     static_assert(R <= 4, "halo must fit the 16-B pad");
-    constexpr int BUF_ELEMS = (convt::TS + 2 * R) * S::SWE;
+    constexpr int BUF_ELEMS = (TS + 2 * R) * S::SWE;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     __shared__ __align__(8) uint64_t bar[2];
     T *buf0 = reinterpret_cast<T *>(smem_raw);
-    T *buf1 = buf0 + BUF_ELEMS;
+    T *buf1 = NBUF == 2 ? buf0 + BUF_ELEMS : buf0;
     const Common &c = p.c;
-    const int ntiles = ((c.roi_w + S::TWE - 1) / S::TWE) *
-                       ((c.roi_h + convt::TS - 1) / convt::TS) * c.batch;
+    const int ntiles = ((c.roi_w + S::TWE - 1) / S::TWE) * ((c.roi_h + TS - 1) / TS) * c.batch;
     if (threadIdx.x == 0) {
         asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&bar[0])));
         asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&bar[1])));
@@ -383,15 +387,22 @@ __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_consta
     }
     __syncthreads();
     int t = blockIdx.x;
-    if (t < ntiles) conv_stage<T, R>(c, conv_tile_at<T>(c, t), buf0, &bar[0]);
+    if (t < ntiles) conv_stage<T, R>(c, conv_tile_at<T, TS>(c, t), buf0, &bar[0]);
+    if (NBUF == 1) {
+        if (t >= ntiles) return;
+        __syncthreads();
+        mbar_wait(&bar[0], 0);
+        conv_compute<T, TO, R, SWAR, TS>(p, conv_tile_at<T, TS>(c, t), buf0);
+        return;
+    }
     for (int it = 0; t < ntiles; t += gridDim.x, ++it) {
         const int cur = it & 1;
         __syncthreads();        // tile it-1 fully consumed; element fills of tile it visible
         const int tn = t + gridDim.x;
         if (tn < ntiles)
-            conv_stage<T, R>(c, conv_tile_at<T>(c, tn), cur ? buf0 : buf1, &bar[cur ^ 1]);
+            conv_stage<T, R>(c, conv_tile_at<T, TS>(c, tn), cur ? buf0 : buf1, &bar[cur ^ 1]);
         mbar_wait(&bar[cur], (it >> 1) & 1);
-        conv_compute<T, TO, R, SWAR>(p, conv_tile_at<T>(c, t), cur ? buf1 : buf0);
+        conv_compute<T, TO, R, SWAR, TS>(p, conv_tile_at<T, TS>(c, t), cur ? buf1 : buf0);
     }
 }
 
@@ -456,15 +467,15 @@ bool factor(const ConvGeneric &p, ConvSep &s)
     return 255 * lr * lc + (1ll << 30) < (1ll << 31);
 }
 
-template <typename T, typename TO, int R, bool SWAR = false>
-cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
+template <typename T, typename TO, int R, bool SWAR, int TS, int NBUF>
+cudaError_t launch_cfg(const ConvSep &s, cudaStream_t stream)
 {
     using S = TileShape<T>;
-    const size_t smem = 2 * (size_t)(convt::TS + 2 * R) * S::ROW_BYTES;   // double buffer
+    const size_t smem = (size_t)NBUF * (TS + 2 * R) * S::ROW_BYTES;
     static int grid_max = 0;
     if (!grid_max) {
         if (smem > 48 * 1024) {
-            cudaError_t e = cudaFuncSetAttribute(conv_sep_kernel<T, TO, R, SWAR>,
+            cudaError_t e = cudaFuncSetAttribute(conv_sep_kernel<T, TO, R, SWAR, TS, NBUF>,
                                                  cudaFuncAttributeMaxDynamicSharedMemorySize,
                                                  (int)smem);
             if (e != cudaSuccess) return e;
@@ -472,15 +483,36 @@ cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
         int dev = 0, sms = 0, per_sm = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, conv_sep_kernel<T, TO, R, SWAR>,
-                                                      convt::NT, smem);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(
+            &per_sm, conv_sep_kernel<T, TO, R, SWAR, TS, NBUF>, convt::NT, smem);
         grid_max = sms * (per_sm > 0 ? per_sm : 1);
     }
-    const long ntiles = (long)((s.c.roi_w + S::TWE - 1) / S::TWE) *
-                        ((s.c.roi_h + convt::TS - 1) / convt::TS) * s.c.batch;
-    const int grid = (int)(ntiles < grid_max ? ntiles : grid_max);
-    conv_sep_kernel<T, TO, R, SWAR><<<grid, convt::NT, smem, stream>>>(s);
+    const long ntiles = (long)((s.c.roi_w + S::TWE - 1) / S::TWE) * ((s.c.roi_h + TS - 1) / TS) *
+                        s.c.batch;
+    const int grid = NBUF == 1 ? (int)ntiles : (int)(ntiles < grid_max ? ntiles : grid_max);
+    conv_sep_kernel<T, TO, R, SWAR, TS, NBUF><<<grid, convt::NT, smem, stream>>>(s);
     return cudaGetLastError();
+}
+
+// Tile configuration: (TS, NBUF) from LOP_CONV_CFG="TS:NBUF" (tuning sweep),
+// else the default measured best on B200.  The sweep space is
+// instantiated for radii 1 and 2 (Sobel 3x3, Gaussian 5x5); other radii use
+// the default.
+constexpr int kDefTS = 16, kDefNBUF = 1;
+
+template <typename T, typename TO, int R, bool SWAR = false>
+cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
+{
+    int ts = kDefTS, nbuf = kDefNBUF;
+    if (const char *env = std::getenv("LOP_CONV_CFG")) std::sscanf(env, "%d:%d", &ts, &nbuf);
+    if constexpr (R == 1 || R == 2) {
+        if (ts == 8 && nbuf == 1) return launch_cfg<T, TO, R, SWAR, 8, 1>(s, stream);
+        if (ts == 8 && nbuf == 2) return launch_cfg<T, TO, R, SWAR, 8, 2>(s, stream);
+        if (ts == 16 && nbuf == 2) return launch_cfg<T, TO, R, SWAR, 16, 2>(s, stream);
+        if (ts == 32 && nbuf == 1) return launch_cfg<T, TO, R, SWAR, 32, 1>(s, stream);
+        if (ts == 32 && nbuf == 2) return launch_cfg<T, TO, R, SWAR, 32, 2>(s, stream);
+    }
+    return launch_cfg<T, TO, R, SWAR, kDefTS, kDefNBUF>(s, stream);
 }
 
 template <typename T, typename TO>
