@@ -498,7 +498,7 @@ cudaError_t launch_cfg(const ConvSep &s, cudaStream_t stream)
 // else the default measured best on B200.  The sweep space is
 // instantiated for radii 1 and 2 (Sobel 3x3, Gaussian 5x5); other radii use
 // the default.
-constexpr int kDefTS = 16, kDefNBUF = 1;
+constexpr int kDefTS = 8, kDefNBUF = 1;   // tools/tune_conv.py on B200, round 1
 
 template <typename T, typename TO, int R, bool SWAR = false>
 cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
@@ -506,7 +506,8 @@ cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
     int ts = kDefTS, nbuf = kDefNBUF;
     if (const char *env = std::getenv("LOP_CONV_CFG")) std::sscanf(env, "%d:%d", &ts, &nbuf);
     if constexpr (R == 1 || R == 2) {
-        if (ts == 8 && nbuf == 1) return launch_cfg<T, TO, R, SWAR, 8, 1>(s, stream);
+        if (ts == 4 && nbuf == 1) return launch_cfg<T, TO, R, SWAR, 4, 1>(s, stream);
+        if (ts == 16 && nbuf == 1) return launch_cfg<T, TO, R, SWAR, 16, 1>(s, stream);
         if (ts == 8 && nbuf == 2) return launch_cfg<T, TO, R, SWAR, 8, 2>(s, stream);
         if (ts == 16 && nbuf == 2) return launch_cfg<T, TO, R, SWAR, 16, 2>(s, stream);
         if (ts == 32 && nbuf == 1) return launch_cfg<T, TO, R, SWAR, 32, 1>(s, stream);

@@ -251,7 +251,7 @@ def test_conv_random_separable_masks(lop, conv_variant, size):
             assert (q[sel] == refq[sel]).all(), (mode, odt)
 
 
-@pytest.mark.parametrize("cfg", ["8:1", "16:1", "32:1", "8:2", "16:2", "32:2"])
+@pytest.mark.parametrize("cfg", ["4:1", "8:1", "16:1", "32:1", "8:2", "16:2", "32:2"])
 def test_conv_tile_configs(lop, cfg, monkeypatch):
     """Every tile configuration of the convolution kernels (LOP_CONV_CFG =
     rows per tile : buffers) gives the oracle's result (u8 bit-exact), including

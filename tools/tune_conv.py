@@ -31,7 +31,7 @@ cases = [("gaussian5x5_f32", lambda k, s: lop.gaussian(f_in[k], 5, "clamp", out=
          ("sobel3x3_f32", lambda k, s: lop.sobel(f_in[k], 0, "clamp", out=f_out[k], stream=s), 8),
          ("gaussian5x5_u8", lambda k, s: lop.gaussian(u_in[k], 5, "clamp", out=u_out[k], stream=s), 2),
          ("sobel3x3_u8_i32", lambda k, s: lop.sobel(u_in[k], 0, "clamp", out=i_out[k], stream=s), 5)]
-cfgs = sys.argv[1:] or ["8:1", "16:1", "32:1", "8:2", "16:2", "32:2"]
+cfgs = sys.argv[1:] or ["4:1", "8:1", "16:1", "32:1", "8:2", "16:2", "32:2"]
 for cfg in cfgs:
     os.environ["LOP_CONV_CFG"] = cfg
     for name, fn, bpp in cases:
