@@ -207,6 +207,9 @@ lop_status lop_pipeline_convolve(lop_pipeline *p, const void *host_in, int32_t i
                                  int64_t in_stride_bytes, void *host_out, int32_t out_dtype,
                                  int64_t out_stride_bytes, int32_t mode, double constant,
                                  const lop_mask *mask);
+/* Host->device and device->host bytes moved by the last pipeline call
+ * (image rows + window halo rows re-uploaded at chunk seams). */
+lop_status lop_pipeline_bytes(const lop_pipeline *p, int64_t *h2d, int64_t *d2h);
 lop_status lop_pipeline_destroy(lop_pipeline *p);
 
 #ifdef __cplusplus

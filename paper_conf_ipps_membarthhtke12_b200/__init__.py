@@ -241,6 +241,12 @@ class Pipeline:
         self._h = h
         self.width, self.height = width, height
 
+    def bytes_moved(self):
+        """(host->device, device->host) bytes of the last call."""
+        h2d, d2h = ctypes.c_int64(), ctypes.c_int64()
+        _check(lib.lop_pipeline_bytes(self._h, ctypes.byref(h2d), ctypes.byref(d2h)))
+        return h2d.value, d2h.value
+
     def close(self):
         if self._h:
             lib.lop_pipeline_destroy(self._h)

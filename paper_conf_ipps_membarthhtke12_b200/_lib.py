@@ -69,6 +69,7 @@ SIGNATURES = {
                                        c_i32, ctypes.POINTER(lop_mask), c_flt, c_flt]),
     "lop_pipeline_convolve": (c_i32, [c_vp, c_vp, c_i32, c_i64, c_vp, c_i32, c_i64, c_i32,
                                       c_dbl, ctypes.POINTER(lop_mask)]),
+    "lop_pipeline_bytes": (c_i32, [c_vp, ctypes.POINTER(c_i64), ctypes.POINTER(c_i64)]),
     "lop_pipeline_destroy": (c_i32, [c_vp]),
 }
 
@@ -82,7 +83,7 @@ class LopError(RuntimeError):
 def load(path: str = LIB_PATH) -> ctypes.CDLL:
     if not os.path.exists(path):
         raise ImportError("liblop.so not built (%s); run "
-                          "`python -m paper_conf_ipps_membarthhtke12_b200.build`" % path)
+                          "`python paper_conf_ipps_membarthhtke12_b200/build.py`" % path)
     lib = ctypes.CDLL(path)
     for name, (res, args) in SIGNATURES.items():
         fn = getattr(lib, name)

@@ -1,6 +1,6 @@
 """Build liblop.so (the C-ABI library + sm_100a kernels) in-tree with nvcc.
 
-    python -m paper_conf_ipps_membarthhtke12_b200.build [--force] [--verbose]
+    python paper_conf_ipps_membarthhtke12_b200/build.py [--force] [--verbose]
 
 Every translation unit is compiled for sm_100a only
 (-gencode arch=compute_100a,code=sm_100a), with -lineinfo so ncu's source

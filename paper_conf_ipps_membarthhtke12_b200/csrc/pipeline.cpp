@@ -13,6 +13,7 @@
 #include <algorithm>
 #include <cstring>
 #include <string>
+#include <vector>
 
 #include "lop.h"
 
@@ -28,6 +29,7 @@ struct lop_pipeline {
     void *d_out[2] = {nullptr, nullptr};
     cudaStream_t s_h2d = nullptr, s_comp = nullptr, s_d2h = nullptr;
     cudaEvent_t up_done[2] = {}, comp_done[2] = {}, down_done[2] = {};
+    int64_t h2d_bytes = 0, d2h_bytes = 0;   // of the last run
 };
 
 namespace {
@@ -72,6 +74,7 @@ lop_status upload_chunk(lop_pipeline *p, int buf, const char *host, int64_t hstr
             const int64_t src = wrap_row(gy, p->H);
             e = cudaMemcpyAsync(own0 + (int64_t)(gy - y0) * dstride, host + src * hstride, dstride,
                                 cudaMemcpyHostToDevice, p->s_h2d);
+            p->h2d_bytes += dstride;
             if (e != cudaSuccess) return perr(e, "pipeline ring row upload");
         }
     }
@@ -79,6 +82,7 @@ lop_status upload_chunk(lop_pipeline *p, int buf, const char *host, int64_t hstr
                           host + (int64_t)lo_in * hstride, hstride, dstride, hi_in - lo_in,
                           cudaMemcpyHostToDevice, p->s_h2d);
     if (e != cudaSuccess) return perr(e, "pipeline upload");
+    p->h2d_bytes += (int64_t)(hi_in - lo_in) * dstride;
     std::memset(view, 0, sizeof *view);
     view->data = own0;
     view->width = p->W;
@@ -93,6 +97,31 @@ lop_status upload_chunk(lop_pipeline *p, int buf, const char *host, int64_t hstr
     return LOP_OK;
 }
 
+// Row cuts of the pipeline: chunks ramp up (c/8, c/4, c/2) at the start and
+// down again at the end, so that only a small first upload and a small last
+// download are not overlapped with the other direction.
+std::vector<int> chunk_schedule(int H, int c)
+{
+    std::vector<int> sizes;
+    int rest = H;
+    std::vector<int> ramp;
+    for (int d = 8; d >= 2; d /= 2)
+        if (c / d >= 16) ramp.push_back(c / d);
+    int ramp_rows = 0;
+    for (int r : ramp) ramp_rows += 2 * r;
+    if (ramp_rows + c > H) ramp.clear();
+    for (int r : ramp) { sizes.push_back(r); rest -= r; }
+    std::vector<int> tail(ramp.rbegin(), ramp.rend());
+    int tail_rows = 0;
+    for (int r : tail) tail_rows += r;
+    rest -= tail_rows;
+    while (rest > 0) { sizes.push_back(std::min(c, rest)); rest -= c; }
+    for (int r : tail) sizes.push_back(r);
+    std::vector<int> cuts(1, 0);
+    for (int sz : sizes) cuts.push_back(cuts.back() + sz);
+    return cuts;
+}
+
 template <typename Exec>
 lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t in_stride,
                void *host_out, int32_t out_dtype, int64_t out_stride, int mode, double constant,
@@ -104,12 +133,14 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
     const int ies = esize(in_dtype), oes = esize(out_dtype);
     if (in_stride < (int64_t)p->W * ies || out_stride < (int64_t)p->W * oes) return LOP_ERR_INVALID;
     DevGuard guard(p->device);
+    p->h2d_bytes = p->d2h_bytes = 0;
     const char *hin = static_cast<const char *>(host_in);
     char *hout = static_cast<char *>(host_out);
-    const int nchunks = (p->H + p->chunk - 1) / p->chunk;
+    const std::vector<int> cuts = chunk_schedule(p->H, p->chunk);
+    const int nchunks = (int)cuts.size() - 1;
     for (int k = 0; k < nchunks; ++k) {
         const int buf = k & 1;
-        const int y0 = k * p->chunk, y1 = std::min(p->H, y0 + p->chunk);
+        const int y0 = cuts[k], y1 = cuts[k + 1];
         cudaError_t e;
         if (k >= 2) {
             e = cudaStreamWaitEvent(p->s_h2d, p->comp_done[buf], 0);
@@ -150,6 +181,7 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
                               (int64_t)p->W * oes, (int64_t)p->W * oes, y1 - y0,
                               cudaMemcpyDeviceToHost, p->s_d2h);
         if (e != cudaSuccess) return perr(e, "pipeline download");
+        p->d2h_bytes += (int64_t)(y1 - y0) * p->W * oes;
         cudaEventRecord(p->down_done[buf], p->s_d2h);
     }
     cudaError_t e = cudaStreamSynchronize(p->s_d2h);
@@ -220,6 +252,14 @@ lop_status lop_pipeline_convolve(lop_pipeline *p, const void *host_in, int32_t i
                [&](const lop_iteration_space *is, const lop_accessor *acc, cudaStream_t s) {
                    return lop_convolve_execute(is, acc, mask, s);
                });
+}
+
+lop_status lop_pipeline_bytes(const lop_pipeline *p, int64_t *h2d, int64_t *d2h)
+{
+    if (!p || !h2d || !d2h) return LOP_ERR_INVALID;
+    *h2d = p->h2d_bytes;
+    *d2h = p->d2h_bytes;
+    return LOP_OK;
 }
 
 lop_status lop_pipeline_destroy(lop_pipeline *p)
