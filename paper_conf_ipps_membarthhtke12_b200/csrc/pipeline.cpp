@@ -4,7 +4,7 @@
 //   stream h2d : chunk k+1 host -> device (rows + window halo)
 //   stream comp: chunk k filtered by the same kernels as lop_*_execute
 //   stream d2h : chunk k-1 device -> host
-// Double-buffered device staging, ordered with events.  The chunk views are
+// A ring of device staging buffers, ordered with events.  The chunk views are
 // row bands of the global image (lop_image.global_y0/global_height), so the
 // boundary handling is exactly that of the whole-image call; REPEAT halo rows
 // outside the image are uploaded as ring rows.
@@ -21,14 +21,18 @@ namespace lop_detail {
 void set_error(const std::string &msg);   // lop_api.cpp
 }
 
+// staging buffers per direction: a ring of 4 decouples the H2D and D2H
+// engines (chunk k+4 may upload while chunk k is still downloading)
+constexpr int kBufs = 4;
+
 struct lop_pipeline {
     int device = 0;
     int W = 0, H = 0, chunk = 0;
     size_t in_bytes = 0, out_bytes = 0;     // per staging buffer
-    void *d_in[2] = {nullptr, nullptr};
-    void *d_out[2] = {nullptr, nullptr};
+    void *d_in[kBufs] = {};
+    void *d_out[kBufs] = {};
     cudaStream_t s_h2d = nullptr, s_comp = nullptr, s_d2h = nullptr;
-    cudaEvent_t up_done[2] = {}, comp_done[2] = {}, down_done[2] = {};
+    cudaEvent_t up_done[kBufs] = {}, comp_done[kBufs] = {}, down_done[kBufs] = {};
     int64_t h2d_bytes = 0, d2h_bytes = 0;   // of the last run
 };
 
@@ -139,10 +143,10 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
     const std::vector<int> cuts = chunk_schedule(p->H, p->chunk);
     const int nchunks = (int)cuts.size() - 1;
     for (int k = 0; k < nchunks; ++k) {
-        const int buf = k & 1;
+        const int buf = k % kBufs;
         const int y0 = cuts[k], y1 = cuts[k + 1];
         cudaError_t e;
-        if (k >= 2) {
+        if (k >= kBufs) {
             e = cudaStreamWaitEvent(p->s_h2d, p->comp_done[buf], 0);
             if (e != cudaSuccess) return perr(e, "wait");
         }
@@ -151,7 +155,7 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
         if (st) return st;
         cudaEventRecord(p->up_done[buf], p->s_h2d);
         cudaStreamWaitEvent(p->s_comp, p->up_done[buf], 0);
-        if (k >= 2) cudaStreamWaitEvent(p->s_comp, p->down_done[buf], 0);
+        if (k >= kBufs) cudaStreamWaitEvent(p->s_comp, p->down_done[buf], 0);
         lop_image out_view;
         std::memset(&out_view, 0, sizeof out_view);
         out_view.data = p->d_out[buf];
@@ -211,7 +215,7 @@ lop_status lop_pipeline_create(int32_t device, int32_t width, int32_t height, in
     p->in_bytes = (size_t)(chunk_rows + 2 * kMaxHalo) * width * 4;
     p->out_bytes = (size_t)chunk_rows * width * 4;
     cudaError_t e = cudaSuccess;
-    for (int i = 0; i < 2 && e == cudaSuccess; ++i) {
+    for (int i = 0; i < kBufs && e == cudaSuccess; ++i) {
         e = cudaMalloc(&p->d_in[i], p->in_bytes);
         if (e == cudaSuccess) e = cudaMalloc(&p->d_out[i], p->out_bytes);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->up_done[i], cudaEventDisableTiming);
@@ -269,7 +273,7 @@ lop_status lop_pipeline_destroy(lop_pipeline *p)
     if (p->s_h2d) cudaStreamSynchronize(p->s_h2d);
     if (p->s_comp) cudaStreamSynchronize(p->s_comp);
     if (p->s_d2h) cudaStreamSynchronize(p->s_d2h);
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < kBufs; ++i) {
         if (p->d_in[i]) cudaFree(p->d_in[i]);
         if (p->d_out[i]) cudaFree(p->d_out[i]);
         if (p->up_done[i]) cudaEventDestroy(p->up_done[i]);
