@@ -321,7 +321,7 @@ def run_lop(args, dist, peaks):
         H = Wd = 4096
         host_in = base.cpu().pin_memory()
         host_out = torch.empty_like(host_in).pin_memory()
-        pipe = lop.Pipeline(Wd, H, device=dist.local, chunk_rows=512)
+        pipe = lop.Pipeline(Wd, H, device=dist.local, chunk_rows=1024)
         for _ in range(2):
             pipe.bilateral(host_in, host_out, sigma_d, sigma_r, args.mode, size=size)
         dist.barrier()
@@ -335,7 +335,7 @@ def run_lop(args, dist, peaks):
                          "unit": "Mpixel/s", "h2d_bytes_per_step": int(h2d),
                          "d2h_bytes_per_step": int(d2h),
                          "api": "lop.Pipeline.bilateral (lop_pipeline_bilateral), pinned host "
-                                "buffers, 512-row chunks (ramped at both ends) on 3 streams, "
+                                "buffers, 1024-row chunks (ramped at both ends) on 3 streams, "
                                 "wall clock"}
     if not args.no_extras and dist.world == 1 and args.workload == "bilateral4096":
         result["filters"] = extras(lop, synthetic, dev, stream, peaks)

@@ -14,6 +14,9 @@
 #include <cstring>
 #include <string>
 #include <vector>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 
 #include "lop.h"
 
@@ -54,6 +57,15 @@ struct DevGuard {
     ~DevGuard() { if (prev >= 0) cudaSetDevice(prev); }
 };
 
+// Row block copy: one linear DMA when both pitches equal the row width.
+cudaError_t copy_rows(void *dst, int64_t dpitch, const void *src, int64_t spitch, int64_t width,
+                      int64_t rows, cudaMemcpyKind kind, cudaStream_t s)
+{
+    if (dpitch == width && spitch == width)
+        return cudaMemcpyAsync(dst, src, (size_t)(width * rows), kind, s);
+    return cudaMemcpy2DAsync(dst, dpitch, src, spitch, width, rows, kind, s);
+}
+
 int64_t wrap_row(int64_t gy, int64_t H)
 {
     int64_t q = gy % H;
@@ -82,9 +94,8 @@ lop_status upload_chunk(lop_pipeline *p, int buf, const char *host, int64_t hstr
             if (e != cudaSuccess) return perr(e, "pipeline ring row upload");
         }
     }
-    e = cudaMemcpy2DAsync(own0 + (int64_t)(lo_in - y0) * dstride, dstride,
-                          host + (int64_t)lo_in * hstride, hstride, dstride, hi_in - lo_in,
-                          cudaMemcpyHostToDevice, p->s_h2d);
+    e = copy_rows(own0 + (int64_t)(lo_in - y0) * dstride, dstride, host + (int64_t)lo_in * hstride,
+                  hstride, dstride, hi_in - lo_in, cudaMemcpyHostToDevice, p->s_h2d);
     if (e != cudaSuccess) return perr(e, "pipeline upload");
     p->h2d_bytes += (int64_t)(hi_in - lo_in) * dstride;
     std::memset(view, 0, sizeof *view);
@@ -138,6 +149,8 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
     if (in_stride < (int64_t)p->W * ies || out_stride < (int64_t)p->W * oes) return LOP_ERR_INVALID;
     DevGuard guard(p->device);
     p->h2d_bytes = p->d2h_bytes = 0;
+    static const bool trace = std::getenv("LOP_PIPELINE_TRACE") != nullptr;
+    const auto t_start = std::chrono::steady_clock::now();
     const char *hin = static_cast<const char *>(host_in);
     char *hout = static_cast<char *>(host_out);
     const std::vector<int> cuts = chunk_schedule(p->H, p->chunk);
@@ -181,12 +194,21 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
         if (st) return st;
         cudaEventRecord(p->comp_done[buf], p->s_comp);
         cudaStreamWaitEvent(p->s_d2h, p->comp_done[buf], 0);
-        e = cudaMemcpy2DAsync(hout + (int64_t)y0 * out_stride, out_stride, p->d_out[buf],
-                              (int64_t)p->W * oes, (int64_t)p->W * oes, y1 - y0,
-                              cudaMemcpyDeviceToHost, p->s_d2h);
+        e = copy_rows(hout + (int64_t)y0 * out_stride, out_stride, p->d_out[buf],
+                      (int64_t)p->W * oes, (int64_t)p->W * oes, y1 - y0, cudaMemcpyDeviceToHost,
+                      p->s_d2h);
         if (e != cudaSuccess) return perr(e, "pipeline download");
         p->d2h_bytes += (int64_t)(y1 - y0) * p->W * oes;
         cudaEventRecord(p->down_done[buf], p->s_d2h);
+    }
+    if (trace) {
+        const double t_enq = std::chrono::duration<double, std::milli>(
+                                 std::chrono::steady_clock::now() - t_start).count();
+        cudaStreamSynchronize(p->s_d2h);
+        const double t_all = std::chrono::duration<double, std::milli>(
+                                 std::chrono::steady_clock::now() - t_start).count();
+        std::fprintf(stderr, "lop_pipeline: %d chunks, enqueue %.3f ms, total %.3f ms\n",
+                     nchunks, t_enq, t_all);
     }
     cudaError_t e = cudaStreamSynchronize(p->s_d2h);
     if (e != cudaSuccess) return perr(e, "pipeline sync");

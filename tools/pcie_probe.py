@@ -47,6 +47,29 @@ def both():
 
 print(json.dumps({"h2d_GB_s": round(bw(h2d), 1), "d2h_GB_s": round(bw(d2h), 1),
                   "bidirectional_each_GB_s": round(bw(both), 1)}), flush=True)
+
+
+def chunked(nchunks):
+    # the pipeline's copy pattern without the kernel: chunk k uploads while chunk k-1 downloads
+    step = N // nchunks
+    ev = [torch.cuda.Event() for _ in range(nchunks)]
+
+    def run():
+        for k in range(nchunks):
+            with torch.cuda.stream(s1):
+                d_a[k * step:(k + 1) * step].copy_(h_src[k * step:(k + 1) * step],
+                                                   non_blocking=True)
+                ev[k].record(s1)
+            s2.wait_event(ev[k])
+            with torch.cuda.stream(s2):
+                h_dst[k * step:(k + 1) * step].copy_(d_a[k * step:(k + 1) * step],
+                                                     non_blocking=True)
+    return run
+
+
+for n in (1, 4, 8, 16):
+    print(json.dumps({"chunked_copies": n, "each_dir_GB_s": round(bw(chunked(n), reps=5), 1)}),
+          flush=True)
 H = W = 4096
 img = synthetic.angio(H, W, seed=synthetic.config_seed(2)).pin_memory()
 out = torch.empty_like(img).pin_memory()
