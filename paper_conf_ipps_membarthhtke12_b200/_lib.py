@@ -9,7 +9,8 @@ import ctypes
 import os
 
 PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(PKG, "liblop.so")
+# LOP_LIBRARY: load an alternative build (A/B experiments); default: the in-tree build
+LIB_PATH = os.environ.get("LOP_LIBRARY") or os.path.join(PKG, "liblop.so")
 
 LOP_OK, LOP_ERR_INVALID, LOP_ERR_UNSUPPORTED, LOP_ERR_CUDA = 0, -1, -2, -3
 LOP_U8, LOP_I32, LOP_F32 = 0, 1, 2

@@ -79,12 +79,32 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB
 
 
+EXAMPLE_SRC = os.path.join(ROOT, "examples", "bilateral_c.c")
+EXAMPLE_BIN = os.path.join(ROOT, "examples", "bilateral_c")
+
+
+def build_example(force: bool = False) -> str:
+    """Plain-C program against include/lop.h + liblop.so (the ABI without Python)."""
+    lib = build(force=force)
+    if not force and os.path.exists(EXAMPLE_BIN) and \
+            os.path.getmtime(EXAMPLE_BIN) >= max(os.path.getmtime(EXAMPLE_SRC),
+                                                 os.path.getmtime(lib)):
+        return EXAMPLE_BIN
+    cmd = [nvcc(), *ARCH, "-O2", "-x", "cu", "-I", INCLUDE, EXAMPLE_SRC, "-o", EXAMPLE_BIN,
+           "-L", PKG, "-llop", "-Xlinker", "-rpath=$ORIGIN/../" + os.path.basename(PKG)]
+    res = subprocess.run(cmd, capture_output=True, text=True)
+    if res.returncode != 0:
+        raise RuntimeError("example build failed:\n%s\n%s" % (" ".join(cmd), res.stderr))
+    return EXAMPLE_BIN
+
+
 def main(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--force", action="store_true")
     ap.add_argument("--verbose", action="store_true")
     a = ap.parse_args(argv)
     print(build(force=a.force, verbose=a.verbose))
+    print(build_example(force=a.force))
 
 
 if __name__ == "__main__":

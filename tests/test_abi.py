@@ -137,3 +137,12 @@ def test_variant_switch():
     assert lop.get_variant() == "generic"
     lop.set_variant("auto")
     assert lop.lib.lop_set_variant(7) == _lib.LOP_ERR_INVALID
+
+
+def test_c_example_is_built_against_the_abi():
+    """examples/bilateral_c.c uses only include/lop.h + the CUDA runtime."""
+    exe = os.path.join(ROOT, "examples", "bilateral_c")
+    assert os.path.exists(exe), "run __graft_entry__.build()"
+    import subprocess
+    out = subprocess.run(["ldd", exe], capture_output=True, text=True).stdout
+    assert "liblop.so" in out

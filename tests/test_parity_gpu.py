@@ -450,3 +450,15 @@ def test_launch_count(lop):
     lop.bilateral(img, 1.0, 0.1)
     lop.gaussian(img)
     assert lop.launch_count() == 2
+
+
+def test_c_example_runs(lop):
+    """The Listing 2 host flow from plain C through include/lop.h (device call +
+    host pipeline, identical results, Listing 4's mask value)."""
+    import os
+    import subprocess
+    from conftest import ROOT
+    res = subprocess.run([os.path.join(ROOT, "examples", "bilateral_c")], capture_output=True,
+                         text=True, timeout=120)
+    assert res.returncode == 0, res.stderr
+    assert "bilateral_c ok" in res.stdout
