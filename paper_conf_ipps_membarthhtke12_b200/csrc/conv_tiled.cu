@@ -90,8 +90,14 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
 #pragma unroll
         for (int q = -R; q <= 5 + R; ++q) {
             const int wi = (q + 4) >> 2, sh = (q + 4) & 3;
-            const uint32_t x = sh == 0 ? W[wi] : __funnelshift_r(W[wi], W[wi + 1], 8 * sh);
-            S[q + R] = x & M;
+            // bytes q and q+2 into the two 16-bit lanes: one PRMT with a zero
+            // source when both lie in the same word, else funnel shift + mask
+            if (sh == 0)
+                S[q + R] = __byte_perm(W[wi], 0u, 0x4240);      // bytes 0, 2 -> lanes
+            else if (sh == 1)
+                S[q + R] = __byte_perm(W[wi], 0u, 0x4341);      // bytes 1, 3 -> lanes
+            else
+                S[q + R] = __funnelshift_r(W[wi], W[wi + 1], 8 * sh) & M;
         }
         uint32_t *hk = h[k % (2 * R + 1)];
         constexpr int J[4] = {0, 1, 4, 5};
@@ -107,10 +113,10 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
         uint32_t q4[4];
 #pragma unroll
         for (int jj = 0; jj < 4; ++jj) {
-            uint32_t s = (uint32_t)p.ci[0] * h[o % (2 * R + 1)][jj];
+            uint32_t s = (uint32_t)p.ci[0] * h[o % (2 * R + 1)][jj] + rnd;   // rounding folded in
 #pragma unroll
             for (int t = 1; t <= 2 * R; ++t) s += (uint32_t)p.ci[t] * h[(o + t) % (2 * R + 1)][jj];
-            q4[jj] = ((s + rnd) >> p.shift) & M;
+            q4[jj] = (s >> p.shift) & M;
         }
         const uint32_t lo = __byte_perm(q4[0], q4[1], 0x6240);
         const uint32_t hi = __byte_perm(q4[2], q4[3], 0x6240);
@@ -498,12 +504,12 @@ cudaError_t launch_cfg(const ConvSep &s, cudaStream_t stream)
 // else the default measured best on B200.  The sweep space is
 // instantiated for radii 1 and 2 (Sobel 3x3, Gaussian 5x5); other radii use
 // the default.
-constexpr int kDefTS = 8, kDefNBUF = 1;   // tools/tune_conv.py on B200, round 1
+constexpr int kDefTS = 8, kDefTSSwar = 16, kDefNBUF = 1;   // tools/tune_conv.py on B200, round 1
 
 template <typename T, typename TO, int R, bool SWAR = false>
 cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
 {
-    int ts = kDefTS, nbuf = kDefNBUF;
+    int ts = SWAR ? kDefTSSwar : kDefTS, nbuf = kDefNBUF;
     if (const char *env = std::getenv("LOP_CONV_CFG")) std::sscanf(env, "%d:%d", &ts, &nbuf);
     if constexpr (R == 1 || R == 2) {
         if (ts == 4 && nbuf == 1) return launch_cfg<T, TO, R, SWAR, 4, 1>(s, stream);
