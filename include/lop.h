@@ -157,6 +157,20 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
 lop_status lop_convolve_execute(const lop_iteration_space *is, const lop_accessor *in,
                                 const lop_mask *mask, void *cuda_stream);
 
+/* Fused two-stage local operator (PAPER.md L107-L122 on
+ * combining operators): out = second (*) (first (*) I), both stages with the
+ * accessor's BoundaryCondition, computed in one pass without the intermediate
+ * image leaving on-chip memory.  Bit-identical to two lop_convolve_execute
+ * calls (the first with an intermediate of the input's type: F32, or U8
+ * rounded and saturated with first->shift).
+ * Masks: square 3x3 or 5x5, exactly separable (Gaussian, Sobel, box ...);
+ * the BoundaryCondition window must be the combined footprint
+ * (first->size + second->size - 1, the paper's "largest window" rule L556-L558).
+ * dtypes: F32 -> F32, U8 -> U8, U8 -> I32.  Whole images only (no band views). */
+lop_status lop_convolve_chain_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                      const lop_mask *first, const lop_mask *second,
+                                      void *cuda_stream);
+
 /* Mask builders (host only).
  * lop_mask_closeness: Eq. (1), float coefficients (Listing 4's mask[]).
  * lop_mask_gaussian:  binomial size x size (size odd; 1..11 for LOP_I32, 1..31

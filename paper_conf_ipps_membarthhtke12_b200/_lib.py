@@ -56,6 +56,9 @@ SIGNATURES = {
     "lop_convolve_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
                                      ctypes.POINTER(lop_accessor), ctypes.POINTER(lop_mask),
                                      c_vp]),
+    "lop_convolve_chain_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
+                                           ctypes.POINTER(lop_accessor), ctypes.POINTER(lop_mask),
+                                           ctypes.POINTER(lop_mask), c_vp]),
     "lop_mask_closeness": (c_i32, [c_flt, c_i32, c_i32, c_vp]),
     "lop_mask_gaussian": (c_i32, [c_i32, c_i32, c_vp, ctypes.POINTER(c_i32)]),
     "lop_mask_sobel": (c_i32, [c_i32, c_i32, c_vp]),

@@ -76,6 +76,21 @@ __device__ __forceinline__ int read_u8(const Geom &g, int b, int ix, int iy, int
     return (int)__ldg(row_ptr<uint8_t>(g, b, row) + col);
 }
 
+__device__ __forceinline__ uint32_t smem_addr(const void *p)
+{
+    return (uint32_t)__cvta_generic_to_shared(p);
+}
+
+// Wait for phase `parity` of an mbarrier (try_wait loop; hardware sleep).
+__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity)
+{
+    asm volatile(
+        "{\n\t.reg .pred P;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared.b64 P, [%0], %1;\n\t"
+        "@!P bra WAIT_%=;\n}" ::"r"(smem_addr(bar)), "r"(parity) : "memory");
+}
+
 __device__ __forceinline__ float ex2_approx(float x)
 {
     float y;

@@ -29,18 +29,11 @@
 #include <type_traits>
 
 #include "boundary.cuh"
+#include "stage.cuh"
 #include "kernels.h"
 #include "lop_params.h"
 
 namespace lop {
-
-struct ConvSep {
-    Common c;
-    int32_t kind;
-    int32_t shift;
-    float rf[9], cf[9];      // f32 row / column coefficients
-    int32_t ri[9], ci[9];    // integer row / column coefficients
-};
 
 namespace convt {
 constexpr int NT = 128;      // threads per CTA
@@ -59,10 +52,6 @@ template <typename T> struct TileShape {
     static constexpr int ROW_BYTES = SWE * sizeof(T);          // multiple of 16
 };
 
-__device__ __forceinline__ uint32_t smem_addr(const void *p)
-{
-    return (uint32_t)__cvta_generic_to_shared(p);
-}
 
 // u8 -> u8 with non-negative coefficients whose sums fit 16 bits: SWAR on two
 // 16-bit lanes per 32-bit register (pixels q and q+2), so every IMAD does two
@@ -162,74 +151,10 @@ __device__ __forceinline__ void conv_stage(const Common &c, const ConvTile &ct, 
                                            uint64_t *bar)
 {
     using S = TileShape<T>;
-    constexpr int SWE = S::SWE, PADE = S::PADE;
-    constexpr bool F = sizeof(T) == 4;
-    const Geom &g = c.in;
-    const int srows = ct.nrows + 2 * R;
-    const int ix0 = ct.tx0 + c.off_x - PADE;                      // input col of smem col 0
-    const int iy0 = ct.ty0 + c.off_y - R;                         // input row of smem row 0
-    const char *fbase = g.data + (int64_t)ct.b * g.bstride;
-    const T cval = F ? (T)c.cval_f : (T)c.cval_i;
-    const bool aligned = ((reinterpret_cast<uintptr_t>(fbase) | (uintptr_t)g.stride |
-                           (uintptr_t)(ix0 * (int)sizeof(T))) % 16 == 0);
-    constexpr int V16 = 16 / sizeof(T);                            // elements per 16 B
-    int xa = max(0, -ix0), xb = min(SWE, g.W - ix0);               // bulk span, smem columns
-    xa = (xa + V16 - 1) / V16 * V16;
-    xb = xb / V16 * V16;
-    const bool bulk = aligned && xb > xa;
-    if (threadIdx.x == 0) {
-        int nbytes = 0;
-        if (bulk)
-            for (int r = 0; r < srows; ++r) {
-                int row;
-                if (resolve_row(iy0 + r, g, c.mode, row)) nbytes += (xb - xa) * (int)sizeof(T);
-            }
-        asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;"
-                     ::"r"(smem_addr(bar)), "r"(nbytes) : "memory");
-    }
-    if (bulk) {
-        for (int r = threadIdx.x; r < srows; r += convt::NT) {
-            int row;
-            if (!resolve_row(iy0 + r, g, c.mode, row)) continue;
-            const char *src = fbase + (int64_t)row * g.stride + (int64_t)(ix0 + xa) * sizeof(T);
-            asm volatile(
-                "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-                ::"r"(smem_addr(tile + r * SWE + xa)), "l"(src), "r"((xb - xa) * (int)sizeof(T)),
-                  "r"(smem_addr(bar))
-                : "memory");
-        }
-    }
-    // element-wise part: the columns outside the bulk span of every row ...
-    const int side = bulk ? xa + (SWE - xb) : SWE;
-    for (int i = threadIdx.x; i < srows * side; i += convt::NT) {
-        const int r = i / side, k = i - r * side;
-        const int x = !bulk ? k : (k < xa ? k : xb + (k - xa));
-        int row, col;
-        T v;
-        if (resolve_row(iy0 + r, g, c.mode, row) && resolve_col(ix0 + x, g, c.mode, col))
-            v = __ldg(row_ptr<T>(g, ct.b, row) + col);
-        else
-            v = cval;
-        tile[r * SWE + x] = v;
-    }
-    // ... and the bulk span of CONSTANT rows (no source row to copy)
-    if (bulk && c.mode == M_CONSTANT) {
-        for (int r = 0; r < srows; ++r) {
-            int row;
-            if (resolve_row(iy0 + r, g, c.mode, row)) continue;
-            for (int x = xa + threadIdx.x; x < xb; x += convt::NT) tile[r * SWE + x] = cval;
-        }
-    }
+    stage_rows<T, S::SWE, convt::NT>(c, ct.b, ct.tx0 + c.off_x - S::PADE, ct.ty0 + c.off_y - R,
+                                     ct.nrows + 2 * R, tile, bar);
 }
 
-__device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity)
-{
-    asm volatile(
-        "{\n\t.reg .pred P;\n"
-        "WAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared.b64 P, [%0], %1;\n\t"
-        "@!P bra WAIT_%=;\n}" ::"r"(smem_addr(bar)), "r"(parity) : "memory");
-}
 
 // Filter one staged tile: each thread streams its PX columns down the tile.
 template <typename T, typename TO, int R, bool SWAR, int TS>
@@ -561,6 +486,8 @@ cudaError_t dispatch_swar(const ConvSep &s, cudaStream_t stream)
 }
 
 }  // namespace
+
+bool conv_factor(const ConvGeneric &p, ConvSep &s) { return factor(p, s); }
 
 bool conv_tiled_supported(const ConvGeneric &p)
 {

@@ -15,5 +15,9 @@ cudaError_t launch_conv_generic(const ConvGeneric &p, cudaStream_t stream);
 // (the caller then falls back to the generic kernel).
 cudaError_t launch_conv_tiled(const ConvGeneric &p, cudaStream_t stream);
 bool conv_tiled_supported(const ConvGeneric &p);
+// Exact separable factorisation (false if the mask is not rank 1 / too large).
+bool conv_factor(const ConvGeneric &p, ConvSep &s);
+// Fused two-stage convolution; cudaErrorNotSupported if no instance matches.
+cudaError_t launch_conv_chain(const ConvChain &p, cudaStream_t stream);
 
 }  // namespace lop

@@ -443,4 +443,76 @@ lop_status lop_convolve_execute(const lop_iteration_space *is, const lop_accesso
     return launched(lop::launch_conv_generic(p, stream), "conv_generic launch");
 }
 
+// ------------------------------------------------- fused two-stage operator
+namespace {
+// One stage's mask -> exact separable factors (reusing the convolution path).
+lop_status chain_stage(const lop::Common &c, const lop_mask *m, int32_t img_dtype,
+                       lop::ConvSep &s, const char *name)
+{
+    if (!m || !m->coeffs) return fail(LOP_ERR_INVALID, "%s mask is NULL", name);
+    if (m->size_x != m->size_y || !(m->size_x & 1))
+        return fail(LOP_ERR_UNSUPPORTED, "%s mask must be square and odd", name);
+    const int r = m->size_x / 2;
+    if (r < 1 || r > 2) return fail(LOP_ERR_UNSUPPORTED, "%s mask must be 3x3 or 5x5", name);
+    static thread_local lop::ConvGeneric g;
+    g.c = c;
+    g.c.rx = g.c.ry = r;
+    const int n = m->size_x * m->size_y;
+    if (img_dtype == LOP_F32) {
+        if (m->dtype != LOP_F32 || m->shift != 0)
+            return fail(LOP_ERR_INVALID, "%s mask must be F32 with shift 0", name);
+        g.kind = lop::CONV_F32;
+        std::memcpy(g.m.f, m->coeffs, sizeof(float) * n);
+    } else {
+        if (m->dtype != LOP_I32 || m->shift < 0 || m->shift > 30)
+            return fail(LOP_ERR_INVALID, "%s mask must be I32 with shift in 0..30", name);
+        g.kind = lop::CONV_U8_U8;
+        std::memcpy(g.m.i, m->coeffs, sizeof(int32_t) * n);
+    }
+    g.shift = m->shift;
+    if (!lop::conv_factor(g, s))
+        return fail(LOP_ERR_UNSUPPORTED, "%s mask is not exactly separable", name);
+    s.c = g.c;
+    s.kind = g.kind;
+    s.shift = g.shift;
+    return LOP_OK;
+}
+}  // namespace
+
+lop_status lop_convolve_chain_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                      const lop_mask *first, const lop_mask *second,
+                                      void *cuda_stream)
+{
+    if (!first || !second) return fail(LOP_ERR_INVALID, "mask is NULL");
+    if (in && in->bc &&
+        (in->bc->size_x != first->size_x + second->size_x - 1 ||
+         in->bc->size_y != first->size_y + second->size_y - 1))
+        return fail(LOP_ERR_INVALID,
+                    "boundary condition window %d x %d must be the combined footprint %d x %d",
+                    in->bc->size_x, in->bc->size_y, first->size_x + second->size_x - 1,
+                    first->size_y + second->size_y - 1);
+    Prepared pp;
+    lop_status st = prepare(is, in, pp);
+    if (st) return st;
+    const lop::Common &c = pp.c;
+    const lop_image &ii = in->bc->image;
+    if (ii.halo_top || ii.halo_bottom || ii.global_y0 ||
+        (ii.global_height && ii.global_height != ii.height))
+        return fail(LOP_ERR_UNSUPPORTED, "fused chains take whole images (no band views)");
+    const int32_t idt = ii.dtype, odt = is->image.dtype;
+    static thread_local lop::ConvChain p;
+    if (idt == LOP_F32 && odt == LOP_F32) p.kind = 0;
+    else if (idt == LOP_U8 && odt == LOP_U8) p.kind = 1;
+    else if (idt == LOP_U8 && odt == LOP_I32) p.kind = 2;
+    else return fail(LOP_ERR_INVALID, "unsupported dtype combination %d -> %d", idt, odt);
+    st = chain_stage(c, first, idt, p.s1, "first");
+    if (st) return st;
+    st = chain_stage(c, second, idt, p.s2, "second");
+    if (st) return st;
+    cudaError_t e = lop::launch_conv_chain(p, static_cast<cudaStream_t>(cuda_stream));
+    if (e == cudaErrorNotSupported)
+        return fail(LOP_ERR_UNSUPPORTED, "no fused chain instance for this mask pair");
+    return launched(e, "conv_chain launch");
+}
+
 }  // extern "C"

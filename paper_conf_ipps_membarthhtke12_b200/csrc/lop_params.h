@@ -85,4 +85,22 @@ struct ConvGeneric {
     } m;
 };
 
+// Separable factorisation of a convolution mask, M = c r^T (conv_tiled.cu).
+struct ConvSep {
+    Common c;
+    int32_t kind;
+    int32_t shift;
+    float rf[9], cf[9];      // f32 row / column coefficients
+    int32_t ri[9], ci[9];    // integer row / column coefficients
+};
+
+// Fused two-stage local operator (conv_chain.cu): out = M2 (*) (M1 (*) I), both
+// stages with the same boundary condition; the intermediate image never
+// leaves shared memory.  Intermediate of the u8 path is quantised to u8
+// exactly like a lop_convolve_execute u8 -> u8 pass.
+struct ConvChain {
+    ConvSep s1, s2;          // s1.c holds the launch geometry
+    int32_t kind;            // 0: f32 -> f32 -> f32; 1: u8 -> u8 -> u8; 2: u8 -> u8 -> i32
+};
+
 }  // namespace lop

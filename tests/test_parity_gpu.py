@@ -462,3 +462,70 @@ def test_c_example_runs(lop):
                          text=True, timeout=120)
     assert res.returncode == 0, res.stderr
     assert "bilateral_c ok" in res.stdout
+
+
+# ------------------------------------------------- fused two-stage chains ----
+
+def _chain_pairs(dtype):
+    g3, k3 = oracle.gaussian_mask(3)
+    g5, k5 = oracle.gaussian_mask(5)
+    sx, sy = oracle.sobel_mask(0), oracle.sobel_mask(1)
+    box = np.ones((3, 3), np.int32)
+    if dtype == "f32":
+        f = lambda m, k: (m / 2.0 ** k).astype(np.float32)   # noqa: E731
+        return [(f(g5, k5), 0, sx.astype(np.float32), 0), (f(g3, k3), 0, f(g5, k5), 0),
+                (box.astype(np.float32) / 9, 0, sy.astype(np.float32), 0),
+                (sx.astype(np.float32), 0, f(g3, k3), 0)]
+    return [(g5, k5, sx, 0), (g3, k3, g5, k5), (box, 3, sy, 0), (g5, k5, g3, k3)]
+
+
+@pytest.mark.parametrize("shape", [(1, 1), (5, 7), (37, 70), (130, 1100), (77, 2050)])
+@pytest.mark.parametrize("mode", MODES)
+def test_chain_equals_two_passes_and_oracle(lop, shape, mode):
+    """lop.convolve_chain == two lop.convolve passes bit for bit (f32 and u8), and
+    == the oracle's composition (f32 within 1e-5 x mask gain, u8 exact)."""
+    H, W = shape
+    img = synthetic.uniform(H, W, seed=H + 7 * W)
+    u8 = synthetic.uniform_u8(H, W, seed=H * 3 + W)
+    for m1, k1, m2, k2 in _chain_pairs("f32"):
+        fused = lop.convolve_chain(img.cuda(), m1, m2, mode, constant=0.5)
+        two = lop.convolve(lop.convolve(img.cuda(), m1, mode, constant=0.5), m2, mode,
+                           constant=0.5)
+        if mode != "undefined":
+            assert torch.equal(fused, two), (mode, shape)
+        g, _ = oracle.convolve_f32(img.numpy(), m1.astype(np.float64), mode, 0.5)
+        ref, _ = oracle.convolve_f32(g.astype(np.float32), m2.astype(np.float64), mode, 0.5)
+        valid = np.ones_like(ref, bool)
+        if mode == "undefined":
+            r = (m1.shape[0] // 2) + (m2.shape[0] // 2)
+            valid[:] = False
+            valid[r:H - r, r:W - r] = True
+        _cmp_float(fused.cpu().numpy(), ref, valid, tol=2e-5)
+    for m1, k1, m2, k2 in _chain_pairs("u8"):
+        for odt, npdt in ((torch.uint8, np.uint8), (torch.int32, np.int32)):
+            fused = lop.convolve_chain(u8.cuda(), m1, m2, mode, constant=200, shift1=k1,
+                                       shift2=k2, out_dtype=odt).cpu()
+            mid = lop.convolve(u8.cuda(), m1, mode, constant=200, shift=k1)
+            two = lop.convolve(mid, m2, mode, constant=200, shift=k2, out_dtype=odt).cpu()
+            if mode != "undefined":
+                assert torch.equal(fused, two), (mode, shape, odt)
+                g, _ = oracle.convolve_u8(u8.numpy(), m1, k1, mode, cval=200)
+                ref, _ = oracle.convolve_u8(g, m2, k2, mode, cval=200, out_dtype=npdt)
+                assert (fused.numpy() == ref).all()
+
+
+def test_chain_roi_offset_and_validation(lop):
+    img = synthetic.angio(90, 600, seed=3).cuda()
+    g5, k5 = lop.gaussian_mask(5, np.float32)
+    sx = lop.sobel_mask(0, np.float32)
+    full = lop.convolve_chain(img, g5, sx, "mirror")
+    out = torch.full_like(img, -1.0)
+    lop.convolve_chain(img, g5, sx, "mirror", out=out, roi=(13, 7, 500, 70))
+    assert torch.equal(out[7:77, 13:513], full[7:77, 13:513])
+    off = lop.convolve_chain(img, g5, sx, "clamp", offset=(2, -3))
+    two = lop.convolve(lop.convolve(img, g5, "clamp"), sx, "clamp", offset=(2, -3))
+    assert torch.equal(off, two)
+    with pytest.raises(lop.LopError, match="separable"):
+        lop.convolve_chain(img, np.random.rand(3, 3).astype(np.float32), sx)
+    with pytest.raises(lop.LopError):
+        lop.convolve_chain(img, np.ones((7, 7), np.float32), sx)
