@@ -403,6 +403,7 @@ def extras(lop, synthetic, dev, stream, peaks):
 
 def conv_extras(lop, synthetic, dev, stream, hbm, img, timed):
     """Gaussian 5x5 / Sobel 3x3 on 4096^2 f32 and u8 (BASELINE config 3): HBM roofline."""
+    import numpy as np
     import torch
     sets = 8
     u8 = synthetic.to_u8(img)
@@ -419,6 +420,26 @@ def conv_extras(lop, synthetic, dev, stream, hbm, img, timed):
                                                          stream=s), 2),
              ("sobel3x3_u8_i32", lambda k, s: lop.sobel(u_in[k], 0, "clamp", out=i_out[k],
                                                         stream=s), 5)]
+    # fused Gaussian 5x5 -> Sobel 3x3 (one pass) vs the two passes
+    gf, _ = lop.gaussian_mask(5, np.float32)
+    sxf = lop.sobel_mask(0, np.float32)
+    gi, gk = lop.gaussian_mask(5, np.int32)
+    sxi = lop.sobel_mask(0, np.int32)
+    mid_f = torch.empty_like(img)
+    mid_u = torch.empty_like(u8)
+    cases += [
+        ("chain_gauss5_sobel3_f32_fused",
+         lambda k, s: lop.convolve_chain(f_in[k], gf, sxf, "clamp", out=f_out[k], stream=s), 8),
+        ("chain_gauss5_sobel3_f32_two_pass",
+         lambda k, s: lop.convolve(lop.convolve(f_in[k], gf, "clamp", out=mid_f, stream=s), sxf,
+                                   "clamp", out=f_out[k], stream=s), 8),
+        ("chain_gauss5_sobel3_u8_i32_fused",
+         lambda k, s: lop.convolve_chain(u_in[k], gi, sxi, "clamp", shift1=gk, out=i_out[k],
+                                         stream=s), 5),
+        ("chain_gauss5_sobel3_u8_i32_two_pass",
+         lambda k, s: lop.convolve(lop.convolve(u_in[k], gi, "clamp", shift=gk, out=mid_u,
+                                                stream=s), sxi, "clamp", out=i_out[k], stream=s),
+         5)]
     res = {}
     H, W = img.shape
     for name, fn, bpp in cases:
