@@ -112,14 +112,16 @@ __device__ __forceinline__ A sep_v(const ConvSep &s, const A *h)
 // Pass-1 value (before quantisation) at in-image (x, y), reading the input with
 // its boundary condition from global memory -- for G positions outside the
 // image, which take G at their mapped position (pass 2's boundary on G).
+// Rarely executed (border tiles only): kept out of line and rolled so that the
+// hot path's instruction footprint stays small.
 template <typename T, typename A, int R1>
-__device__ A sep_point(const ConvSep &s, const Common &c, int b, int x, int y)
+__device__ __noinline__ A sep_point(const ConvSep &s, const Common &c, int b, int x, int y)
 {
     A h[2 * R1 + 1];
 #pragma unroll
     for (int t = 0; t <= 2 * R1; ++t) {
         A v[2 * R1 + 1];
-#pragma unroll
+#pragma unroll 1
         for (int k = 0; k <= 2 * R1; ++k) {
             if constexpr (sizeof(T) == 4)
                 v[k] = read_f32(c.in, b, x + k - R1, y + t - R1, c.mode, c.cval_f);
@@ -136,6 +138,48 @@ __device__ __forceinline__ TG to_g(A v, int shift)
 {
     if constexpr (std::is_same<TG, float>::value) return v;
     else return (TG)min(max(quantize_shift(v, shift), 0), 255);
+}
+
+// One output row of PX values (vector store when aligned, else per element).
+template <typename TO, int PX, typename A>
+__device__ __forceinline__ void store_row(char *orow, int ox0, int roi_x1, bool ovec,
+                                          const A *out, int shift)
+{
+    if constexpr (std::is_same<TO, float>::value) {
+        float *op = reinterpret_cast<float *>(orow) + ox0;
+        if (ovec) {
+            *reinterpret_cast<float4 *>(op) = make_float4(out[0], out[1], out[2], out[3]);
+        } else {
+            for (int j = 0; j < PX; ++j)
+                if (ox0 + j < roi_x1) op[j] = out[j];
+        }
+    } else if constexpr (sizeof(TO) == 1) {
+        uint32_t w[2] = {0u, 0u};
+#pragma unroll
+        for (int j = 0; j < PX; ++j) {
+            const int q = min(max(quantize_shift(out[j], shift), 0), 255);
+            w[j >> 2] |= (uint32_t)q << (8 * (j & 3));
+        }
+        uint8_t *op = reinterpret_cast<uint8_t *>(orow) + ox0;
+        if (ovec) {
+            *reinterpret_cast<uint2 *>(op) = make_uint2(w[0], w[1]);
+        } else {
+            for (int j = 0; j < PX; ++j)
+                if (ox0 + j < roi_x1) op[j] = (uint8_t)(w[j >> 2] >> (8 * (j & 3)));
+        }
+    } else {
+        int32_t *op = reinterpret_cast<int32_t *>(orow) + ox0;
+        int q[PX];
+#pragma unroll
+        for (int j = 0; j < PX; ++j) q[j] = quantize_shift(out[j], shift);
+        if (ovec) {
+            *reinterpret_cast<int4 *>(op) = make_int4(q[0], q[1], q[2], q[3]);
+            *reinterpret_cast<int4 *>(op + 4) = make_int4(q[4], q[5], q[6], q[7]);
+        } else {
+            for (int j = 0; j < PX; ++j)
+                if (ox0 + j < roi_x1) op[j] = q[j];
+        }
+    }
 }
 
 template <typename T, typename TO, int R1, int R2>
@@ -171,35 +215,42 @@ __global__ void __launch_bounds__(chain::NT) conv_chain_kernel(const __grid_cons
     __syncthreads();
     mbar_wait(&bar, 0);
 
-    // ---- pass 1: G over the tile + R2 halo (thread: PX columns, all G rows)
+    // ---- pass 1: G over the tile + R2 halo (thread: PX columns, all G rows).
+    // The row loop is rolled in groups of one ring period (2R1+1 rows) so the
+    // ring slots stay compile-time register indices while the code stays small.
     {
+        constexpr int P = 2 * R1 + 1;
         const T *tcol = itile + IPAD + threadIdx.x * PX;
-        A h[2 * R1 + 1][PX];
+        A h[P][PX];
+#pragma unroll 1
+        for (int k0 = 0; k0 < ni; k0 += P) {
 #pragma unroll
-        for (int k = 0; k < TS + 2 * R2 + 2 * R1; ++k) {
-            if (k >= ni) break;
-            A v[PX + 2 * R1];
-            chain_gather<T, R1, A>(tcol + k * ISW, v);
+            for (int i = 0; i < P; ++i) {
+                const int k = k0 + i;
+                if (k >= ni) break;
+                A v[PX + 2 * R1];
+                chain_gather<T, R1, A>(tcol + k * ISW, v);
 #pragma unroll
-            for (int j = 0; j < PX; ++j) h[k % (2 * R1 + 1)][j] = sep_h<A, R1>(p.s1, v + j);
-            const int g = k - 2 * R1;
-            if (g < 0) continue;
-            TG out[PX];
+                for (int j = 0; j < PX; ++j) h[i][j] = sep_h<A, R1>(p.s1, v + j);
+                const int g = k - 2 * R1;
+                if (g < 0) continue;
+                TG out[PX];
 #pragma unroll
-            for (int j = 0; j < PX; ++j) {
-                A col[2 * R1 + 1];
+                for (int j = 0; j < PX; ++j) {
+                    A col[P];
 #pragma unroll
-                for (int t = 0; t <= 2 * R1; ++t) col[t] = h[(g + t) % (2 * R1 + 1)][j];
-                out[j] = to_g<A, TG>(sep_v<A, R1>(p.s1, col), p.s1.shift);
-            }
-            TG *gp = gtile + g * GW + threadIdx.x * PX;
-            if constexpr (F) {
-                *reinterpret_cast<float4 *>(gp) = make_float4(out[0], out[1], out[2], out[3]);
-            } else {
-                uint32_t w[2] = {0u, 0u};
+                    for (int t = 0; t < P; ++t) col[t] = h[(i + 1 + t) % P][j];   // rows g..k
+                    out[j] = to_g<A, TG>(sep_v<A, R1>(p.s1, col), p.s1.shift);
+                }
+                TG *gp = gtile + g * GW + threadIdx.x * PX;
+                if constexpr (F) {
+                    *reinterpret_cast<float4 *>(gp) = make_float4(out[0], out[1], out[2], out[3]);
+                } else {
+                    uint32_t w[2] = {0u, 0u};
 #pragma unroll
-                for (int j = 0; j < 8; ++j) w[j >> 2] |= (uint32_t)out[j] << (8 * (j & 3));
-                *reinterpret_cast<uint2 *>(gp) = make_uint2(w[0], w[1]);
+                    for (int j = 0; j < 8; ++j) w[j >> 2] |= (uint32_t)out[j] << (8 * (j & 3));
+                    *reinterpret_cast<uint2 *>(gp) = make_uint2(w[0], w[1]);
+                }
             }
         }
     }
@@ -232,62 +283,30 @@ __global__ void __launch_bounds__(chain::NT) conv_chain_kernel(const __grid_cons
                       (((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) %
                         (sizeof(TO) * PX > 16 ? 16 : sizeof(TO) * PX)) == 0);
     const TG *gcol = gtile + HALO + threadIdx.x * PX;
-    A h[2 * R2 + 1][PX];
+    constexpr int P2 = 2 * R2 + 1;
+    A h[P2][PX];
+#pragma unroll 1
+    for (int k0 = 0; k0 < ng; k0 += P2) {
 #pragma unroll
-    for (int k = 0; k < TS + 2 * R2; ++k) {
-        if (k >= ng) break;
-        A v[PX + 2 * R2];
-        chain_gather<TG, R2, A>(gcol + k * GW, v);
+        for (int i = 0; i < P2; ++i) {
+            const int k = k0 + i;
+            if (k >= ng) break;
+            A v[PX + 2 * R2];
+            chain_gather<TG, R2, A>(gcol + k * GW, v);
 #pragma unroll
-        for (int j = 0; j < PX; ++j) h[k % (2 * R2 + 1)][j] = sep_h<A, R2>(p.s2, v + j);
-        const int o = k - 2 * R2;
-        if (o < 0) continue;
-        A out[PX];
-#pragma unroll
-        for (int j = 0; j < PX; ++j) {
-            A col[2 * R2 + 1];
-#pragma unroll
-            for (int t = 0; t <= 2 * R2; ++t) col[t] = h[(o + t) % (2 * R2 + 1)][j];
-            out[j] = sep_v<A, R2>(p.s2, col);
-        }
-        char *orow = obase + (int64_t)(ty0 + o) * c.out.stride;
-        if constexpr (F) {
-            float *op = reinterpret_cast<float *>(orow) + ox0;
-            if (ovec) {
-                *reinterpret_cast<float4 *>(op) = make_float4(out[0], out[1], out[2], out[3]);
-            } else {
-#pragma unroll
-                for (int j = 0; j < PX; ++j)
-                    if (ox0 + j < roi_x1) op[j] = out[j];
-            }
-        } else if constexpr (sizeof(TO) == 1) {
-            uint32_t w[2] = {0u, 0u};
+            for (int j = 0; j < PX; ++j) h[i][j] = sep_h<A, R2>(p.s2, v + j);
+            const int o = k - 2 * R2;
+            if (o < 0) continue;
+            A out[PX];
 #pragma unroll
             for (int j = 0; j < PX; ++j) {
-                const int q = min(max(quantize_shift(out[j], p.s2.shift), 0), 255);
-                w[j >> 2] |= (uint32_t)q << (8 * (j & 3));
-            }
-            uint8_t *op = reinterpret_cast<uint8_t *>(orow) + ox0;
-            if (ovec) {
-                *reinterpret_cast<uint2 *>(op) = make_uint2(w[0], w[1]);
-            } else {
+                A col[P2];
 #pragma unroll
-                for (int j = 0; j < PX; ++j)
-                    if (ox0 + j < roi_x1) op[j] = (uint8_t)(w[j >> 2] >> (8 * (j & 3)));
+                for (int t = 0; t < P2; ++t) col[t] = h[(i + 1 + t) % P2][j];   // rows o..k
+                out[j] = sep_v<A, R2>(p.s2, col);
             }
-        } else {
-            int32_t *op = reinterpret_cast<int32_t *>(orow) + ox0;
-            int q[PX];
-#pragma unroll
-            for (int j = 0; j < PX; ++j) q[j] = quantize_shift(out[j], p.s2.shift);
-            if (ovec) {
-                *reinterpret_cast<int4 *>(op) = make_int4(q[0], q[1], q[2], q[3]);
-                *reinterpret_cast<int4 *>(op + 4) = make_int4(q[4], q[5], q[6], q[7]);
-            } else {
-#pragma unroll
-                for (int j = 0; j < PX; ++j)
-                    if (ox0 + j < roi_x1) op[j] = q[j];
-            }
+            store_row<TO, PX>(obase + (int64_t)(ty0 + o) * c.out.stride, ox0, roi_x1, ovec, out,
+                              p.s2.shift);
         }
     }
 }
