@@ -13,10 +13,11 @@
 //      G at the per-axis mapped position, recomputed from global memory);
 //   3. stream the output rows from the G tile (pass 2) and store them.
 // Tile: f32 4 columns/thread (G 512 wide, output 504), u8 8 columns/thread
-// (G 1024 wide, output 1008); TS = 8 output rows.
+// (G 1024 wide, output 992: 16-B aligned input origin); TS = 8 output rows.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <cstdlib>
 #include <type_traits>
 
 #include "boundary.cuh"
@@ -28,12 +29,13 @@ namespace lop {
 
 namespace chain {
 constexpr int NT = 128;
-constexpr int TS = 8;
+constexpr int kDefTS_f32 = 8, kDefTS_u8 = 8;   // output rows per tile (tools/tune_chain)
 
 template <typename T> struct Shape {
     static constexpr int PX = sizeof(T) == 4 ? 4 : 8;      // columns per thread
     static constexpr int GW = NT * PX;                     // intermediate tile width
-    static constexpr int HALO = PX;                        // G halo columns per side (>= R2)
+    static constexpr int HALO = 16 / sizeof(T);            // G halo per side (>= R2): keeps the
+                                                           // input origin 16-B aligned
     static constexpr int OW = GW - 2 * HALO;               // output tile width
     static constexpr int IPAD = 16 / sizeof(T);            // input pad beyond G (>= R1), 16 B
     static constexpr int ISW = GW + 2 * IPAD;              // input smem pitch (elements)
@@ -121,7 +123,7 @@ __device__ __noinline__ A sep_point(const ConvSep &s, const Common &c, int b, in
 #pragma unroll
     for (int t = 0; t <= 2 * R1; ++t) {
         A v[2 * R1 + 1];
-#pragma unroll 1
+#pragma unroll
         for (int k = 0; k <= 2 * R1; ++k) {
             if constexpr (sizeof(T) == 4)
                 v[k] = read_f32(c.in, b, x + k - R1, y + t - R1, c.mode, c.cval_f);
@@ -182,12 +184,12 @@ __device__ __forceinline__ void store_row(char *orow, int ox0, int roi_x1, bool 
     }
 }
 
-template <typename T, typename TO, int R1, int R2>
+template <typename T, typename TO, int R1, int R2, int TS>
 __global__ void __launch_bounds__(chain::NT) conv_chain_kernel(const __grid_constant__ ConvChain p)
 {
     using S = chain::Shape<T>;
     constexpr int PX = S::PX, GW = S::GW, HALO = S::HALO, OW = S::OW, IPAD = S::IPAD,
-                  ISW = S::ISW, TS = chain::TS;
+                  ISW = S::ISW;
     constexpr bool F = sizeof(T) == 4;
     using A = typename std::conditional<F, float, int>::type;
     using TG = T;                                                   // intermediate type
@@ -211,14 +213,19 @@ __global__ void __launch_bounds__(chain::NT) conv_chain_kernel(const __grid_cons
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
-    stage_rows<T, ISW, chain::NT>(c, b, gx0 - IPAD, gy0 - R1, ni, itile, &bar);
+    // columns the outputs of this tile need: G [x_lo, x_hi), input up to x_hi + R1
+    const int x_lo = HALO - R2;
+    const int x_hi = min(GW, HALO + (min(roi_x1, tx0 + OW) - tx0) + R2);
+    constexpr int V16 = 16 / sizeof(T);
+    const int icols = min(ISW, (IPAD + x_hi + R1 + V16 - 1) / V16 * V16);
+    stage_rows<T, ISW, chain::NT>(c, b, gx0 - IPAD, gy0 - R1, ni, itile, &bar, icols);
     __syncthreads();
     mbar_wait(&bar, 0);
 
     // ---- pass 1: G over the tile + R2 halo (thread: PX columns, all G rows).
     // The row loop is rolled in groups of one ring period (2R1+1 rows) so the
     // ring slots stay compile-time register indices while the code stays small.
-    {
+    if (threadIdx.x * PX < x_hi) {
         constexpr int P = 2 * R1 + 1;
         const T *tcol = itile + IPAD + threadIdx.x * PX;
         A h[P][PX];
@@ -254,13 +261,18 @@ __global__ void __launch_bounds__(chain::NT) conv_chain_kernel(const __grid_cons
             }
         }
     }
-    // ---- G positions outside the image: pass 2's boundary condition on G
+    // ---- G positions outside the image: pass 2's boundary condition on G.
+    // Only the G positions the tile's outputs read are fixed up (columns
+    // [x_lo, x_hi), all G rows).  A mapped position that lies inside this tile
+    // (clamp, mirror, and repeat for narrow images) is copied from the tile;
+    // otherwise (repeat across the image) it is recomputed from global memory.
     const int GH = c.in.GH, IW = c.in.W;
-    const bool border = gx0 < 0 || gx0 + GW > IW || gy0 < 0 || gy0 + ng > GH;
+    const bool border = gx0 + x_lo < 0 || gx0 + x_hi > IW || gy0 < 0 || gy0 + ng > GH;
     if (border) {
         __syncthreads();                      // all in-tile G values written
-        for (int i = threadIdx.x; i < ng * GW; i += chain::NT) {
-            const int r = i / GW, x = i - r * GW;
+        const int span = x_hi - x_lo;
+        for (int i = threadIdx.x; i < ng * span; i += chain::NT) {
+            const int r = i / span, x = x_lo + (i - r * span);
             const int gx = gx0 + x, gy = gy0 + r;
             if ((unsigned)gx < (unsigned)IW && (unsigned)gy < (unsigned)GH) continue;
             TG val;
@@ -268,7 +280,11 @@ __global__ void __launch_bounds__(chain::NT) conv_chain_kernel(const __grid_cons
                 val = F ? (TG)c.cval_f : (TG)c.cval_i;
             } else {
                 const int mx = map_axis(gx, IW, c.mode), my = map_axis(gy, GH, c.mode);
-                val = to_g<A, TG>(sep_point<T, A, R1>(p.s1, c, b, mx, my), p.s1.shift);
+                const int tx = mx - gx0, ty = my - gy0;
+                if (tx >= 0 && tx < GW && ty >= 0 && ty < ng)
+                    val = gtile[ty * GW + tx];                         // computed in pass 1
+                else
+                    val = to_g<A, TG>(sep_point<T, A, R1>(p.s1, c, b, mx, my), p.s1.shift);
             }
             gtile[r * GW + x] = val;
         }
@@ -313,23 +329,36 @@ __global__ void __launch_bounds__(chain::NT) conv_chain_kernel(const __grid_cons
 
 namespace {
 
-template <typename T, typename TO, int R1, int R2>
-cudaError_t launch_chain_rr(const ConvChain &p, cudaStream_t stream)
+template <typename T, typename TO, int R1, int R2, int TS>
+cudaError_t launch_chain_cfg(const ConvChain &p, cudaStream_t stream)
 {
     using S = chain::Shape<T>;
-    const size_t smem = (size_t)(chain::TS + 2 * R1 + 2 * R2) * S::ISW * sizeof(T) +
-                        (size_t)(chain::TS + 2 * R2) * S::GW * sizeof(T);
+    const size_t smem = (size_t)(TS + 2 * R1 + 2 * R2) * S::ISW * sizeof(T) +
+                        (size_t)(TS + 2 * R2) * S::GW * sizeof(T);
     static bool configured = false;
     if (!configured) {
-        cudaError_t e = cudaFuncSetAttribute(conv_chain_kernel<T, TO, R1, R2>,
+        cudaError_t e = cudaFuncSetAttribute(conv_chain_kernel<T, TO, R1, R2, TS>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
         configured = true;
     }
     const Common &c = p.s1.c;
-    dim3 grid((c.roi_w + S::OW - 1) / S::OW, (c.roi_h + chain::TS - 1) / chain::TS, c.batch);
-    conv_chain_kernel<T, TO, R1, R2><<<grid, chain::NT, smem, stream>>>(p);
+    dim3 grid((c.roi_w + S::OW - 1) / S::OW, (c.roi_h + TS - 1) / TS, c.batch);
+    conv_chain_kernel<T, TO, R1, R2, TS><<<grid, chain::NT, smem, stream>>>(p);
     return cudaGetLastError();
+}
+
+// output rows per tile: LOP_CHAIN_TS overrides (tuning); default per type
+template <typename T, typename TO, int R1, int R2>
+cudaError_t launch_chain_rr(const ConvChain &p, cudaStream_t stream)
+{
+    int ts = sizeof(T) == 4 ? chain::kDefTS_f32 : chain::kDefTS_u8;
+    if (const char *env = std::getenv("LOP_CHAIN_TS")) ts = std::atoi(env);
+    switch (ts) {
+    case 4: return launch_chain_cfg<T, TO, R1, R2, 4>(p, stream);
+    case 16: return launch_chain_cfg<T, TO, R1, R2, 16>(p, stream);
+    default: return launch_chain_cfg<T, TO, R1, R2, 8>(p, stream);
+    }
 }
 
 template <typename T, typename TO>

@@ -15,9 +15,11 @@ namespace lop {
 
 // rows [iy0, iy0 + srows) x columns [ix0, ix0 + SWE) of frame b -> tile
 // (row pitch SWE elements); NT threads participate.
+// Only columns [0, ncols) are staged (ncols <= SWE; the rest of each smem row
+// is left untouched for callers whose tile extends past the needed range).
 template <typename T, int SWE, int NT>
 __device__ __forceinline__ void stage_rows(const Common &c, int b, int ix0, int iy0, int srows,
-                                           T *tile, uint64_t *bar)
+                                           T *tile, uint64_t *bar, int ncols = SWE)
 {
     constexpr bool F = sizeof(T) == 4;
     const Geom &g = c.in;
@@ -26,7 +28,7 @@ __device__ __forceinline__ void stage_rows(const Common &c, int b, int ix0, int 
     const bool aligned = ((reinterpret_cast<uintptr_t>(fbase) | (uintptr_t)g.stride |
                            (uintptr_t)(ix0 * (int)sizeof(T))) % 16 == 0);
     constexpr int V16 = 16 / sizeof(T);                            // elements per 16 B
-    int xa = max(0, -ix0), xb = min(SWE, g.W - ix0);               // bulk span, smem columns
+    int xa = max(0, -ix0), xb = min(ncols, g.W - ix0);             // bulk span, smem columns
     xa = (xa + V16 - 1) / V16 * V16;
     xb = xb / V16 * V16;
     const bool bulk = aligned && xb > xa;
@@ -53,7 +55,7 @@ __device__ __forceinline__ void stage_rows(const Common &c, int b, int ix0, int 
         }
     }
     // element-wise part: the columns outside the bulk span of every row ...
-    const int side = bulk ? xa + (SWE - xb) : SWE;
+    const int side = bulk ? xa + (ncols - xb) : ncols;
     for (int i = threadIdx.x; i < srows * side; i += NT) {
         const int r = i / side, k = i - r * side;
         const int x = !bulk ? k : (k < xa ? k : xb + (k - xa));
