@@ -489,8 +489,6 @@ cudaError_t dispatch_swar(const ConvSep &s, cudaStream_t stream)
 
 bool conv_factor(const ConvGeneric &p, ConvSep &s) { return factor(p, s); }
 
-constexpr bool kDefaultStream = false;   // see DESIGN.md §6 (tools/tune_conv.py)
-
 bool conv_tiled_supported(const ConvGeneric &p)
 {
     if (p.c.rx != p.c.ry || p.c.rx > 4) return false;
@@ -505,14 +503,6 @@ cudaError_t launch_conv_tiled(const ConvGeneric &p, cudaStream_t stream)
     s.c = p.c;
     s.kind = p.kind;
     s.shift = p.shift;
-    // implementation: register streaming (conv_stream.cu) or smem tiles (this
-    // file); LOP_CONV_IMPL=stream|tile overrides the measured default
-    bool use_stream = kDefaultStream;
-    if (const char *env = std::getenv("LOP_CONV_IMPL")) use_stream = env[0] == 's';
-    if (use_stream) {
-        const cudaError_t e = launch_conv_stream(s, swar_ok(s), stream);
-        if (e != cudaErrorNotSupported) return e;
-    }
     switch (p.kind) {
     case CONV_F32: return dispatch_r<float, float>(s, stream);
     case CONV_U8_U8:

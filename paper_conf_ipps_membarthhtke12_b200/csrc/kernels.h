@@ -17,9 +17,6 @@ cudaError_t launch_conv_tiled(const ConvGeneric &p, cudaStream_t stream);
 bool conv_tiled_supported(const ConvGeneric &p);
 // Exact separable factorisation (false if the mask is not rank 1 / too large).
 bool conv_factor(const ConvGeneric &p, ConvSep &s);
-// Register-streaming separable convolution (conv_stream.cu); cudaErrorNotSupported
-// if no instance matches.
-cudaError_t launch_conv_stream(const ConvSep &s, bool swar, cudaStream_t stream);
 // Fused two-stage convolution; cudaErrorNotSupported if no instance matches.
 cudaError_t launch_conv_chain(const ConvChain &p, cudaStream_t stream);
 

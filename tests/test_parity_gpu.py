@@ -529,38 +529,3 @@ def test_chain_roi_offset_and_validation(lop):
         lop.convolve_chain(img, np.random.rand(3, 3).astype(np.float32), sx)
     with pytest.raises(lop.LopError):
         lop.convolve_chain(img, np.ones((7, 7), np.float32), sx)
-
-
-@pytest.mark.parametrize("rows", ["16", "32", "64"])
-def test_conv_stream_impl_bit_identical_to_tiles(lop, rows, monkeypatch):
-    """The register-streaming convolution (LOP_CONV_IMPL=stream) reproduces the
-    smem-tile kernel bit for bit (f32, u8 SWAR, u8 -> i32) in every mode, on
-    ragged shapes, frames, band views, ROI, offsets and strided views."""
-    monkeypatch.setenv("LOP_CONV_STREAM_ROWS", rows)
-    shapes = [(1, 1), (7, 5), (37, 70), (203, 1037), (77, 2100)]
-    gi, gk = oracle.gaussian_mask(5)
-    g3, k3 = oracle.gaussian_mask(3)
-    cases = []
-    for H, W in shapes:
-        f = synthetic.uniform(H, W, seed=H + W).cuda()
-        u = synthetic.uniform_u8(H, W, seed=H * W).cuda()
-        for mode in MODES:
-            cases += [lambda f=f, mode=mode: lop.gaussian(f, 5, mode, constant=0.5),
-                      lambda f=f, mode=mode: lop.sobel(f, 1, mode, constant=0.5),
-                      lambda u=u, mode=mode: lop.gaussian(u, 5, mode, constant=9),
-                      lambda u=u, mode=mode: lop.gaussian(u, 3, mode, constant=9),
-                      lambda u=u, mode=mode: lop.sobel(u, 0, mode, constant=9),
-                      lambda u=u, mode=mode: lop.convolve(u, np.outer([1, 2, 1], [1, 0, 1, 2, 1]).astype(np.int32)[:, :3], mode, shift=2)]
-    fr = torch.stack([synthetic.uniform(150, 700, seed=s) for s in range(3)]).cuda()
-    cases.append(lambda: lop.gaussian(fr, 5, "mirror"))
-    big = synthetic.angio(120, 1300, seed=4).cuda()
-    cases.append(lambda: lop.gaussian(big, 5, "repeat", roi=(17, 9, 1100, 90), offset=(3, -2)))
-    cases.append(lambda: lop.sobel(big[:, 5:1201], 0, "clamp"))
-    buf = synthetic.angio(112, 520, seed=5).cuda()
-    cases.append(lambda: lop.gaussian(buf[6:106], 5, "clamp", band=(6, 6, 40, 300)))
-    for fn in cases:
-        monkeypatch.setenv("LOP_CONV_IMPL", "tile")
-        a = fn()
-        monkeypatch.setenv("LOP_CONV_IMPL", "stream")
-        b = fn()
-        assert torch.equal(a, b)
