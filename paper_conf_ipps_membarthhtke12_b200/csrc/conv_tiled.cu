@@ -37,7 +37,6 @@ namespace lop {
 
 namespace convt {
 constexpr int NT = 128;      // threads per CTA
-constexpr int TS = 16;       // output rows per tile
 }  // namespace convt
 
 template <typename T> struct Px;

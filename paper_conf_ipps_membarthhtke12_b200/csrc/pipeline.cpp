@@ -49,6 +49,12 @@ lop_status perr(cudaError_t e, const char *what)
     return LOP_ERR_CUDA;
 }
 
+lop_status pfail(lop_status st, const char *msg)
+{
+    lop_detail::set_error(std::string("pipeline: ") + msg);
+    return st;
+}
+
 int esize(int32_t dt) { return dt == LOP_U8 ? 1 : 4; }
 
 struct DevGuard {
@@ -142,11 +148,13 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
                void *host_out, int32_t out_dtype, int64_t out_stride, int mode, double constant,
                int size_x, int size_y, Exec exec)
 {
-    if (!p || !host_in || !host_out) return LOP_ERR_INVALID;
+    if (!p || !host_in || !host_out) return pfail(LOP_ERR_INVALID, "NULL pipeline or host buffer");
     const int ry = size_y / 2;
-    if (ry > kMaxHalo || size_x / 2 > kMaxHalo) return LOP_ERR_UNSUPPORTED;
+    if (ry > kMaxHalo || size_x / 2 > kMaxHalo)
+        return pfail(LOP_ERR_UNSUPPORTED, "window larger than 63 x 63");
     const int ies = esize(in_dtype), oes = esize(out_dtype);
-    if (in_stride < (int64_t)p->W * ies || out_stride < (int64_t)p->W * oes) return LOP_ERR_INVALID;
+    if (in_stride < (int64_t)p->W * ies || out_stride < (int64_t)p->W * oes)
+        return pfail(LOP_ERR_INVALID, "host row stride smaller than the row");
     DevGuard guard(p->device);
     p->h2d_bytes = p->d2h_bytes = 0;
     static const bool trace = std::getenv("LOP_PIPELINE_TRACE") != nullptr;
@@ -224,7 +232,8 @@ extern "C" {
 lop_status lop_pipeline_create(int32_t device, int32_t width, int32_t height, int32_t chunk_rows,
                                lop_pipeline **out)
 {
-    if (!out || width <= 0 || height <= 0) return LOP_ERR_INVALID;
+    if (!out || width <= 0 || height <= 0)
+        return pfail(LOP_ERR_INVALID, "out is NULL or width/height <= 0");
     *out = nullptr;
     if (chunk_rows <= 0) chunk_rows = 512;
     chunk_rows = std::min(chunk_rows, height);
@@ -272,7 +281,7 @@ lop_status lop_pipeline_convolve(lop_pipeline *p, const void *host_in, int32_t i
                                  int64_t out_stride_bytes, int32_t mode, double constant,
                                  const lop_mask *mask)
 {
-    if (!mask) return LOP_ERR_INVALID;
+    if (!mask) return pfail(LOP_ERR_INVALID, "mask is NULL");
     return run(p, host_in, in_dtype, in_stride_bytes, host_out, out_dtype, out_stride_bytes, mode,
                constant, mask->size_x, mask->size_y,
                [&](const lop_iteration_space *is, const lop_accessor *acc, cudaStream_t s) {
@@ -282,7 +291,7 @@ lop_status lop_pipeline_convolve(lop_pipeline *p, const void *host_in, int32_t i
 
 lop_status lop_pipeline_bytes(const lop_pipeline *p, int64_t *h2d, int64_t *d2h)
 {
-    if (!p || !h2d || !d2h) return LOP_ERR_INVALID;
+    if (!p || !h2d || !d2h) return pfail(LOP_ERR_INVALID, "NULL argument");
     *h2d = p->h2d_bytes;
     *d2h = p->d2h_bytes;
     return LOP_OK;

@@ -146,3 +146,21 @@ def test_c_example_is_built_against_the_abi():
     import subprocess
     out = subprocess.run(["ldd", exe], capture_output=True, text=True).stdout
     assert "liblop.so" in out
+
+
+def test_pipeline_argument_errors_have_messages():
+    h = ctypes.c_void_p()
+    assert lop.lib.lop_pipeline_create(0, 0, 10, 128, ctypes.byref(h)) == _lib.LOP_ERR_INVALID
+    assert b"pipeline" in lop.lib.lop_last_error()
+    assert lop.lib.lop_pipeline_bilateral(None, None, 0, None, 0, 1, 0.0, 3, 3, None, 1.0,
+                                          1.0) == _lib.LOP_ERR_INVALID
+    assert lop.lib.lop_pipeline_destroy(None) == _lib.LOP_OK
+
+
+def test_chain_rejects_bad_masks_before_launch():
+    bc, acc, is_ = _views()
+    bc.size_x = bc.size_y = 7
+    m1 = _lib.lop_mask(5, 5, _lib.LOP_F32, None, 0)
+    st = lop.lib.lop_convolve_chain_execute(ctypes.byref(is_), ctypes.byref(acc), None,
+                                            ctypes.byref(m1), None)
+    assert st == _lib.LOP_ERR_INVALID

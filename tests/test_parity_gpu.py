@@ -90,7 +90,7 @@ def test_bilateral_small_shapes(lop, variant, shape, mode):
         _cmp_float(out.cpu().numpy(), ref, valid if mode == "undefined" else None)
 
 
-@pytest.mark.parametrize("size", [(5, 3), (3, 9), (15, 1), (1, 1), (9, 9), (7, 13)])
+@pytest.mark.parametrize("size", [(5, 3), (3, 9), (15, 1), (1, 1), (9, 9), (7, 13), (11, 11), (15, 15)])
 def test_bilateral_asymmetric_windows(lop, variant, size):
     img = synthetic.angio(61, 75, seed=77)
     for mode in MODES:
