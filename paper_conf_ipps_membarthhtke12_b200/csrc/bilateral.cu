@@ -40,7 +40,7 @@ __global__ void __launch_bounds__(256) bilateral_generic_kernel(const __grid_con
     const int ix = ox + c.off_x, iy = oy + c.off_y;
     // centre Input(): the pixel itself (for offset accessors it is read
     // through the boundary condition like every other tap)
-    const bool sc = p.sep && p.scaled;
+    const bool sc = p.scaled != 0;
     float centre = read_f32(c.in, b, ix, iy, c.mode, c.cval_f);
     if (sc) centre = __fmul_rn(centre, p.alpha);
     const int sx = 2 * c.rx + 1;
@@ -76,7 +76,8 @@ __global__ void __launch_bounds__(256) bilateral_generic_kernel(const __grid_con
                 int col;
                 float v = c.cval_f;
                 if (row_ok && resolve_col(ix + xf, c.in, c.mode, col)) v = __ldg(rp + col);
-                bilateral_tap(v, centre, lc[xf], p.nk, d, pacc);
+                if (sc) bilateral_tap<true>(__fmul_rn(v, p.alpha), centre, lc[xf], p.nk, d, pacc);
+                else bilateral_tap<false>(v, centre, lc[xf], p.nk, d, pacc);
             }
         }
     }
@@ -181,8 +182,20 @@ __device__ __forceinline__ void load_row(const float4 *rowv, float *v)
 }
 
 // ------------------------------------------------- user-mask tiled kernel
-template <int RX>
-__global__ void __launch_bounds__(tiled::NT, 4) bilateral_tiled_kernel(const __grid_constant__ BilateralTiled p)
+// One window row of taps for the 4 outputs of a thread with the mask row m
+// (log2 coefficients) from shared memory.
+template <int RX, int VOFF, bool SC>
+__device__ __forceinline__ void mask_row(const float *v, const float cen[4], const float *m,
+                                         float nk, float d[4], float pp[4])
+{
+#pragma unroll
+    for (int xf = 0; xf <= 2 * RX; ++xf)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) bilateral_tap<SC>(v[VOFF + xf + j], cen[j], m[xf], nk, d[j], pp[j]);
+}
+
+template <int RX, bool SC>
+__global__ void __launch_bounds__(tiled::NT, 3) bilateral_tiled_kernel(const __grid_constant__ BilateralTiled p)
 {
     using S = tiled::Shape<RX>;
     constexpr int TW = tiled::TW, TH = tiled::TH, NT = tiled::NT;
@@ -204,37 +217,51 @@ __global__ void __launch_bounds__(tiled::NT, 4) bilateral_tiled_kernel(const __g
         const int r = i / (4 * MV), k = i - r * (4 * MV);
         msk[i] = k < 2 * RX + 1 ? p.lc[r * kTiledMaskPitch + k] : 0.0f;
     }
-    stage_tile<SW>(c, b, tx0 + c.off_x - PAD, ty0 + c.off_y - ry, min(TH, roi_y1 - ty0) + 2 * ry,
-                   tile);
+    stage_tile<SW, SC>(c, b, tx0 + c.off_x - PAD, ty0 + c.off_y - ry,
+                       min(TH, roi_y1 - ty0) + 2 * ry, tile, p.alpha);
     __syncthreads();
 
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int x_out = tx0 + 4 * lane;
     const float nk = p.nk;
-    for (int r = warp; r < TH; r += NT / 32) {
-        const int oy = ty0 + r;
+    const float4 *mrow = reinterpret_cast<const float4 *>(msk);
+    // pairs of output rows (r0, r0+1) share every staged row they read
+    for (int r0 = 2 * warp; r0 < TH; r0 += 2 * (NT / 32)) {
+        const int oy = ty0 + r0;
         if (oy >= roi_y1) break;
-        const float4 cen4 = smem4[((r + ry) * SW + PAD) / 4 + lane];
-        const float cen[4] = {cen4.x, cen4.y, cen4.z, cen4.w};
-        float d[4] = {0.f, 0.f, 0.f, 0.f}, pp[4] = {0.f, 0.f, 0.f, 0.f};
-        const float4 *rowv = smem4 + (r * SW) / 4 + lane;
-        const float4 *mrow = reinterpret_cast<const float4 *>(msk);
+        const float4 c0 = smem4[((r0 + ry) * SW + PAD) / 4 + lane];
+        const float4 c1 = smem4[((r0 + 1 + ry) * SW + PAD) / 4 + lane];
+        const float cen0[4] = {c0.x, c0.y, c0.z, c0.w}, cen1[4] = {c1.x, c1.y, c1.z, c1.w};
+        float d0[4] = {0.f, 0.f, 0.f, 0.f}, p0[4] = {0.f, 0.f, 0.f, 0.f};
+        float d1[4] = {0.f, 0.f, 0.f, 0.f}, p1[4] = {0.f, 0.f, 0.f, 0.f};
+        const float4 *rowv = smem4 + (r0 * SW) / 4 + lane;
+        float v[4 * NV], m[4 * MV];
+        load_row<NV>(rowv, v);
+        load_row<MV>(mrow, m);
+        mask_row<RX, S::VOFF, SC>(v, cen0, m, nk, d0, p0);                  // yf = 0 of r0
 #pragma unroll 1
-        for (int yf = 0; yf <= 2 * ry; ++yf) {
-            float v[4 * NV];
-            load_row<NV>(rowv + yf * (SW / 4), v);
-            float m[4 * MV];
-            load_row<MV>(mrow + yf * MV, m);
-#pragma unroll
-            for (int xf = 0; xf <= 2 * RX; ++xf)
-#pragma unroll
-                for (int j = 0; j < 4; ++j)
-                    bilateral_tap(v[S::VOFF + xf + j], cen[j], m[xf], nk, d[j], pp[j]);
+        for (int r = 1; r <= 2 * ry; ++r) {
+            load_row<NV>(rowv + r * (SW / 4), v);
+            float m1[4 * MV];
+            load_row<MV>(mrow + (r - 1) * MV, m1);
+            load_row<MV>(mrow + r * MV, m);
+            mask_row<RX, S::VOFF, SC>(v, cen0, m, nk, d0, p0);              // r0, yf = r
+            mask_row<RX, S::VOFF, SC>(v, cen1, m1, nk, d1, p1);             // r0+1, yf = r-1
         }
+        load_row<NV>(rowv + (2 * ry + 1) * (SW / 4), v);
+        load_row<MV>(mrow + 2 * ry * MV, m);
+        mask_row<RX, S::VOFF, SC>(v, cen1, m, nk, d1, p1);                  // yf = 2ry of r0+1
         float res[4];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) res[j] = bilateral_finish(d[j], pp[j]);
+        for (int j = 0; j < 4; ++j)
+            res[j] = SC ? bilateral_finish_scaled(d0[j], p0[j], p.inv_alpha) : bilateral_finish(d0[j], p0[j]);
         store4(c, b, oy, x_out, res);
+        if (oy + 1 < roi_y1) {
+#pragma unroll
+            for (int j = 0; j < 4; ++j)
+                res[j] = SC ? bilateral_finish_scaled(d1[j], p1[j], p.inv_alpha) : bilateral_finish(d1[j], p1[j]);
+            store4(c, b, oy + 1, x_out, res);
+        }
     }
 }
 
@@ -344,14 +371,20 @@ static cudaError_t launch_tiled(K kernel, const P &p, size_t smem, cudaStream_t 
     return cudaGetLastError();
 }
 
-template <int RX>
-static cudaError_t launch_tiled_rx(const BilateralTiled &p, cudaStream_t stream)
+template <int RX, bool SC>
+static cudaError_t launch_tiled_rx_sc(const BilateralTiled &p, cudaStream_t stream)
 {
     using S = tiled::Shape<RX>;
     static size_t configured = 0;
     const size_t smem = (size_t)((tiled::TH + 2 * p.c.ry) * S::SW + (2 * p.c.ry + 1) * 4 * S::MV) *
                         sizeof(float);
-    return launch_tiled(bilateral_tiled_kernel<RX>, p, smem, stream, configured);
+    return launch_tiled(bilateral_tiled_kernel<RX, SC>, p, smem, stream, configured);
+}
+
+template <int RX>
+static cudaError_t launch_tiled_rx(const BilateralTiled &p, cudaStream_t stream)
+{
+    return p.scaled ? launch_tiled_rx_sc<RX, true>(p, stream) : launch_tiled_rx_sc<RX, false>(p, stream);
 }
 
 template <int RX, int NP, bool SC>

@@ -103,12 +103,21 @@ __device__ __forceinline__ float ex2_approx(float x)
 //     = ex2(lc + nk * (v - centre)^2),  lc = log2 c,  nk = -log2(e)/(2 sigma_r^2)
 //   d += w;  p += w * v
 // Explicit _rn intrinsics: never contracted or reassociated by the compiler.
+// SCALED: v, centre are alpha * I (see bilateral_weight below): exponent
+// lc - (v - centre)^2 without the FMUL by nk.
+template <bool SCALED = false>
 __device__ __forceinline__ void bilateral_tap(float v, float centre, float lc, float nk,
                                               float &d, float &p)
 {
     const float diff = __fsub_rn(v, centre);
-    const float t = __fmul_rn(diff, diff);
-    const float w = ex2_approx(__fmaf_rn(t, nk, lc));
+    float e;
+    if (SCALED) {
+        e = __fmaf_rn(-diff, diff, lc);
+    } else {
+        const float t = __fmul_rn(diff, diff);
+        e = __fmaf_rn(t, nk, lc);
+    }
+    const float w = ex2_approx(e);
     d = __fadd_rn(d, w);
     p = __fmaf_rn(w, v, p);
 }

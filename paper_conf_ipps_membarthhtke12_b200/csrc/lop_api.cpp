@@ -344,12 +344,9 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
         npoly = std::max(0, std::min(npoly, lop::bilateral_sep_max_npoly(c.rx)));
     }
     // scaled-difference exponent: LOP_BILATERAL_SCALED overrides
-    int scaled = 0;
-    if (!closeness) {
-        scaled = kDefaultScaled;
-        if (const char *env = std::getenv("LOP_BILATERAL_SCALED")) scaled = std::atoi(env) != 0;
-        if (scaled) npoly = 0;
-    }
+    int scaled = kDefaultScaled;
+    if (const char *env = std::getenv("LOP_BILATERAL_SCALED")) scaled = std::atoi(env) != 0;
+    if (scaled) npoly = 0;
     const double alpha_d = std::sqrt(kLog2e / (2.0 * (double)sigma_r * (double)sigma_r));
     const float alpha = (float)alpha_d, inv_alpha = (float)(1.0 / alpha_d);
     if (variant != LOP_VARIANT_GENERIC && tiled_ok && !closeness) {
@@ -368,6 +365,9 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
         static thread_local lop::BilateralTiled p;
         p.c = c;
         p.nk = nk;
+        p.scaled = scaled;
+        p.alpha = alpha;
+        p.inv_alpha = inv_alpha;
         for (int r = 0; r < sy; ++r)
             for (int k = 0; k < lop::kTiledMaskPitch; ++k)
                 p.lc[r * lop::kTiledMaskPitch + k] = k < sx ? lc[r * sx + k] : 0.0f;

@@ -70,6 +70,8 @@ struct BilateralSep {
 struct BilateralTiled {
     Common c;
     float nk;
+    int32_t scaled;                  // stage alpha * I; exponent lc - (J - J0)^2
+    float alpha, inv_alpha;
     float lc[kTiledMaxTaps];   // row pitch kTiledMaskPitch
 };
 

@@ -115,6 +115,28 @@ def test_bilateral_user_mask(lop, variant):
     _cmp_float(out.cpu().numpy(), ref)
 
 
+@pytest.mark.parametrize("scaled", ["0", "1"])
+@pytest.mark.parametrize("msize", [(3, 3), (5, 7), (13, 13), (9, 3), (15, 15)])
+def test_bilateral_user_mask_paths(lop, scaled, msize, monkeypatch):
+    """Listing 5's precomputed-Mask path: the 2-rows-per-thread tiled kernel
+    and the generic kernel agree bit for bit under both exponent forms, and
+    both match the oracle; ragged 70-row / 201-column tiles, every mode."""
+    monkeypatch.setenv("LOP_BILATERAL_SCALED", scaled)
+    rng = np.random.default_rng(msize[0] * 31 + msize[1])
+    cm = (rng.random(msize) + 0.05).astype(np.float32)
+    img = synthetic.angio(70, 201, seed=21)
+    for mode in MODES:
+        lop.set_variant("generic")
+        a = lop.bilateral(img.cuda(), 0.0, 0.1, mode, constant=0.5, mask=cm)
+        lop.set_variant("tiled")
+        b = lop.bilateral(img.cuda(), 0.0, 0.1, mode, constant=0.5, mask=cm)
+        lop.set_variant("auto")
+        assert torch.equal(a, b), mode
+        ref, valid = oracle.bilateral_f32(img.numpy(), 0.0, 0.1, mode, cval=0.5,
+                                          cmask=cm.astype(np.float64))
+        _cmp_float(b.cpu().numpy(), ref, valid if mode == "undefined" else None)
+
+
 def test_bilateral_generic_and_tiled_bit_identical(lop):
     img = synthetic.angio(300, 517, seed=11).cuda()
     for mode in MODES:
