@@ -13,7 +13,9 @@ One JSON line on rank 0 (driver contract):
                   (lop.Pipeline: pinned host in -> device -> pinned host out,
                   copies inside the timed region)
   roofline        the dominant kernel against its bound (SFU for the
-                  bilateral filter: 168 ex2 per pixel = (13*13 - 1))
+                  bilateral filter: 84 distinct ex2 per pixel = (13*13 - 1) / 2 with
+                  symmetric pair-sharing; frac_vs_168_ex2_per_px against the
+                  unshared count)
   cpu_baseline    the C oracle (double, OpenMP) on a bounded sample, rank 0, N=1
   clocks          nvidia-smi samples taken during the timed region
   gpu_launches    lop kernel launches inside the timed region (liblop counter)
@@ -293,20 +295,28 @@ def run_lop(args, dist, peaks):
     px_total = px_per_step_rank * dist.world * K
     value = px_total / (total_ms / 1000.0) / 1e6
     avg_launch_ms = sum(per) / len(per)
-    ex2_per_launch = taps * px_per_step_rank
+    # symmetric pair-sharing kernel (default): w(p,q) = w(q,p), so the method
+    # needs (W^2-1)/2 = 84 distinct ex2 per pixel -- SURVEY §8(d)'s tighter bound
+    pair = os.environ.get("LOP_BILATERAL_PAIR", "1") != "0"
+    ex2_px = taps // 2 if pair else taps
+    ex2_per_launch = ex2_px * px_per_step_rank
     achieved = ex2_per_launch / (avg_launch_ms / 1000.0) / 1e12
+    achieved_168 = taps * px_per_step_rank / (avg_launch_ms / 1000.0) / 1e12
     sm_mhz_peak = float(peaks.get("sm_max_mhz", 1965.0))
     peak = SM_COUNT * MUFU_PER_CLK_PER_SM * sm_mhz_peak * 1e6 / 1e12
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
         with open(tp) as f:
-            traffic = json.load(f).get("bilateral_tiled_13x13_4096", None)
-    roofline = {"bound": "alu", "kernel": "lop::bilateral_sep_kernel<6>",
+            tj = json.load(f)
+            traffic = tj.get("bilateral_13x13_4096" if pair else "bilateral_sep_13x13_4096")
+    roofline = {"bound": "alu",
+                "kernel": "lop::bilateral_pair_kernel<6>" if pair else "lop::bilateral_sep_kernel<6>",
                 "achieved": round(achieved, 4), "peak": round(peak, 4), "unit": "Tex2/s",
                 "frac": round(achieved / peak, 4), "traffic": traffic,
-                "work_per_launch": "%d ex2 (= 168 per px x %d px)" % (ex2_per_launch,
-                                                                      px_per_step_rank),
+                "work_per_launch": "%d ex2 (= %d per px x %d px)" % (ex2_per_launch, ex2_px,
+                                                                    px_per_step_rank),
+                "frac_vs_168_ex2_per_px": round(achieved_168 / peak, 4),
                 "peak_basis": "148 SM x 16 MUFU.EX2/clk x %.0f MHz (sm_max_mhz, %s)" %
                               (sm_mhz_peak, peaks["_source"]),
                 "avg_launch_ms": round(avg_launch_ms, 5)}

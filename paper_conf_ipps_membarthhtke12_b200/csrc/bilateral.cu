@@ -24,6 +24,9 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
+#include <cstdlib>
+
 #include "boundary.cuh"
 #include "lop_params.h"
 
@@ -45,6 +48,44 @@ __global__ void __launch_bounds__(256) bilateral_generic_kernel(const __grid_con
     if (sc) centre = __fmul_rn(centre, p.alpha);
     const int sx = 2 * c.rx + 1;
     float d = 0.0f, pacc = 0.0f;
+    if (p.pair) {
+        // Pair-sharing order of bilateral_pair_kernel (below): the same 169
+        // weights, each computed by the pair's owner p with q = p + (dx, dy),
+        // dy > 0 or (dy = 0, dx > 0), as ex2(lx[dx] - (J(q) - J(p))^2), and the
+        // same per-row partial sums folded in the same order:
+        //   rows above (partner side, dy = R..1), own row (own, then partner),
+        //   rows below (own side, dy = 1..R).
+        const int R = c.rx;
+        auto J = [&](int x, int y) { return __fmul_rn(read_f32(c.in, b, x, y, c.mode, c.cval_f), p.alpha); };
+        auto partner_row = [&](int dy, int dx0) {
+            float qd = 0.f, qp = 0.f;
+            for (int dx = dx0; dx <= R; ++dx) {
+                const float jp = J(ix - dx, iy - dy);
+                const float w = bilateral_weight<false, true>(centre, jp, p.lx[dx + R], p.nk);
+                if (dx == dx0) { qd = w; qp = __fmul_rn(w, jp); }
+                else { qd = __fadd_rn(qd, w); qp = __fmaf_rn(w, jp, qp); }
+            }
+            bilateral_row_fold(p.cy[dy + R], qd, qp, d, pacc);
+        };
+        auto own_row = [&](int dy, int dx0) {
+            float rd = 0.f, rp = 0.f;
+            for (int dx = dx0; dx <= R; ++dx) {
+                const float jq = J(ix + dx, iy + dy);
+                const float w = bilateral_weight<false, true>(jq, centre, p.lx[dx + R], p.nk);
+                if (dx == dx0) { rd = w; rp = __fmul_rn(w, jq); }
+                else { rd = __fadd_rn(rd, w); rp = __fmaf_rn(w, jq, rp); }
+            }
+            bilateral_row_fold(p.cy[dy + R], rd, rp, d, pacc);
+        };
+        for (int dy = R; dy >= 1; --dy) partner_row(dy, -R);
+        own_row(0, 0);
+        partner_row(0, 1);
+        for (int dy = 1; dy <= R; ++dy) own_row(dy, -R);
+        float *orow = reinterpret_cast<float *>(c.out.data + (int64_t)b * c.out.bstride +
+                                                (int64_t)oy * c.out.stride);
+        orow[ox] = bilateral_finish_scaled(d, pacc, p.inv_alpha);
+        return;
+    }
     for (int yf = -c.ry; yf <= c.ry; ++yf) {
         int row;
         const bool row_ok = resolve_row(iy + yf, c.in, c.mode, row);
@@ -354,6 +395,349 @@ __global__ void __launch_bounds__(tiled::NT, 3) bilateral_sep_kernel(const __gri
     }
 }
 
+// --------------------------------------- pair-sharing separable kernel
+// The range weight is symmetric: w(p, q) = c(q - p) s(J(q) - J(p)) = w(q, p)
+// (c is even in both axes, (J(q) - J(p))^2 = (J(p) - J(q))^2 exactly), so the
+// 168 exps of a 13x13 window are 84 distinct ones per pixel (SURVEY.md §8(d)
+// "symmetric pair-sharing").  Each pair {p, q} is evaluated once by its owner
+// p, with q = p + (dx, dy) in the half window dy > 0 or (dy = 0, dx > 0), and
+// contributes (w, w J(q)) to p and (w, w J(p)) to q.
+//  * A warp owns a 128-column frame (lane L: columns 4L..4L+3) and streams
+//    down T output rows.  Partner contributions to columns of other lanes
+//    travel by SHFL; the frame's HLN outer lanes each side are halo (they own
+//    pairs, but their own outputs would miss partners outside the frame), so
+//    a warp writes OW = 128 - 8 HLN columns.
+//  * Partner contributions to rows below (dy > 0) go to a register ring of
+//    per-row accumulators D/P[0..R]; row s is complete after step s.  The
+//    warp starts R rows early (warm-up steps evaluate only the pairs that
+//    reach row >= y0).
+//  * Input rows stream through a per-warp ring of R+2 rows in shared memory
+//    (alpha * I, boundary resolved at staging); no block-level barriers.
+// Summation order per output (mirrored by bilateral_generic_kernel, p.pair):
+// partner rows dy = R..1, own row (own, partner), own rows dy = 1..R, each a
+// left-to-right partial sum folded with cy[dy].
+#ifndef LOP_PAIR_NW
+#define LOP_PAIR_NW 2
+#endif
+#ifndef LOP_PAIR_MAXREG
+#define LOP_PAIR_MAXREG 168
+#endif
+namespace pair {
+constexpr int NW = LOP_PAIR_NW;                        // warps per CTA
+template <int R> struct Shape {
+    static constexpr int HLN = (R + 3) / 4;            // halo lanes each side
+    static constexpr int HL = 4 * HLN;                 // halo columns each side
+    static constexpr int OW = 128 - 2 * HL;            // output columns per warp
+    static constexpr int PAD = HL;                     // smem columns left of frame column 0
+    static constexpr int SW = 128 + 2 * PAD;           // smem row (floats)
+    static constexpr int NV = PAD / 2 + 1;             // float4 per lane per row: 4L-PAD .. 4L+3+PAD
+    static constexpr int NR = R + 2;                   // ring slots
+    // per-warp shared memory (floats): interleaved row-pair ring (slot k holds
+    // rows (r, r+1) as (J(r,x), J(r+1,x)) pairs), plain row ring, staging row
+    static constexpr int RING2 = NR * SW * 2, RING1 = NR * SW;
+    static constexpr int WARP_FLOATS = RING2 + RING1 + SW;
+};
+}  // namespace pair
+
+// Stage input row iy (columns ix0 .. ix0 + SW - 1) of frame b into dst as
+// alpha * I, boundary resolved per element where the row or a 4-column group
+// leaves the image.
+template <int SW>
+__device__ __forceinline__ void pair_stage_row(const Common &c, int b, int iy, int ix0, float alpha,
+                                               float4 *dst, int lane, bool vec_ok)
+{
+    const Geom &g = c.in;
+    int row;
+    const bool row_ok = resolve_row(iy, g, c.mode, row);
+    const float *rp = row_ok ? row_ptr<float>(g, b, row) : nullptr;
+#pragma unroll
+    for (int k = lane; k < SW / 4; k += 32) {
+        const int ix = ix0 + 4 * k;
+        float4 q;
+        if (row_ok && vec_ok && ix >= 0 && ix + 3 < g.W) {
+            q = __ldg(reinterpret_cast<const float4 *>(rp + ix));
+        } else {
+            float e[4];
+#pragma unroll
+            for (int jj = 0; jj < 4; ++jj) {
+                int col;
+                e[jj] = (row_ok && resolve_col(ix + jj, g, c.mode, col)) ? __ldg(rp + col) : c.cval_f;
+            }
+            q = make_float4(e[0], e[1], e[2], e[3]);
+        }
+        q.x = __fmul_rn(q.x, alpha); q.y = __fmul_rn(q.y, alpha);
+        q.z = __fmul_rn(q.z, alpha); q.w = __fmul_rn(q.w, alpha);
+        dst[k] = q;
+    }
+}
+
+// Value x of lane (this lane + o); o is a compile-time constant after unrolling.
+__device__ __forceinline__ float lane_shift(float x, int o)
+{
+    if (o == 0) return x;
+    if (o > 0) return __shfl_down_sync(0xffffffffu, x, o);
+    return __shfl_up_sync(0xffffffffu, x, -o);
+}
+
+// One (dy, dx) of the half window for this lane's 4 owners (columns j):
+// own side (rd, rp; first dx initialises) and partner side (qd, qp): receiver
+// column j' takes the weight its owner (column 4L + j' - dx) computed, from
+// lane L + floor((j' - dx) / 4).  All indices fold to constants when unrolled
+// (dx is unrolled; dy only selects the row of v, so DY0 = dy == 0).
+template <int R, int PAD, bool DY0>
+__device__ __forceinline__ void pair_tap(int dx, const float *v, const float *u, const float cen[4],
+                                         const float *lx, float nk, float rd[4], float rp[4],
+                                         float qd[4], float qp[4])
+{
+    const int dx0 = DY0 ? 0 : -R;              // own side: first dx of this row
+    const int px0 = DY0 ? 1 : -R;              // partner side: first dx of this row
+    float w[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        const float jq = v[PAD + j + dx];
+        w[j] = bilateral_weight<false, true>(jq, cen[j], lx[dx + R], nk);
+        if (dx == dx0) { rd[j] = w[j]; rp[j] = __fmul_rn(w[j], jq); }
+        else { rd[j] = __fadd_rn(rd[j], w[j]); rp[j] = __fmaf_rn(w[j], jq, rp[j]); }
+    }
+    if (DY0 && dx == 0) return;                // centre tap: no partner
+#pragma unroll
+    for (int jr = 0; jr < 4; ++jr) {
+        const int t = jr - dx;
+        const int o = t >= 0 ? t / 4 : -((-t + 3) / 4);     // floor(t / 4)
+        const float wr = lane_shift(w[t - 4 * o], o);
+        const float jp = u[PAD + t];
+        if (dx == px0) { qd[jr] = wr; qp[jr] = __fmul_rn(wr, jp); }
+        else { qd[jr] = __fadd_rn(qd[jr], wr); qp[jr] = __fmaf_rn(wr, jp, qp[jr]); }
+    }
+}
+
+__device__ __forceinline__ void fold4(float cy, const float rd[4], const float rp[4], float d[4], float pp[4])
+{
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        d[j] = __fmaf_rn(cy, rd[j], d[j]);
+        pp[j] = __fmaf_rn(cy, rp[j], pp[j]);
+    }
+}
+
+// Packed form of pair_tap for two window rows (a, b) = (s+dy, s+dy+1) at once:
+// v[i] = (J(a, col i), J(b, col i)) from the interleaved ring; each FADD2 /
+// FFMA2 lane does exactly the scalar pair_tap arithmetic of its row (same
+// rounding), so packing changes no result bit.  cen / J(p) enter as scalar
+// broadcast operands, (lx, lx) as a uniform-register pair.
+template <int R, int PAD>
+__device__ __forceinline__ void pair_tap2(int dx, const float2 *v, const float *u, const float cen[4],
+                                          const float2 *lx2, float2 rd[4], float2 rp[4],
+                                          float2 qd[4], float2 qp[4])
+{
+    float2 w[4];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+        const float2 jq = v[PAD + j + dx];
+        const float2 diff = __fadd2_rn(jq, make_float2(-cen[j], -cen[j]));
+        const float2 e = __ffma2_rn(make_float2(-diff.x, -diff.y), diff, lx2[dx + R]);
+        w[j] = make_float2(ex2_approx(e.x), ex2_approx(e.y));
+        if (dx == -R) { rd[j] = w[j]; rp[j] = __fmul2_rn(w[j], jq); }
+        else { rd[j] = __fadd2_rn(rd[j], w[j]); rp[j] = __ffma2_rn(w[j], jq, rp[j]); }
+    }
+#pragma unroll
+    for (int jr = 0; jr < 4; ++jr) {
+        const int t = jr - dx;
+        const int o = t >= 0 ? t / 4 : -((-t + 3) / 4);     // floor(t / 4)
+        const float2 wr = make_float2(lane_shift(w[t - 4 * o].x, o), lane_shift(w[t - 4 * o].y, o));
+        const float jp = u[PAD + t];
+        if (dx == -R) { qd[jr] = wr; qp[jr] = __fmul2_rn(wr, make_float2(jp, jp)); }
+        else { qd[jr] = __fadd2_rn(qd[jr], wr); qp[jr] = __ffma2_rn(wr, make_float2(jp, jp), qp[jr]); }
+    }
+}
+
+__device__ __forceinline__ void cp_async16(void *smem_dst, const void *gsrc)
+{
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_addr(smem_dst)), "l"(gsrc)
+                 : "memory");
+}
+
+// Row prefetch, part 1 (start of a step): 16-B chunks wholly inside the image
+// go global -> staging row asynchronously (LDGSTS), raw I.
+template <int SW>
+__device__ __forceinline__ void pair_issue_row(const Common &c, int b, int iy, int ix0, float4 *stg,
+                                               int lane, bool vec_ok)
+{
+    const Geom &g = c.in;
+    int row;
+    if (!vec_ok || !resolve_row(iy, g, c.mode, row)) return;
+    const float *rp = row_ptr<float>(g, b, row);
+#pragma unroll
+    for (int k = lane; k < SW / 4; k += 32) {
+        const int ix = ix0 + 4 * k;
+        if (ix >= 0 && ix + 3 < g.W) cp_async16(stg + k, rp + ix);
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+}
+
+// Part 2 (end of the step; also the synchronous initial fill with
+// from_stg = false): chunk values alpha * I (async chunks from the staging
+// row, the others element-wise with the boundary resolved) written to the
+// plain ring slot of the row, the first half of its interleaved slot and the
+// second half of the previous row's interleaved slot.
+template <int SW>
+__device__ __forceinline__ void pair_put_row(const Common &c, int b, int iy, int ix0, float alpha,
+                                             const float4 *stg, bool from_stg, float4 *plain,
+                                             float2 *first, float2 *second, int lane, bool vec_ok)
+{
+    const Geom &g = c.in;
+    int row;
+    const bool row_ok = resolve_row(iy, g, c.mode, row);
+    const float *rp = row_ok ? row_ptr<float>(g, b, row) : nullptr;
+    if (from_stg) asm volatile("cp.async.wait_all;" ::: "memory");
+#pragma unroll
+    for (int k = lane; k < SW / 4; k += 32) {
+        const int ix = ix0 + 4 * k;
+        float4 q;
+        if (row_ok && vec_ok && ix >= 0 && ix + 3 < g.W) {
+            q = from_stg ? stg[k] : __ldg(reinterpret_cast<const float4 *>(rp + ix));
+        } else {
+            float e[4];
+#pragma unroll
+            for (int jj = 0; jj < 4; ++jj) {
+                int col;
+                e[jj] = (row_ok && resolve_col(ix + jj, g, c.mode, col)) ? __ldg(rp + col) : c.cval_f;
+            }
+            q = make_float4(e[0], e[1], e[2], e[3]);
+        }
+        q.x = __fmul_rn(q.x, alpha); q.y = __fmul_rn(q.y, alpha);
+        q.z = __fmul_rn(q.z, alpha); q.w = __fmul_rn(q.w, alpha);
+        plain[k] = q;
+        float *f = reinterpret_cast<float *>(first + 4 * k);
+        f[0] = q.x; f[2] = q.y; f[4] = q.z; f[6] = q.w;
+        if (second) {
+            float *sc = reinterpret_cast<float *>(second + 4 * k) + 1;
+            sc[0] = q.x; sc[2] = q.y; sc[4] = q.z; sc[6] = q.w;
+        }
+    }
+}
+
+template <int R>
+__global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_constant__ BilateralSep p)
+{
+    using S = pair::Shape<R>;
+    constexpr int SW = S::SW, SW4 = S::SW / 4, NV = S::NV, NR = S::NR, PAD = S::PAD, HLN = S::HLN;
+    const Common &c = p.c;
+    const Geom &g = c.in;
+    extern __shared__ float4 smem4[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    float *wbase = reinterpret_cast<float *>(smem4) + warp * S::WARP_FLOATS;
+    float2 *ring2 = reinterpret_cast<float2 *>(wbase);                    // NR x SW pairs
+    float4 *ring1 = reinterpret_cast<float4 *>(wbase + S::RING2);          // NR x SW
+    float4 *stg = reinterpret_cast<float4 *>(wbase + S::RING2 + S::RING1); // SW
+    const float2 *lx2 = reinterpret_cast<const float2 *>(p.lx2);
+    const int b = blockIdx.z;
+    const int ox0 = c.roi_x0 + blockIdx.x * S::OW;               // first output column of the warp
+    const int T = p.pair_rows;
+    const int y0 = c.roi_y0 + (blockIdx.y * pair::NW + warp) * T;
+    const int roi_y1 = c.roi_y0 + c.roi_h;
+    if (y0 >= roi_y1) return;                                    // warp-uniform; warps are independent
+    const int yend = min(y0 + T, roi_y1);
+    const int ix0 = ox0 - S::HL + c.off_x - PAD;                 // input column of smem column 0
+    const bool vec_ok = ((ix0 & 3) == 0) && ((g.stride & 15) == 0) &&
+                        ((reinterpret_cast<uintptr_t>(g.data + (int64_t)b * g.bstride) & 15) == 0);
+    for (int r = 0; r <= R; ++r)                                 // rows y0-R .. y0 -> slots 0..R
+        pair_put_row<SW>(c, b, y0 - R + r + c.off_y, ix0, p.alpha, stg, false, ring1 + r * SW4,
+                         ring2 + r * SW, r > 0 ? ring2 + (r - 1) * SW : nullptr, lane, vec_ok);
+    __syncwarp();
+
+    float D[R + 1][4], P[R + 1][4];                              // D/P[k]: row s + k
+#pragma unroll
+    for (int k = 0; k <= R; ++k)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) D[k][j] = P[k][j] = 0.0f;
+    const bool out_lane = lane >= HLN && lane < 32 - HLN;
+    const int x_out = ox0 + 4 * (lane - HLN);
+    int slot0 = 0;                                               // ring slot of row s
+#pragma unroll 1
+    for (int s = y0 - R; s < yend; ++s) {
+        // prefetch row s + R + 1 (its slot = that of row s - 1, not read by step s)
+        const bool pre = s + 1 < yend;
+        if (pre) pair_issue_row<SW>(c, b, s + R + 1 + c.off_y, ix0, stg, lane, vec_ok);
+
+        const int kmin = y0 - s;                                 // warm-up: rows < y0 are not outputs
+        float u[4 * NV];
+        load_row<NV>(ring1 + slot0 * SW4 + lane, u);
+        const float cen[4] = {u[PAD], u[PAD + 1], u[PAD + 2], u[PAD + 3]};
+        if (kmin <= 0) {                                         // dy = 0: own row (scalar)
+            float rd[4], rp[4], qd[4], qp[4];
+#pragma unroll
+            for (int dx = 0; dx <= R; ++dx) pair_tap<R, PAD, true>(dx, u, u, cen, p.lx, p.nk, rd, rp, qd, qp);
+            const float cy = p.cy[R];
+            fold4(cy, rd, rp, D[0], P[0]);
+            fold4(cy, qd, qp, D[0], P[0]);
+        }
+#pragma unroll 1
+        for (int dy = 1; dy + 1 <= R; dy += 2) {                 // row pairs (dy, dy+1): packed
+            if (dy + 1 < kmin) continue;
+            const int sl = slot0 + dy >= NR ? slot0 + dy - NR : slot0 + dy;
+            float2 v[4 * NV];
+            {
+                const float4 *src = reinterpret_cast<const float4 *>(ring2 + sl * SW) + 2 * lane;
+#pragma unroll
+                for (int k = 0; k < 2 * NV; ++k) {
+                    const float4 q = src[k];
+                    v[2 * k] = make_float2(q.x, q.y);
+                    v[2 * k + 1] = make_float2(q.z, q.w);
+                }
+            }
+            float2 rd[4], rp[4], qd[4], qp[4];
+#pragma unroll
+            for (int dx = -R; dx <= R; ++dx) pair_tap2<R, PAD>(dx, v, u, cen, lx2, rd, rp, qd, qp);
+            const float cya = p.cy[dy + R], cyb = p.cy[dy + 1 + R];
+            float ta[4], tb[4], sa[4], sb[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) { ta[j] = rd[j].x; sa[j] = rp[j].x; tb[j] = rd[j].y; sb[j] = rp[j].y; }
+            fold4(cya, ta, sa, D[0], P[0]);
+            fold4(cyb, tb, sb, D[0], P[0]);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) { ta[j] = qd[j].x; sa[j] = qp[j].x; tb[j] = qd[j].y; sb[j] = qp[j].y; }
+            switch (dy) {                                        // partner rows: register ring
+#define LOP_PAIR_FOLD(K) case K: if constexpr (K + 1 <= R) { fold4(cya, ta, sa, D[K], P[K]); fold4(cyb, tb, sb, D[K + 1], P[K + 1]); } break;
+            LOP_PAIR_FOLD(1) LOP_PAIR_FOLD(3) LOP_PAIR_FOLD(5)
+#undef LOP_PAIR_FOLD
+            default: break;
+            }
+        }
+        if constexpr (R % 2 == 1) {                              // odd R: last row dy = R (scalar)
+            const int sl = slot0 + R >= NR ? slot0 + R - NR : slot0 + R;
+            float v[4 * NV];
+            load_row<NV>(ring1 + sl * SW4 + lane, v);
+            float rd[4], rp[4], qd[4], qp[4];
+#pragma unroll
+            for (int dx = -R; dx <= R; ++dx) pair_tap<R, PAD, false>(dx, v, u, cen, p.lx, p.nk, rd, rp, qd, qp);
+            const float cy = p.cy[2 * R];
+            fold4(cy, rd, rp, D[0], P[0]);
+            fold4(cy, qd, qp, D[R], P[R]);
+        }
+        if (s >= y0 && out_lane) {
+            float res[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) res[j] = bilateral_finish_scaled(D[0][j], P[0][j], p.inv_alpha);
+            if (x_out < c.roi_x0 + c.roi_w) store4(c, b, s, x_out, res);
+        }
+#pragma unroll
+        for (int k = 0; k < R; ++k)
+#pragma unroll
+            for (int j = 0; j < 4; ++j) { D[k][j] = D[k + 1][j]; P[k][j] = P[k + 1][j]; }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) D[R][j] = P[R][j] = 0.0f;
+        if (pre) {
+            const int sn = slot0 + R + 1 >= NR ? slot0 + R + 1 - NR : slot0 + R + 1;
+            const int sp = slot0 + R >= NR ? slot0 + R - NR : slot0 + R;
+            pair_put_row<SW>(c, b, s + R + 1 + c.off_y, ix0, p.alpha, stg, true, ring1 + sn * SW4,
+                             ring2 + sn * SW, ring2 + sp * SW, lane, vec_ok);
+        }
+        __syncwarp();
+        slot0 = slot0 + 1 == NR ? 0 : slot0 + 1;
+    }
+}
+
 // ------------------------------------------------------------- launchers
 template <typename P, typename K>
 static cudaError_t launch_tiled(K kernel, const P &p, size_t smem, cudaStream_t stream,
@@ -412,6 +796,73 @@ static cudaError_t launch_sep_rx(const BilateralSep &p, cudaStream_t stream)
 }
 
 int bilateral_sep_max_npoly(int rx) { return rx >= 4 ? 1 : 0; }
+
+// Pair kernel: rows per warp T from a wave-quantisation model (the paper's
+// Alg. 2 idea -- pick the configuration from occupancy -- on B200 terms):
+// cost(T) = waves(T) * (T + warm-up), waves = ceil(CTAs / resident CTAs);
+// LOP_PAIR_ROWS overrides.
+template <int R>
+static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
+{
+    using S = pair::Shape<R>;
+    static int resident = 0;
+    const size_t smem = (size_t)pair::NW * S::WARP_FLOATS * sizeof(float);
+    if (!resident) {
+        int dev = 0, sms = 0, per_sm = 0;
+        cudaError_t e = cudaFuncSetAttribute(bilateral_pair_kernel<R>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e == cudaSuccess) e = cudaGetDevice(&dev);
+        if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (e == cudaSuccess)
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bilateral_pair_kernel<R>,
+                                                              pair::NW * 32, smem);
+        if (e != cudaSuccess) return e;
+        resident = std::max(1, sms * per_sm);
+    }
+    BilateralSep p = p0;
+    const int64_t strips = (p.c.roi_w + S::OW - 1) / S::OW;
+    int T = 0;
+    if (const char *env = std::getenv("LOP_PAIR_ROWS")) T = std::atoi(env);
+    static thread_local int64_t memo_key[3] = {-1, -1, -1};
+    static thread_local int memo_T = 0;
+    if (T <= 0 && memo_key[0] == p.c.roi_h && memo_key[1] == strips && memo_key[2] == p.c.batch)
+        T = memo_T;
+    if (T <= 0) {
+        // every T from 8 to the ROI height: waves of resident CTAs x rows per warp
+        // (+ warm-up); a partial wave costs a full one (few warps per SM
+        // cannot saturate the SFU)
+        double best = 0;
+        const int tmax = std::max(8, p.c.roi_h);
+        for (int t = 8; t <= tmax; ++t) {
+            const int64_t segs = (p.c.roi_h + t - 1) / t;
+            const int64_t ctas = strips * ((segs + pair::NW - 1) / pair::NW) * p.c.batch;
+            const double cost = (double)((ctas + resident - 1) / resident) * (t + 0.55 * R);
+            if (T == 0 || cost < best) { best = cost; T = t; }
+            if (segs == 1) break;
+        }
+        memo_key[0] = p.c.roi_h; memo_key[1] = strips; memo_key[2] = p.c.batch;
+        memo_T = T;
+    }
+    p.pair_rows = T;
+    const int64_t segs = (p.c.roi_h + T - 1) / T;
+    dim3 grid((unsigned)strips, (unsigned)((segs + pair::NW - 1) / pair::NW), p.c.batch);
+    bilateral_pair_kernel<R><<<grid, pair::NW * 32, smem, stream>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_bilateral_pair(const BilateralSep &p, cudaStream_t stream)
+{
+    switch (p.c.rx) {
+    case 1: return launch_pair_r<1>(p, stream);
+    case 2: return launch_pair_r<2>(p, stream);
+    case 3: return launch_pair_r<3>(p, stream);
+    case 4: return launch_pair_r<4>(p, stream);
+    case 5: return launch_pair_r<5>(p, stream);
+    case 6: return launch_pair_r<6>(p, stream);
+    case 7: return launch_pair_r<7>(p, stream);
+    default: return cudaErrorInvalidValue;
+    }
+}
 
 cudaError_t launch_bilateral_tiled(const BilateralTiled &p, cudaStream_t stream)
 {

@@ -9,6 +9,7 @@ namespace lop {
 cudaError_t launch_bilateral_generic(const BilateralGeneric &p, cudaStream_t stream);
 cudaError_t launch_bilateral_tiled(const BilateralTiled &p, cudaStream_t stream);
 cudaError_t launch_bilateral_sep(const BilateralSep &p, cudaStream_t stream);
+cudaError_t launch_bilateral_pair(const BilateralSep &p, cudaStream_t stream);
 int bilateral_sep_max_npoly(int rx);
 cudaError_t launch_conv_generic(const ConvGeneric &p, cudaStream_t stream);
 // Tiled convolution; returns cudaErrorNotSupported when no instance matches

@@ -53,6 +53,7 @@ int elem_size(int32_t dt)
 const double kLog2e = 1.4426950408889634073599246810019;
 const int kDefaultNpoly = 0;   // MUFU offload: slower on B200, kept for tuning
 const int kDefaultScaled = 1;  // scaled-difference exponent: +2.5 % on B200
+const int kDefaultPair = 1;    // symmetric pair-sharing kernel
 
 // ---------------------------------------------------------------- validation
 lop_status check_image(const lop_image &im, const char *name)
@@ -347,6 +348,11 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
     int scaled = kDefaultScaled;
     if (const char *env = std::getenv("LOP_BILATERAL_SCALED")) scaled = std::atoi(env) != 0;
     if (scaled) npoly = 0;
+    // symmetric pair-sharing: square separable windows, scaled
+    // exponent; LOP_BILATERAL_PAIR overrides
+    int pair = kDefaultPair;
+    if (const char *env = std::getenv("LOP_BILATERAL_PAIR")) pair = std::atoi(env) != 0;
+    pair = pair && !closeness && scaled && c.rx == c.ry && c.rx >= 1 && c.rx <= lop::kTiledMaxRX;
     const double alpha_d = std::sqrt(kLog2e / (2.0 * (double)sigma_r * (double)sigma_r));
     const float alpha = (float)alpha_d, inv_alpha = (float)(1.0 / alpha_d);
     if (variant != LOP_VARIANT_GENERIC && tiled_ok && !closeness) {
@@ -359,6 +365,9 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
         p.inv_alpha = inv_alpha;
         std::memcpy(p.lx, lx, sizeof(float) * sx);
         std::memcpy(p.cy, cy, sizeof(float) * sy);
+        for (int k = 0; k < sx; ++k) p.lx2[2 * k] = p.lx2[2 * k + 1] = lx[k];
+        p.pair_rows = 0;
+        if (pair) return launched(lop::launch_bilateral_pair(p, stream), "bilateral_pair launch");
         return launched(lop::launch_bilateral_sep(p, stream), "bilateral_sep launch");
     }
     if (variant != LOP_VARIANT_GENERIC && tiled_ok) {
@@ -377,6 +386,7 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
     p.c = c;
     p.nk = nk;
     p.sep = closeness ? 0 : 1;
+    p.pair = pair;
     p.npoly = npoly;
     p.scaled = scaled;
     p.alpha = alpha;

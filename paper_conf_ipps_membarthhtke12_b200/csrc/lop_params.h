@@ -53,6 +53,7 @@ struct BilateralGeneric {
     int32_t sep;
     int32_t npoly;                   // sep form: columns xf = -rx .. -rx+npoly-1 use ex2_poly
     int32_t scaled;                  // sep form: scaled-difference exponent (alpha * I)
+    int32_t pair;                    // sep form: symmetric pair-sharing summation order
     float alpha, inv_alpha;
     float lx[2 * kMaxRadius + 1];
     float cy[2 * kMaxRadius + 1];
@@ -63,9 +64,11 @@ struct BilateralSep {
     float nk;
     int32_t npoly;                   // leftmost npoly window columns use ex2_poly (FMA pipe)
     int32_t scaled;                  // stage alpha * I; exponent lx - (J - J0)^2
+    int32_t pair_rows;               // pair kernel: output rows per warp (0: not the pair kernel)
     float alpha, inv_alpha;          // alpha = sqrt(log2(e) / (2 sigma_r^2))
     float lx[2 * kTiledMaxRX + 1];   // log2 of the x factor (compile-time indexed)
     float cy[2 * kMaxRadius + 1];    // linear y factor
+    alignas(8) float lx2[2 * (2 * kTiledMaxRX + 1)];   // (lx, lx) pairs: packed FFMA2 operand
 };
 struct BilateralTiled {
     Common c;
