@@ -433,43 +433,12 @@ template <int R> struct Shape {
     static constexpr int NV = PAD / 2 + 1;             // float4 per lane per row: 4L-PAD .. 4L+3+PAD
     static constexpr int NR = R + 2;                   // ring slots
     // per-warp shared memory (floats): interleaved row-pair ring (slot k holds
-    // rows (r, r+1) as (J(r,x), J(r+1,x)) pairs), plain row ring, staging row
+    // rows (r, r+1) as (J(r,x), J(r+1,x)) pairs), plain row ring, staging row,
+    // column map (ints)
     static constexpr int RING2 = NR * SW * 2, RING1 = NR * SW;
-    static constexpr int WARP_FLOATS = RING2 + RING1 + SW;
+    static constexpr int WARP_FLOATS = RING2 + RING1 + SW + SW;   // + staging row, column map
 };
 }  // namespace pair
-
-// Stage input row iy (columns ix0 .. ix0 + SW - 1) of frame b into dst as
-// alpha * I, boundary resolved per element where the row or a 4-column group
-// leaves the image.
-template <int SW>
-__device__ __forceinline__ void pair_stage_row(const Common &c, int b, int iy, int ix0, float alpha,
-                                               float4 *dst, int lane, bool vec_ok)
-{
-    const Geom &g = c.in;
-    int row;
-    const bool row_ok = resolve_row(iy, g, c.mode, row);
-    const float *rp = row_ok ? row_ptr<float>(g, b, row) : nullptr;
-#pragma unroll
-    for (int k = lane; k < SW / 4; k += 32) {
-        const int ix = ix0 + 4 * k;
-        float4 q;
-        if (row_ok && vec_ok && ix >= 0 && ix + 3 < g.W) {
-            q = __ldg(reinterpret_cast<const float4 *>(rp + ix));
-        } else {
-            float e[4];
-#pragma unroll
-            for (int jj = 0; jj < 4; ++jj) {
-                int col;
-                e[jj] = (row_ok && resolve_col(ix + jj, g, c.mode, col)) ? __ldg(rp + col) : c.cval_f;
-            }
-            q = make_float4(e[0], e[1], e[2], e[3]);
-        }
-        q.x = __fmul_rn(q.x, alpha); q.y = __fmul_rn(q.y, alpha);
-        q.z = __fmul_rn(q.z, alpha); q.w = __fmul_rn(q.w, alpha);
-        dst[k] = q;
-    }
-}
 
 // Value x of lane (this lane + o); o is a compile-time constant after unrolling.
 __device__ __forceinline__ float lane_shift(float x, int o)
@@ -557,53 +526,80 @@ __device__ __forceinline__ void cp_async16(void *smem_dst, const void *gsrc)
                  : "memory");
 }
 
-// Row prefetch, part 1 (start of a step): 16-B chunks wholly inside the image
-// go global -> staging row asynchronously (LDGSTS), raw I.
+__device__ __forceinline__ void cp_async4(void *smem_dst, const void *gsrc)
+{
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_addr(smem_dst)), "l"(gsrc)
+                 : "memory");
+}
+
+// Column map of a warp's frame, resolved once per kernel (columns do not
+// change from row to row): cm[i] = input column read for smem column i, or -1
+// where CONSTANT substitutes the constant (Table I).
 template <int SW>
-__device__ __forceinline__ void pair_issue_row(const Common &c, int b, int iy, int ix0, float4 *stg,
-                                               int lane, bool vec_ok)
+__device__ __forceinline__ void pair_colmap(const Common &c, int ix0, int *cm, int lane)
+{
+#pragma unroll
+    for (int i = lane; i < SW; i += 32) {
+        int col;
+        cm[i] = resolve_col(ix0 + i, c.in, c.mode, col) ? col : -1;
+    }
+}
+
+// Row fetch, part 1: raw I of input row iy (smem columns 0 .. SW-1) goes
+// global -> dst asynchronously: 16-B chunks wholly inside the image as one
+// LDGSTS.128, border chunks element-wise through the column map (LDGSTS.32).
+// Nothing is fetched for a CONSTANT row.  Border warps thus never wait on a
+// synchronous load, and the per-element boundary arithmetic (the modulo of
+// REPEAT / MIRROR) is paid once per kernel, not per row (mode invariance, E5).
+template <int SW>
+__device__ __forceinline__ void pair_issue_row(const Common &c, int b, int iy, int ix0, float4 *dst,
+                                               const int *cm, int lane, bool vec_ok)
 {
     const Geom &g = c.in;
     int row;
-    if (!vec_ok || !resolve_row(iy, g, c.mode, row)) return;
-    const float *rp = row_ptr<float>(g, b, row);
+    if (resolve_row(iy, g, c.mode, row)) {
+        const float *rp = row_ptr<float>(g, b, row);
 #pragma unroll
-    for (int k = lane; k < SW / 4; k += 32) {
-        const int ix = ix0 + 4 * k;
-        if (ix >= 0 && ix + 3 < g.W) cp_async16(stg + k, rp + ix);
+        for (int k = lane; k < SW / 4; k += 32) {
+            const int ix = ix0 + 4 * k;
+            if (vec_ok && ix >= 0 && ix + 3 < g.W) {
+                cp_async16(dst + k, rp + ix);
+            } else {
+                float *d = reinterpret_cast<float *>(dst + k);
+#pragma unroll
+                for (int jj = 0; jj < 4; ++jj)
+                    if (cm[4 * k + jj] >= 0) cp_async4(d + jj, rp + cm[4 * k + jj]);
+            }
+        }
     }
     asm volatile("cp.async.commit_group;" ::: "memory");
 }
 
-// Part 2 (end of the step; also the synchronous initial fill with
-// from_stg = false): chunk values alpha * I (async chunks from the staging
-// row, the others element-wise with the boundary resolved) written to the
-// plain ring slot of the row, the first half of its interleaved slot and the
-// second half of the previous row's interleaved slot.
+// Part 2 (after cp.async.wait_all): chunk values alpha * I (fetched chunks
+// from src, CONSTANT elements substituted) written to the plain ring slot of
+// the row (may alias src: each lane reads its chunk before writing it), the
+// first half of its interleaved slot and the second half of the previous
+// row's interleaved slot.
 template <int SW>
-__device__ __forceinline__ void pair_put_row(const Common &c, int b, int iy, int ix0, float alpha,
-                                             const float4 *stg, bool from_stg, float4 *plain,
-                                             float2 *first, float2 *second, int lane, bool vec_ok)
+__device__ __forceinline__ void pair_put_row(const Common &c, int iy, int ix0, float alpha,
+                                             const float4 *src, float4 *plain, float2 *first,
+                                             float2 *second, const int *cm, int lane, bool vec_ok)
 {
     const Geom &g = c.in;
     int row;
     const bool row_ok = resolve_row(iy, g, c.mode, row);
-    const float *rp = row_ok ? row_ptr<float>(g, b, row) : nullptr;
-    if (from_stg) asm volatile("cp.async.wait_all;" ::: "memory");
 #pragma unroll
     for (int k = lane; k < SW / 4; k += 32) {
         const int ix = ix0 + 4 * k;
         float4 q;
         if (row_ok && vec_ok && ix >= 0 && ix + 3 < g.W) {
-            q = from_stg ? stg[k] : __ldg(reinterpret_cast<const float4 *>(rp + ix));
+            q = src[k];
         } else {
-            float e[4];
-#pragma unroll
-            for (int jj = 0; jj < 4; ++jj) {
-                int col;
-                e[jj] = (row_ok && resolve_col(ix + jj, g, c.mode, col)) ? __ldg(rp + col) : c.cval_f;
-            }
-            q = make_float4(e[0], e[1], e[2], e[3]);
+            const float4 r = src[k];
+            q.x = (row_ok && cm[4 * k + 0] >= 0) ? r.x : c.cval_f;
+            q.y = (row_ok && cm[4 * k + 1] >= 0) ? r.y : c.cval_f;
+            q.z = (row_ok && cm[4 * k + 2] >= 0) ? r.z : c.cval_f;
+            q.w = (row_ok && cm[4 * k + 3] >= 0) ? r.w : c.cval_f;
         }
         q.x = __fmul_rn(q.x, alpha); q.y = __fmul_rn(q.y, alpha);
         q.z = __fmul_rn(q.z, alpha); q.w = __fmul_rn(q.w, alpha);
@@ -630,6 +626,7 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
     float2 *ring2 = reinterpret_cast<float2 *>(wbase);                    // NR x SW pairs
     float4 *ring1 = reinterpret_cast<float4 *>(wbase + S::RING2);          // NR x SW
     float4 *stg = reinterpret_cast<float4 *>(wbase + S::RING2 + S::RING1); // SW
+    int *cm = reinterpret_cast<int *>(wbase + S::RING2 + S::RING1 + SW);   // SW
     const float2 *lx2 = reinterpret_cast<const float2 *>(p.lx2);
     const int b = blockIdx.z;
     const int ox0 = c.roi_x0 + blockIdx.x * S::OW;               // first output column of the warp
@@ -641,9 +638,14 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
     const int ix0 = ox0 - S::HL + c.off_x - PAD;                 // input column of smem column 0
     const bool vec_ok = ((ix0 & 3) == 0) && ((g.stride & 15) == 0) &&
                         ((reinterpret_cast<uintptr_t>(g.data + (int64_t)b * g.bstride) & 15) == 0);
+    pair_colmap<SW>(c, ix0, cm, lane);
+    __syncwarp();
     for (int r = 0; r <= R; ++r)                                 // rows y0-R .. y0 -> slots 0..R
-        pair_put_row<SW>(c, b, y0 - R + r + c.off_y, ix0, p.alpha, stg, false, ring1 + r * SW4,
-                         ring2 + r * SW, r > 0 ? ring2 + (r - 1) * SW : nullptr, lane, vec_ok);
+        pair_issue_row<SW>(c, b, y0 - R + r + c.off_y, ix0, ring1 + r * SW4, cm, lane, vec_ok);
+    asm volatile("cp.async.wait_all;" ::: "memory");
+    for (int r = 0; r <= R; ++r)
+        pair_put_row<SW>(c, y0 - R + r + c.off_y, ix0, p.alpha, ring1 + r * SW4, ring1 + r * SW4,
+                         ring2 + r * SW, r > 0 ? ring2 + (r - 1) * SW : nullptr, cm, lane, vec_ok);
     __syncwarp();
 
     float D[R + 1][4], P[R + 1][4];                              // D/P[k]: row s + k
@@ -658,7 +660,7 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
     for (int s = y0 - R; s < yend; ++s) {
         // prefetch row s + R + 1 (its slot = that of row s - 1, not read by step s)
         const bool pre = s + 1 < yend;
-        if (pre) pair_issue_row<SW>(c, b, s + R + 1 + c.off_y, ix0, stg, lane, vec_ok);
+        if (pre) pair_issue_row<SW>(c, b, s + R + 1 + c.off_y, ix0, stg, cm, lane, vec_ok);
 
         const int kmin = y0 - s;                                 // warm-up: rows < y0 are not outputs
         float u[4 * NV];
@@ -730,8 +732,9 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
         if (pre) {
             const int sn = slot0 + R + 1 >= NR ? slot0 + R + 1 - NR : slot0 + R + 1;
             const int sp = slot0 + R >= NR ? slot0 + R - NR : slot0 + R;
-            pair_put_row<SW>(c, b, s + R + 1 + c.off_y, ix0, p.alpha, stg, true, ring1 + sn * SW4,
-                             ring2 + sn * SW, ring2 + sp * SW, lane, vec_ok);
+            asm volatile("cp.async.wait_all;" ::: "memory");
+            pair_put_row<SW>(c, s + R + 1 + c.off_y, ix0, p.alpha, stg, ring1 + sn * SW4,
+                             ring2 + sn * SW, ring2 + sp * SW, cm, lane, vec_ok);
         }
         __syncwarp();
         slot0 = slot0 + 1 == NR ? 0 : slot0 + 1;
