@@ -33,6 +33,15 @@
 namespace lop {
 
 // ------------------------------------------------------------------ generic
+// pair kernel lane groups (see bilateral_pair_kernel): floor(t / 4), and
+// the dx of the first partner value of receiving column jr (owner push)
+__host__ __device__ constexpr int pair_floor4(int t) { return t >= 0 ? t / 4 : -((-t + 3) / 4); }
+__host__ __device__ constexpr int pair_first_dx(int jr, int dx0, int R)
+{
+    return pair_floor4(jr - dx0) == 0 ? dx0
+                                      : (jr - 4 * pair_floor4(jr - dx0) < R ? jr - 4 * pair_floor4(jr - dx0) : R);
+}
+
 __global__ void __launch_bounds__(256) bilateral_generic_kernel(const __grid_constant__ BilateralGeneric p)
 {
     const Common &c = p.c;
@@ -57,13 +66,30 @@ __global__ void __launch_bounds__(256) bilateral_generic_kernel(const __grid_con
         //   rows below (own side, dy = 1..R).
         const int R = c.rx;
         auto J = [&](int x, int y) { return __fmul_rn(read_f32(c.in, b, x, y, c.mode, c.cval_f), p.alpha); };
+        // partner terms of a row in dx order; a run of dx whose owners sit in
+        // another lane of the pair kernel (column group floor(x / 4)) is
+        // pre-summed by that lane and added as one value (owner push)
+        const int jr = ox & 3;
         auto partner_row = [&](int dy, int dx0) {
             float qd = 0.f, qp = 0.f;
-            for (int dx = dx0; dx <= R; ++dx) {
-                const float jp = J(ix - dx, iy - dy);
-                const float w = bilateral_weight<false, true>(centre, jp, p.lx[dx + R], p.nk);
-                if (dx == dx0) { qd = w; qp = __fmul_rn(w, jp); }
-                else { qd = __fadd_rn(qd, w); qp = __fmaf_rn(w, jp, qp); }
+            for (int dx = dx0; dx <= R;) {
+                const int o = pair_floor4(jr - dx);
+                const int dx_end = o == 0 ? dx : min(jr - 4 * o, R);
+                float sd = 0.f, sp = 0.f;
+                for (int k = dx; k <= dx_end; ++k) {
+                    const float jp = J(ix - k, iy - dy);
+                    const float w = bilateral_weight<false, true>(centre, jp, p.lx[k + R], p.nk);
+                    if (k == dx) { sd = w; sp = __fmul_rn(w, jp); }
+                    else { sd = __fadd_rn(sd, w); sp = __fmaf_rn(w, jp, sp); }
+                }
+                if (dx == dx0) { qd = sd; qp = sp; }
+                else if (o == 0) {
+                    // in-lane term: accumulated like an own term
+                    const float jp = J(ix - dx, iy - dy);
+                    const float w = bilateral_weight<false, true>(centre, jp, p.lx[dx + R], p.nk);
+                    qd = __fadd_rn(qd, w); qp = __fmaf_rn(w, jp, qp);
+                } else { qd = __fadd_rn(qd, sd); qp = __fadd_rn(qp, sp); }
+                dx = dx_end + 1;
             }
             bilateral_row_fold(p.cy[dy + R], qd, qp, d, pacc);
         };
@@ -448,35 +474,60 @@ __device__ __forceinline__ float lane_shift(float x, int o)
     return __shfl_up_sync(0xffffffffu, x, -o);
 }
 
-// One (dy, dx) of the half window for this lane's 4 owners (columns j):
-// own side (rd, rp; first dx initialises) and partner side (qd, qp): receiver
-// column j' takes the weight its owner (column 4L + j' - dx) computed, from
-// lane L + floor((j' - dx) / 4).  All indices fold to constants when unrolled
-// (dx is unrolled; dy only selects the row of v, so DY0 = dy == 0).
+// Partner-side exchange (owner push).  Owner column j of this lane pairs with
+// q at column c = j + dx (relative to the lane's first column).  A partner in
+// this lane (0 <= c <= 3) takes (w, w J(p)) directly; one in another lane is
+// served by an outgoing sum per destination column, accumulated by the owner
+// over the dx that reach c (owners j = c - dx, dx ascending) and sent with one
+// SHFL per value when complete (at dx = min(c, R)) -- 2 SHFL per destination
+// column and row instead of one per pair.  The receiver (column jr = c - 4o of
+// lane L + o, o = floor(c / 4)) adds the sums in dx order of its partner terms,
+// each off-lane run of dx as one pre-summed value.
+// pair_first_dx: dx at which receiver column jr gets its first partner value,
+// for partner dx running dx0 .. R.
+// One window row dy of the half window for this lane's 4 owners (scalar; DY0:
+// dy = 0, own side dx = 0..R with the centre, partner side dx = 1..R): own
+// sums (rd, rp) and partner sums (qd, qp) of the receiving columns.
 template <int R, int PAD, bool DY0>
-__device__ __forceinline__ void pair_tap(int dx, const float *v, const float *u, const float cen[4],
-                                         const float *lx, float nk, float rd[4], float rp[4],
-                                         float qd[4], float qp[4])
+__device__ __forceinline__ void pair_row1(const float *v, const float cen[4], const float *lx, float nk,
+                                          float rd[4], float rp[4], float qd[4], float qp[4])
 {
-    const int dx0 = DY0 ? 0 : -R;              // own side: first dx of this row
-    const int px0 = DY0 ? 1 : -R;              // partner side: first dx of this row
-    float w[4];
+    constexpr int dx0 = DY0 ? 0 : -R;             // own side: first dx of this row
+    constexpr int px0 = DY0 ? 1 : -R;             // partner side: first dx of this row
+    float od[2 * R + 4], op[2 * R + 4];           // outgoing sums, index c + R
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-        const float jq = v[PAD + j + dx];
-        w[j] = bilateral_weight<false, true>(jq, cen[j], lx[dx + R], nk);
-        if (dx == dx0) { rd[j] = w[j]; rp[j] = __fmul_rn(w[j], jq); }
-        else { rd[j] = __fadd_rn(rd[j], w[j]); rp[j] = __fmaf_rn(w[j], jq, rp[j]); }
-    }
-    if (DY0 && dx == 0) return;                // centre tap: no partner
+    for (int dx = dx0; dx <= R; ++dx) {
+        float w[4];
 #pragma unroll
-    for (int jr = 0; jr < 4; ++jr) {
-        const int t = jr - dx;
-        const int o = t >= 0 ? t / 4 : -((-t + 3) / 4);     // floor(t / 4)
-        const float wr = lane_shift(w[t - 4 * o], o);
-        const float jp = u[PAD + t];
-        if (dx == px0) { qd[jr] = wr; qp[jr] = __fmul_rn(wr, jp); }
-        else { qd[jr] = __fadd_rn(qd[jr], wr); qp[jr] = __fmaf_rn(wr, jp, qp[jr]); }
+        for (int j = 0; j < 4; ++j) {
+            const float jq = v[PAD + j + dx];
+            w[j] = bilateral_weight<false, true>(jq, cen[j], lx[dx + R], nk);
+            if (dx == dx0) { rd[j] = w[j]; rp[j] = __fmul_rn(w[j], jq); }
+            else { rd[j] = __fadd_rn(rd[j], w[j]); rp[j] = __fmaf_rn(w[j], jq, rp[j]); }
+        }
+        if (DY0 && dx == 0) continue;             // centre tap: no partner
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int c = j + dx;
+            if (c >= 0 && c <= 3) {
+                if (dx == pair_first_dx(c, px0, R)) { qd[c] = w[j]; qp[c] = __fmul_rn(w[j], cen[j]); }
+                else { qd[c] = __fadd_rn(qd[c], w[j]); qp[c] = __fmaf_rn(w[j], cen[j], qp[c]); }
+            } else {
+                const int first = c - 3 > px0 ? c - 3 : px0;
+                if (dx == first) { od[c + R] = w[j]; op[c + R] = __fmul_rn(w[j], cen[j]); }
+                else { od[c + R] = __fadd_rn(od[c + R], w[j]); op[c + R] = __fmaf_rn(w[j], cen[j], op[c + R]); }
+            }
+        }
+        // destinations complete at this dx: c = dx (c < 0), or c >= 4 with min(c, R) == dx
+#pragma unroll
+        for (int c = -R; c <= R + 3; ++c) {
+            if (c >= 0 && c <= 3) continue;
+            if ((c < R ? c : R) != dx) continue;
+            const int o = pair_floor4(c), jr = c - 4 * o;
+            const float a = lane_shift(od[c + R], -o), bq = lane_shift(op[c + R], -o);
+            if (dx == pair_first_dx(jr, px0, R)) { qd[jr] = a; qp[jr] = bq; }
+            else { qd[jr] = __fadd_rn(qd[jr], a); qp[jr] = __fadd_rn(qp[jr], bq); }
+        }
     }
 }
 
@@ -489,34 +540,51 @@ __device__ __forceinline__ void fold4(float cy, const float rd[4], const float r
     }
 }
 
-// Packed form of pair_tap for two window rows (a, b) = (s+dy, s+dy+1) at once:
-// v[i] = (J(a, col i), J(b, col i)) from the interleaved ring; each FADD2 /
-// FFMA2 lane does exactly the scalar pair_tap arithmetic of its row (same
+// Packed form of pair_row1 for two window rows (a, b) = (s+dy, s+dy+1) at
+// once: v[i] = (J(a, col i), J(b, col i)) from the interleaved ring; each
+// FADD2 / FFMA2 lane does exactly the scalar arithmetic of its row (same
 // rounding), so packing changes no result bit.  cen / J(p) enter as scalar
-// broadcast operands, (lx, lx) as a uniform-register pair.
+// broadcast operands, (lx, lx) as a broadcast pair.
 template <int R, int PAD>
-__device__ __forceinline__ void pair_tap2(int dx, const float2 *v, const float *u, const float cen[4],
-                                          const float2 *lx2, float2 rd[4], float2 rp[4],
-                                          float2 qd[4], float2 qp[4])
+__device__ __forceinline__ void pair_row2(const float2 *v, const float cen[4], const float *lx,
+                                          float2 rd[4], float2 rp[4], float2 qd[4], float2 qp[4])
 {
-    float2 w[4];
+    float2 od[2 * R + 4], op[2 * R + 4];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-        const float2 jq = v[PAD + j + dx];
-        const float2 diff = __fadd2_rn(jq, make_float2(-cen[j], -cen[j]));
-        const float2 e = __ffma2_rn(make_float2(-diff.x, -diff.y), diff, lx2[dx + R]);
-        w[j] = make_float2(ex2_approx(e.x), ex2_approx(e.y));
-        if (dx == -R) { rd[j] = w[j]; rp[j] = __fmul2_rn(w[j], jq); }
-        else { rd[j] = __fadd2_rn(rd[j], w[j]); rp[j] = __ffma2_rn(w[j], jq, rp[j]); }
-    }
+    for (int dx = -R; dx <= R; ++dx) {
+        float2 w[4];
 #pragma unroll
-    for (int jr = 0; jr < 4; ++jr) {
-        const int t = jr - dx;
-        const int o = t >= 0 ? t / 4 : -((-t + 3) / 4);     // floor(t / 4)
-        const float2 wr = make_float2(lane_shift(w[t - 4 * o].x, o), lane_shift(w[t - 4 * o].y, o));
-        const float jp = u[PAD + t];
-        if (dx == -R) { qd[jr] = wr; qp[jr] = __fmul2_rn(wr, make_float2(jp, jp)); }
-        else { qd[jr] = __fadd2_rn(qd[jr], wr); qp[jr] = __ffma2_rn(wr, make_float2(jp, jp), qp[jr]); }
+        for (int j = 0; j < 4; ++j) {
+            const float2 jq = v[PAD + j + dx];
+            const float2 diff = __fadd2_rn(jq, make_float2(-cen[j], -cen[j]));
+            const float2 e = __ffma2_rn(make_float2(-diff.x, -diff.y), diff, make_float2(lx[dx + R], lx[dx + R]));
+            w[j] = make_float2(ex2_approx(e.x), ex2_approx(e.y));
+            if (dx == -R) { rd[j] = w[j]; rp[j] = __fmul2_rn(w[j], jq); }
+            else { rd[j] = __fadd2_rn(rd[j], w[j]); rp[j] = __ffma2_rn(w[j], jq, rp[j]); }
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int c = j + dx;
+            const float2 cj = make_float2(cen[j], cen[j]);
+            if (c >= 0 && c <= 3) {
+                if (dx == pair_first_dx(c, -R, R)) { qd[c] = w[j]; qp[c] = __fmul2_rn(w[j], cj); }
+                else { qd[c] = __fadd2_rn(qd[c], w[j]); qp[c] = __ffma2_rn(w[j], cj, qp[c]); }
+            } else {
+                const int first = c - 3 > -R ? c - 3 : -R;
+                if (dx == first) { od[c + R] = w[j]; op[c + R] = __fmul2_rn(w[j], cj); }
+                else { od[c + R] = __fadd2_rn(od[c + R], w[j]); op[c + R] = __ffma2_rn(w[j], cj, op[c + R]); }
+            }
+        }
+#pragma unroll
+        for (int c = -R; c <= R + 3; ++c) {
+            if (c >= 0 && c <= 3) continue;
+            if ((c < R ? c : R) != dx) continue;
+            const int o = pair_floor4(c), jr = c - 4 * o;
+            const float2 a = make_float2(lane_shift(od[c + R].x, -o), lane_shift(od[c + R].y, -o));
+            const float2 bq = make_float2(lane_shift(op[c + R].x, -o), lane_shift(op[c + R].y, -o));
+            if (dx == pair_first_dx(jr, -R, R)) { qd[jr] = a; qp[jr] = bq; }
+            else { qd[jr] = __fadd2_rn(qd[jr], a); qp[jr] = __fadd2_rn(qp[jr], bq); }
+        }
     }
 }
 
@@ -627,9 +695,11 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
     float4 *ring1 = reinterpret_cast<float4 *>(wbase + S::RING2);          // NR x SW
     float4 *stg = reinterpret_cast<float4 *>(wbase + S::RING2 + S::RING1); // SW
     int *cm = reinterpret_cast<int *>(wbase + S::RING2 + S::RING1 + SW);   // SW
-    const float2 *lx2 = reinterpret_cast<const float2 *>(p.lx2);
     const int b = blockIdx.z;
-    const int ox0 = c.roi_x0 + blockIdx.x * S::OW;               // first output column of the warp
+    // lane column groups are anchored to x = 0 mod 4 of the output (not to
+    // the ROI), so that every pixel's summation order -- and result -- is
+    // independent of the iteration space (owner push groups by lane)
+    const int ox0 = (c.roi_x0 & ~3) + blockIdx.x * S::OW;        // first output column of the warp
     const int T = p.pair_rows;
     const int y0 = c.roi_y0 + (blockIdx.y * pair::NW + warp) * T;
     const int roi_y1 = c.roi_y0 + c.roi_h;
@@ -669,7 +739,7 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
         if (kmin <= 0) {                                         // dy = 0: own row (scalar)
             float rd[4], rp[4], qd[4], qp[4];
 #pragma unroll
-            for (int dx = 0; dx <= R; ++dx) pair_tap<R, PAD, true>(dx, u, u, cen, p.lx, p.nk, rd, rp, qd, qp);
+            pair_row1<R, PAD, true>(u, cen, p.lx, p.nk, rd, rp, qd, qp);
             const float cy = p.cy[R];
             fold4(cy, rd, rp, D[0], P[0]);
             fold4(cy, qd, qp, D[0], P[0]);
@@ -689,8 +759,7 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
                 }
             }
             float2 rd[4], rp[4], qd[4], qp[4];
-#pragma unroll
-            for (int dx = -R; dx <= R; ++dx) pair_tap2<R, PAD>(dx, v, u, cen, lx2, rd, rp, qd, qp);
+            pair_row2<R, PAD>(v, cen, p.lx, rd, rp, qd, qp);
             const float cya = p.cy[dy + R], cyb = p.cy[dy + 1 + R];
             float ta[4], tb[4], sa[4], sb[4];
 #pragma unroll
@@ -711,8 +780,7 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
             float v[4 * NV];
             load_row<NV>(ring1 + sl * SW4 + lane, v);
             float rd[4], rp[4], qd[4], qp[4];
-#pragma unroll
-            for (int dx = -R; dx <= R; ++dx) pair_tap<R, PAD, false>(dx, v, u, cen, p.lx, p.nk, rd, rp, qd, qp);
+            pair_row1<R, PAD, false>(v, cen, p.lx, p.nk, rd, rp, qd, qp);
             const float cy = p.cy[2 * R];
             fold4(cy, rd, rp, D[0], P[0]);
             fold4(cy, qd, qp, D[R], P[R]);
@@ -721,7 +789,17 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
             float res[4];
 #pragma unroll
             for (int j = 0; j < 4; ++j) res[j] = bilateral_finish_scaled(D[0][j], P[0][j], p.inv_alpha);
-            if (x_out < c.roi_x0 + c.roi_w) store4(c, b, s, x_out, res);
+            if (x_out < c.roi_x0 + c.roi_w) {
+                if (x_out >= c.roi_x0) {
+                    store4(c, b, s, x_out, res);
+                } else {                                         // group straddling the ROI start
+                    float *orow = reinterpret_cast<float *>(c.out.data + (int64_t)b * c.out.bstride +
+                                                            (int64_t)s * c.out.stride);
+#pragma unroll
+                    for (int j = 0; j < 4; ++j)
+                        if (x_out + j >= c.roi_x0 && x_out + j < c.roi_x0 + c.roi_w) orow[x_out + j] = res[j];
+                }
+            }
         }
 #pragma unroll
         for (int k = 0; k < R; ++k)
@@ -823,7 +901,7 @@ static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
         resident = std::max(1, sms * per_sm);
     }
     BilateralSep p = p0;
-    const int64_t strips = (p.c.roi_w + S::OW - 1) / S::OW;
+    const int64_t strips = ((p.c.roi_x0 & 3) + p.c.roi_w + S::OW - 1) / S::OW;
     int T = 0;
     if (const char *env = std::getenv("LOP_PAIR_ROWS")) T = std::atoi(env);
     static thread_local int64_t memo_key[3] = {-1, -1, -1};
