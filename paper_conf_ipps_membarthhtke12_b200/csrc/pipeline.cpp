@@ -24,13 +24,15 @@ namespace lop_detail {
 void set_error(const std::string &msg);   // lop_api.cpp
 }
 
-// staging buffers per direction: a ring of 4 decouples the H2D and D2H
-// engines (chunk k+4 may upload while chunk k is still downloading)
-constexpr int kBufs = 4;
+// staging buffers per direction: by default one per chunk of the schedule
+// (HBM is not the constraint: 2 x 64 MiB for a 4096^2 f32 image), so no
+// upload ever waits for a buffer to be released; LOP_PIPELINE_BUFS caps the
+// ring (a ring of >= 2 still decouples the H2D and D2H engines).
+constexpr int kBufs = 64;
 
 struct lop_pipeline {
     int device = 0;
-    int W = 0, H = 0, chunk = 0;
+    int W = 0, H = 0, chunk = 0, nbufs = 0;
     size_t in_bytes = 0, out_bytes = 0;     // per staging buffer
     void *d_in[kBufs] = {};
     void *d_out[kBufs] = {};
@@ -163,20 +165,31 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
     char *hout = static_cast<char *>(host_out);
     const std::vector<int> cuts = chunk_schedule(p->H, p->chunk);
     const int nchunks = (int)cuts.size() - 1;
+    // trace mode: per-chunk timeline (upload start/end, compute end, download end)
+    std::vector<cudaEvent_t> tev;
+    auto tmark = [&](cudaStream_t s) {
+        if (!trace) return;
+        cudaEvent_t ev;
+        cudaEventCreate(&ev);
+        cudaEventRecord(ev, s);
+        tev.push_back(ev);
+    };
     for (int k = 0; k < nchunks; ++k) {
-        const int buf = k % kBufs;
+        const int buf = k % p->nbufs;
         const int y0 = cuts[k], y1 = cuts[k + 1];
         cudaError_t e;
-        if (k >= kBufs) {
+        if (k >= p->nbufs) {
             e = cudaStreamWaitEvent(p->s_h2d, p->comp_done[buf], 0);
             if (e != cudaSuccess) return perr(e, "wait");
         }
         lop_image in_view;
+        tmark(p->s_h2d);
         lop_status st = upload_chunk(p, buf, hin, in_stride, ies, in_dtype, y0, y1, ry, mode, &in_view);
         if (st) return st;
+        tmark(p->s_h2d);
         cudaEventRecord(p->up_done[buf], p->s_h2d);
         cudaStreamWaitEvent(p->s_comp, p->up_done[buf], 0);
-        if (k >= kBufs) cudaStreamWaitEvent(p->s_comp, p->down_done[buf], 0);
+        if (k >= p->nbufs) cudaStreamWaitEvent(p->s_comp, p->down_done[buf], 0);
         lop_image out_view;
         std::memset(&out_view, 0, sizeof out_view);
         out_view.data = p->d_out[buf];
@@ -198,8 +211,10 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
         lop_iteration_space is;
         std::memset(&is, 0, sizeof is);
         is.image = out_view;
+        tmark(p->s_comp);
         st = exec(&is, &acc, p->s_comp);
         if (st) return st;
+        tmark(p->s_comp);
         cudaEventRecord(p->comp_done[buf], p->s_comp);
         cudaStreamWaitEvent(p->s_d2h, p->comp_done[buf], 0);
         e = copy_rows(hout + (int64_t)y0 * out_stride, out_stride, p->d_out[buf],
@@ -207,6 +222,7 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
                       p->s_d2h);
         if (e != cudaSuccess) return perr(e, "pipeline download");
         p->d2h_bytes += (int64_t)(y1 - y0) * p->W * oes;
+        tmark(p->s_d2h);
         cudaEventRecord(p->down_done[buf], p->s_d2h);
     }
     if (trace) {
@@ -217,6 +233,14 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
                                  std::chrono::steady_clock::now() - t_start).count();
         std::fprintf(stderr, "lop_pipeline: %d chunks, enqueue %.3f ms, total %.3f ms\n",
                      nchunks, t_enq, t_all);
+        // per chunk: rows, upload [start, end], compute [start, end], download end (ms from the first mark)
+        for (int k = 0; k < nchunks && (size_t)(5 * k + 4) < tev.size(); ++k) {
+            float t[5];
+            for (int i = 0; i < 5; ++i) cudaEventElapsedTime(&t[i], tev[0], tev[5 * k + i]);
+            std::fprintf(stderr, "  chunk %2d rows %4d  up %.3f-%.3f  comp %.3f-%.3f  down-end %.3f\n", k,
+                         cuts[k + 1] - cuts[k], t[0], t[1], t[2], t[3], t[4]);
+        }
+        for (cudaEvent_t ev : tev) cudaEventDestroy(ev);
     }
     cudaError_t e = cudaStreamSynchronize(p->s_d2h);
     if (e != cudaSuccess) return perr(e, "pipeline sync");
@@ -245,8 +269,10 @@ lop_status lop_pipeline_create(int32_t device, int32_t width, int32_t height, in
     p->chunk = chunk_rows;
     p->in_bytes = (size_t)(chunk_rows + 2 * kMaxHalo) * width * 4;
     p->out_bytes = (size_t)chunk_rows * width * 4;
+    p->nbufs = std::min(kBufs, (int)chunk_schedule(height, chunk_rows).size() - 1);
+    if (const char *env = std::getenv("LOP_PIPELINE_BUFS")) p->nbufs = std::max(2, std::min(kBufs, std::atoi(env)));
     cudaError_t e = cudaSuccess;
-    for (int i = 0; i < kBufs && e == cudaSuccess; ++i) {
+    for (int i = 0; i < p->nbufs && e == cudaSuccess; ++i) {
         e = cudaMalloc(&p->d_in[i], p->in_bytes);
         if (e == cudaSuccess) e = cudaMalloc(&p->d_out[i], p->out_bytes);
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&p->up_done[i], cudaEventDisableTiming);
