@@ -909,12 +909,14 @@ static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
     if (T <= 0 && memo_key[0] == p.c.roi_h && memo_key[1] == strips && memo_key[2] == p.c.batch)
         T = memo_T;
     if (T <= 0) {
-        // every T from 8 to the ROI height: waves of resident CTAs x rows per warp
+        // every T from 1 to the ROI height: waves of resident CTAs x rows per warp
         // (+ warm-up); a partial wave costs a full one (few warps per SM
-        // cannot saturate the SFU)
+        // cannot saturate the SFU).  Small images take small T: the row steps of
+        // a warp are serial (one global row fetch each), so a launch that fits
+        // in one wave is latency-bound by T + R steps (config 1: T = 1).
         double best = 0;
-        const int tmax = std::max(8, p.c.roi_h);
-        for (int t = 8; t <= tmax; ++t) {
+        const int tmax = std::max(1, p.c.roi_h);
+        for (int t = 1; t <= tmax; ++t) {
             const int64_t segs = (p.c.roi_h + t - 1) / t;
             const int64_t ctas = strips * ((segs + pair::NW - 1) / pair::NW) * p.c.batch;
             const double cost = (double)((ctas + resident - 1) / resident) * (t + 0.55 * R);

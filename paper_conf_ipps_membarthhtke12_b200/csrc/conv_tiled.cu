@@ -54,16 +54,26 @@ template <typename T> struct TileShape {
 
 // u8 -> u8 with non-negative coefficients whose sums fit 16 bits: SWAR on two
 // 16-bit lanes per 32-bit register (pixels q and q+2), so every IMAD does two
-// exact integer MACs.  Sources: funnel shift of the staged words + byte mask;
-// outputs: (S + 2^(k-1)) >> k per lane, two lanes packed back with PRMT.
-// Exactness conditions are checked on the host (launch_conv_tiled).
-template <int R, int TS>
+// exact integer MACs.  Exactness conditions are checked on the host
+// (launch_conv_tiled).  MODE bits: SW_SYM -- both factors are palindromes
+// (every Gaussian): taps t and 2R-t are added first (IADD, ALU pipe) and
+// multiplied once (IMAD, FMA pipe), R+1 instead of 2R+1 IMADs per sum;
+// SW_SH8 -- shift 8 (5x5 binomial): the rounded result of each lane is its
+// byte 1, so two PRMTs pack 8 outputs with no shift or mask.
+// Sources: each staged word W splits into E(W) = lanes (b0, b2) and O(W) =
+// lanes (b1, b3) (PRMT with a zero source); the lanes (q, q+2) that straddle
+// two words are one PRMT of two E (or O) words.  All integer arithmetic is
+// exact, so every MODE gives the same bits.
+enum { SW_ON = 1, SW_SYM = 2, SW_SH8 = 4 };
+
+template <int R, int TS, int MODE>
 __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tcol, int srows,
                                              char *orow0, int64_t ostride, int ox0, int roi_x1,
                                              bool ovec)
 {
     constexpr int SWE = TileShape<uint8_t>::SWE;
     constexpr uint32_t M = 0x00FF00FFu;
+    constexpr bool SYM = (MODE & SW_SYM) != 0, SH8 = (MODE & SW_SH8) != 0;
     static_assert(R <= 3, "SWAR sources cover bytes -4..11");
     const uint32_t rnd = p.shift > 0 ? (1u << (p.shift - 1)) * 0x00010001u : 0u;
     uint32_t h[2 * R + 1][4];                     // pairs (0,2) (1,3) (4,6) (5,7)
@@ -74,26 +84,35 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
         const uint2 cv = *reinterpret_cast<const uint2 *>(rp);
         const uint32_t W[4] = {*reinterpret_cast<const uint32_t *>(rp - 4), cv.x, cv.y,
                                *reinterpret_cast<const uint32_t *>(rp + 8)};
+        uint32_t E[4], O[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            E[i] = __byte_perm(W[i], 0u, 0x4240);            // bytes 0, 2 -> lanes
+            O[i] = __byte_perm(W[i], 0u, 0x4341);            // bytes 1, 3 -> lanes
+        }
         uint32_t S[6 + 2 * R];                    // S[q + R] = lanes (q, q+2), q in [-R, 5+R]
 #pragma unroll
         for (int q = -R; q <= 5 + R; ++q) {
             const int wi = (q + 4) >> 2, sh = (q + 4) & 3;
-            // bytes q and q+2 into the two 16-bit lanes: one PRMT with a zero
-            // source when both lie in the same word, else funnel shift + mask
-            if (sh == 0)
-                S[q + R] = __byte_perm(W[wi], 0u, 0x4240);      // bytes 0, 2 -> lanes
-            else if (sh == 1)
-                S[q + R] = __byte_perm(W[wi], 0u, 0x4341);      // bytes 1, 3 -> lanes
-            else
-                S[q + R] = __funnelshift_r(W[wi], W[wi + 1], 8 * sh) & M;
+            if (sh == 0) S[q + R] = E[wi];
+            else if (sh == 1) S[q + R] = O[wi];
+            else if (sh == 2) S[q + R] = __byte_perm(E[wi], E[wi + 1], 0x5412);   // (b2, b4')
+            else S[q + R] = __byte_perm(O[wi], O[wi + 1], 0x5412);                // (b3, b5')
         }
         uint32_t *hk = h[k % (2 * R + 1)];
         constexpr int J[4] = {0, 1, 4, 5};
 #pragma unroll
         for (int jj = 0; jj < 4; ++jj) {
-            uint32_t s = (uint32_t)p.ri[0] * S[J[jj]];
+            uint32_t s;
+            if constexpr (SYM) {
+                s = (uint32_t)p.ri[R] * S[J[jj] + R];
 #pragma unroll
-            for (int t = 1; t <= 2 * R; ++t) s += (uint32_t)p.ri[t] * S[J[jj] + t];
+                for (int t = 0; t < R; ++t) s += (uint32_t)p.ri[t] * (S[J[jj] + t] + S[J[jj] + 2 * R - t]);
+            } else {
+                s = (uint32_t)p.ri[0] * S[J[jj]];
+#pragma unroll
+                for (int t = 1; t <= 2 * R; ++t) s += (uint32_t)p.ri[t] * S[J[jj] + t];
+            }
             hk[jj] = s;
         }
         const int o = k - 2 * R;
@@ -101,13 +120,22 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
         uint32_t q4[4];
 #pragma unroll
         for (int jj = 0; jj < 4; ++jj) {
-            uint32_t s = (uint32_t)p.ci[0] * h[o % (2 * R + 1)][jj] + rnd;   // rounding folded in
+            uint32_t s;
+            if constexpr (SYM) {
+                s = (uint32_t)p.ci[R] * h[(o + R) % (2 * R + 1)][jj] + rnd;    // rounding folded in
 #pragma unroll
-            for (int t = 1; t <= 2 * R; ++t) s += (uint32_t)p.ci[t] * h[(o + t) % (2 * R + 1)][jj];
-            q4[jj] = (s >> p.shift) & M;
+                for (int t = 0; t < R; ++t)
+                    s += (uint32_t)p.ci[t] * (h[(o + t) % (2 * R + 1)][jj] + h[(o + 2 * R - t) % (2 * R + 1)][jj]);
+            } else {
+                s = (uint32_t)p.ci[0] * h[o % (2 * R + 1)][jj] + rnd;
+#pragma unroll
+                for (int t = 1; t <= 2 * R; ++t) s += (uint32_t)p.ci[t] * h[(o + t) % (2 * R + 1)][jj];
+            }
+            q4[jj] = SH8 ? s : (s >> p.shift) & M;
         }
-        const uint32_t lo = __byte_perm(q4[0], q4[1], 0x6240);
-        const uint32_t hi = __byte_perm(q4[2], q4[3], 0x6240);
+        // lo = pixels 0..3 = lanes of q4[0] (0, 2) and q4[1] (1, 3); hi likewise
+        const uint32_t lo = SH8 ? __byte_perm(q4[0], q4[1], 0x7351) : __byte_perm(q4[0], q4[1], 0x6240);
+        const uint32_t hi = SH8 ? __byte_perm(q4[2], q4[3], 0x7351) : __byte_perm(q4[2], q4[3], 0x6240);
         uint8_t *op = reinterpret_cast<uint8_t *>(orow0 + (int64_t)o * ostride) + ox0;
         if (ovec) {
             *reinterpret_cast<uint2 *>(op) = make_uint2(lo, hi);
@@ -156,7 +184,7 @@ __device__ __forceinline__ void conv_stage(const Common &c, const ConvTile &ct, 
 
 
 // Filter one staged tile: each thread streams its PX columns down the tile.
-template <typename T, typename TO, int R, bool SWAR, int TS>
+template <typename T, typename TO, int R, int SWAR, int TS>
 __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &ct, const T *tile)
 {
     constexpr int RX = R, RY = R;
@@ -175,8 +203,8 @@ __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &c
                       (((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) %
                         (sizeof(TO) * PX > 16 ? 16 : sizeof(TO) * PX)) == 0);
     const T *tcol = tile + PADE + threadIdx.x * PX;              // this thread's centre column
-    if constexpr (SWAR) {
-        conv_u8_swar<R, TS>(p, reinterpret_cast<const uint8_t *>(tcol), srows,
+    if constexpr (SWAR != 0) {
+        conv_u8_swar<R, TS, SWAR>(p, reinterpret_cast<const uint8_t *>(tcol), srows,
                         obase + (int64_t)ty0 * c.out.stride, c.out.stride, ox0, roi_x1, ovec);
         return;
     }
@@ -298,7 +326,7 @@ __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &c
 // filtered.  NBUF = 1: one tile per CTA (grid = #tiles), latency hidden by
 // co-resident CTAs.  TS = output rows per tile.  (Configuration space of the
 // paper's §V-D exploration, re-done for sm_100a: tools/tune_conv.py.)
-template <typename T, typename TO, int R, bool SWAR, int TS, int NBUF>
+template <typename T, typename TO, int R, int SWAR, int TS, int NBUF>
 __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_constant__ ConvSep p)
 {
     using S = TileShape<T>;
@@ -397,7 +425,7 @@ bool factor(const ConvGeneric &p, ConvSep &s)
     return 255 * lr * lc + (1ll << 30) < (1ll << 31);
 }
 
-template <typename T, typename TO, int R, bool SWAR, int TS, int NBUF>
+template <typename T, typename TO, int R, int SWAR, int TS, int NBUF>
 cudaError_t launch_cfg(const ConvSep &s, cudaStream_t stream)
 {
     using S = TileShape<T>;
@@ -430,7 +458,7 @@ cudaError_t launch_cfg(const ConvSep &s, cudaStream_t stream)
 // the default.
 constexpr int kDefTS = 8, kDefTSSwar = 16, kDefNBUF = 1;   // tools/tune_conv.py on B200, round 1
 
-template <typename T, typename TO, int R, bool SWAR = false>
+template <typename T, typename TO, int R, int SWAR = 0>
 cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
 {
     int ts = SWAR ? kDefTSSwar : kDefTS, nbuf = kDefNBUF;
@@ -474,12 +502,36 @@ bool swar_ok(const ConvSep &s)
     return lr * lc <= (1ll << s.shift) && 255 * lr * lc + rnd < 65536;
 }
 
+// SWAR variant (conv_u8_swar): palindromic factors with shift 8 (the 5x5
+// binomial) take SW_SYM | SW_SH8; everything else the plain variant.  Measured
+// on B200 (profiles/r01_session4/u8_swar_ab.txt): SYM|SH8 is 3.6 % faster than
+// plain for the 5x5 Gaussian, while SYM alone is 14 % slower than plain for the
+// 3x3 one (the compiler moves the pre-adds onto the FMA pipe as IMAD.IADD).
+// LOP_CONV_SWAR=1 forces the plain variant (A/B, parity).
+int swar_mode(const ConvSep &s)
+{
+    if (const char *env = std::getenv("LOP_CONV_SWAR"))
+        if (std::atoi(env) == 1) return SW_ON;
+    const int n = 2 * s.c.rx;
+    bool sym = true;
+    for (int t = 0; t <= n; ++t) sym = sym && s.ri[t] == s.ri[n - t] && s.ci[t] == s.ci[n - t];
+    return sym && s.shift == 8 ? (SW_ON | SW_SYM | SW_SH8) : SW_ON;
+}
+
+template <int R>
+cudaError_t dispatch_swar_r(const ConvSep &s, cudaStream_t stream)
+{
+    if (swar_mode(s) == (SW_ON | SW_SYM | SW_SH8))
+        return launch_sep<uint8_t, uint8_t, R, SW_ON | SW_SYM | SW_SH8>(s, stream);
+    return launch_sep<uint8_t, uint8_t, R, SW_ON>(s, stream);
+}
+
 cudaError_t dispatch_swar(const ConvSep &s, cudaStream_t stream)
 {
     switch (s.c.rx) {
-    case 1: return launch_sep<uint8_t, uint8_t, 1, true>(s, stream);
-    case 2: return launch_sep<uint8_t, uint8_t, 2, true>(s, stream);
-    case 3: return launch_sep<uint8_t, uint8_t, 3, true>(s, stream);
+    case 1: return dispatch_swar_r<1>(s, stream);
+    case 2: return dispatch_swar_r<2>(s, stream);
+    case 3: return dispatch_swar_r<3>(s, stream);
     default: return cudaErrorNotSupported;
     }
 }
