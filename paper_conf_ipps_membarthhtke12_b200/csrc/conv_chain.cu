@@ -17,6 +17,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
 #include <cstdlib>
 #include <type_traits>
 
@@ -184,8 +185,27 @@ __device__ __forceinline__ void store_row(char *orow, int ox0, int roi_x1, bool 
     }
 }
 
+// One output tile (tx0, ty0) of at most TS rows, ending before row ry1 (the
+// iteration space's end, or a band's); every thread of the CTA takes part
+// (block barriers inside).
+// One output row of PX values at ox, per element, only columns in [x0, x1).
+template <typename TO, int PX, typename A>
+__device__ __forceinline__ void store_row_masked(char *orow, int ox, int x0, int x1, const A *out,
+                                                 int shift)
+{
+    TO *op = reinterpret_cast<TO *>(orow);
+#pragma unroll
+    for (int j = 0; j < PX; ++j) {
+        if (ox + j < x0 || ox + j >= x1) continue;
+        if constexpr (std::is_same<TO, float>::value) op[ox + j] = out[j];
+        else if constexpr (sizeof(TO) == 1) op[ox + j] = (TO)min(max(quantize_shift(out[j], shift), 0), 255);
+        else op[ox + j] = quantize_shift(out[j], shift);
+    }
+}
+
 template <typename T, typename TO, int R1, int R2, int TS>
-__global__ void __launch_bounds__(chain::NT) conv_chain_kernel(const __grid_constant__ ConvChain p)
+__device__ __forceinline__ void chain_tile(const ConvChain &p, int b, int tx0, int ty0, int ry1,
+                                           unsigned char *smem_raw, uint64_t &bar)
 {
     using S = chain::Shape<T>;
     constexpr int PX = S::PX, GW = S::GW, HALO = S::HALO, OW = S::OW, IPAD = S::IPAD,
@@ -195,14 +215,9 @@ __global__ void __launch_bounds__(chain::NT) conv_chain_kernel(const __grid_cons
     using TG = T;                                                   // intermediate type
     static_assert(R1 <= IPAD && R2 <= 4 && R2 <= HALO, "halo");
     const Common &c = p.s1.c;
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ __align__(8) uint64_t bar;
     T *itile = reinterpret_cast<T *>(smem_raw);                     // ni x ISW
-    const int b = blockIdx.z;
-    const int tx0 = c.roi_x0 + blockIdx.x * OW;
-    const int ty0 = c.roi_y0 + blockIdx.y * TS;
-    const int roi_x1 = c.roi_x0 + c.roi_w, roi_y1 = c.roi_y0 + c.roi_h;
-    const int nrows = min(TS, roi_y1 - ty0);
+    const int roi_x1 = c.roi_x0 + c.roi_w;
+    const int nrows = min(TS, ry1 - ty0);
     const int ng = nrows + 2 * R2, ni = ng + 2 * R1;
     TG *gtile = reinterpret_cast<TG *>(smem_raw + (size_t)(TS + 2 * R1 + 2 * R2) * ISW * sizeof(T));
     const int gx0 = tx0 + c.off_x - HALO;                           // input col of G col 0
@@ -327,6 +342,348 @@ __global__ void __launch_bounds__(chain::NT) conv_chain_kernel(const __grid_cons
     }
 }
 
+template <typename T, typename TO, int R1, int R2, int TS>
+__global__ void __launch_bounds__(chain::NT) conv_chain_kernel(const __grid_constant__ ConvChain p)
+{
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ __align__(8) uint64_t bar;
+    const Common &c = p.s1.c;
+    chain_tile<T, TO, R1, R2, TS>(p, blockIdx.z, c.roi_x0 + blockIdx.x * chain::Shape<T>::OW,
+                                  c.roi_y0 + blockIdx.y * TS, c.roi_y0 + c.roi_h, smem_raw, bar);
+}
+
+// ------------------------------------------------ row-streaming fused chain
+// Each warp owns a frame of 32 lanes x PX G columns (lane L: G columns
+// gxb + PX L .. + PX-1) and streams down T output rows; the outer lane on each
+// side is halo (its G values feed its neighbour's pass 2; its own outputs are
+// not stored), so a warp writes OWS = 30 PX columns.  Per input row:
+//   cp.async of the row PD rows ahead into a per-warp smem ring (16-B chunks;
+//   chunks outside the image: REPEAT fetches the wrapped chunk, the other
+//   modes fill from the row itself / the constant once the row has landed),
+//   pass-1 horizontal sums into a register ring, pass-1 vertical -> one G row
+//   (kept in registers, quantised like a u8 pass), G columns outside the image
+//   per pass 2's boundary condition (edge frames: constant, or the G value at
+//   the mapped column fetched by shuffle; REPEAT: the naive G there already
+//   equals G at the wrapped column), the G neighbours of the pass-2 window by
+//   shuffles, pass-2 horizontal sums into a second register ring, pass-2
+//   vertical -> one output row.  No block barrier, no G tile, no HBM round
+//   trip of G.  The arithmetic (sep_h / sep_v, the same operations in the same
+//   order) is that of two conv_sep_kernel passes, so the result is bit-identical
+//   to two lop_convolve_execute calls.  The output rows whose pass 2 reads G
+//   rows outside the image (the top and bottom R2 rows) are tiles of chain_tile
+//   in the same launch.
+namespace chain {
+template <typename T> struct SShape {
+    static constexpr int PX = sizeof(T) == 4 ? 4 : 8;          // G columns per lane
+    static constexpr int FW = 32 * PX;                         // frame width (G columns)
+    static constexpr int OWS = FW - 2 * PX;                    // output columns per warp
+    static constexpr int PAD = PX;                             // input columns beyond the frame
+    static constexpr int SW = FW + 2 * PAD;                    // smem ring row (elements)
+    static constexpr int V16 = 16 / (int)sizeof(T);            // elements per 16-B chunk
+    static constexpr int NCH = SW / V16;                       // chunks per row
+    static constexpr int PD = 6;                               // prefetch distance (rows)
+    static constexpr int NS = PD + 1;                          // ring slots
+    static constexpr int RING_BYTES = NS * SW * (int)sizeof(T);
+    static constexpr int WARP_BYTES = RING_BYTES + SW * 4;     // + column map
+};
+constexpr int NW = NT / 32;          // warps per CTA
+constexpr int TSB = 2;               // rows per band tile
+}  // namespace chain
+
+__device__ __forceinline__ void chain_cp_async16(void *smem_dst, const void *gsrc)
+{
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_addr(smem_dst)), "l"(gsrc)
+                 : "memory");
+}
+
+// G[e] of lane m / PX for a warp-uniform frame column m (clamped into the frame).
+template <typename A, int PX>
+__device__ __forceinline__ A chain_frame_value(const A (&G)[PX], int m)
+{
+    m = min(max(m, 0), 32 * PX - 1);
+    const int e = m % PX;
+    A x = G[0];
+#pragma unroll
+    for (int j = 1; j < PX; ++j) x = e == j ? G[j] : x;
+    return __shfl_sync(0xffffffffu, x, m / PX);
+}
+
+// Rare paths of the streaming loop, out of line so that the unrolled loop body
+// stays small (I-cache): the row index of an input row outside the image, and
+// the fill of a landed ring row (CONSTANT rows; out-of-image columns of edge
+// frames from the row itself or the constant).
+__device__ __noinline__ bool chain_row_outside(int iy, const Geom &g, int mode, int &row)
+{
+    return resolve_row(iy, g, mode, row);
+}
+
+template <typename T>
+__device__ __noinline__ void chain_fill_row(T *row, int lane, int ix0, int IW, const int *cm,
+                                            bool row_ok, T cval)
+{
+    constexpr int SW = chain::SShape<T>::SW;
+    for (int e = lane; e < SW; e += 32) {
+        if (!row_ok) { row[e] = cval; continue; }
+        if ((unsigned)(ix0 + e) < (unsigned)IW) continue;
+        row[e] = cm[e] >= 0 ? row[cm[e] - ix0] : cval;
+    }
+}
+
+// Per-warp geometry of the streaming path.
+struct ChainWarp {
+    int y0, nsteps;          // first output row, input rows streamed (T + 2 (R1 + R2))
+    int ix0, gxb, iy0;       // input column of smem column 0 / of lane 0's G column 0; input row of step 0
+    int ox;                  // this lane's first output column
+    bool col_edge, rows_inside;
+};
+
+// The streaming loop.  SIMPLE: every input row inside the image and no frame
+// column outside it (all but the edge warps) -- no row resolution, no fills,
+// no G boundary, one running source pointer.
+template <typename T, typename TO, int R1, int R2, bool SIMPLE>
+__device__ __forceinline__ void chain_stream_run(const ConvChain &p, int b, const ChainWarp &cw,
+                                                 unsigned char *wsmem)
+{
+    using S = chain::SShape<T>;
+    constexpr int PX = S::PX, PAD = S::PAD, SW = S::SW, V16 = S::V16, NCH = S::NCH,
+                  PD = S::PD, NS = S::NS;
+    constexpr bool F = sizeof(T) == 4;
+    using A = typename std::conditional<F, float, int>::type;
+    constexpr int P1 = 2 * R1 + 1, P2 = 2 * R2 + 1;
+    const Common &c = p.s1.c;
+    const Geom &g = c.in;
+    const int lane = threadIdx.x & 31;
+    const int IW = g.W, mode = c.mode, nsteps = cw.nsteps, ix0 = cw.ix0, iy0 = cw.iy0;
+    T *ring = reinterpret_cast<T *>(wsmem);
+    const int *cm = reinterpret_cast<const int *>(wsmem + S::RING_BYTES);
+    const T cval = F ? (T)c.cval_f : (T)c.cval_i;
+    const bool fill_cols = !SIMPLE && cw.col_edge && mode != M_REPEAT;
+    // this lane's chunks (q = lane, lane + 32): source column, or -1 (filled after landing)
+    int src0 = -1, src1 = -1;
+    {
+        const int ixa = ix0 + lane * V16, ixb = ixa + 32 * V16;
+        if (lane >= NCH) {                                        // u8: 17 chunks per row
+        } else if ((unsigned)ixa < (unsigned)IW) src0 = ixa;
+        else if (!SIMPLE && mode == M_REPEAT) src0 = cm[lane * V16];
+        if (NCH > 32 && lane + 32 < NCH) {
+            if ((unsigned)ixb < (unsigned)IW) src1 = ixb;
+            else if (!SIMPLE && mode == M_REPEAT) src1 = cm[(lane + 32) * V16];
+        }
+    }
+    const char *fbase = g.data + (int64_t)b * g.bstride;
+    const T *srow = reinterpret_cast<const T *>(fbase + (int64_t)iy0 * g.stride);   // SIMPLE: row of step k
+    const uint32_t sdst = smem_addr(ring + lane * V16);
+    // input row iy0 + k into ring slot sl (one commit group per call)
+    auto issue = [&](int k, int sl, const T *rp) {
+        if (k < nsteps) {
+            bool ok = true;
+            if (!SIMPLE) {
+                int row = iy0 + k;
+                if ((unsigned)row >= (unsigned)g.H) ok = chain_row_outside(row, g, mode, row);
+                rp = reinterpret_cast<const T *>(fbase + (int64_t)row * g.stride);
+            }
+            if (ok) {
+                const uint32_t d = sdst + sl * (SW * (int)sizeof(T));
+                if (src0 >= 0)
+                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(rp + src0) : "memory");
+                if (NCH > 32 && src1 >= 0)
+                    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d + 32 * 16), "l"(rp + src1)
+                                 : "memory");
+            }
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    const int64_t sstride = g.stride / (int64_t)sizeof(T);
+#pragma unroll
+    for (int k = 0; k < PD; ++k) issue(k, k, srow + k * sstride);
+    const T *pre = srow + PD * sstride;                           // SIMPLE: row of step k + PD
+
+    // frame columns of G at the mapped positions of G columns -1-t and IW+t
+    int gml[R2], gmr[R2];
+#pragma unroll
+    for (int t = 0; t < R2; ++t) {
+        gml[t] = fill_cols ? map_axis(-1 - t, IW, mode) - cw.gxb : 0;
+        gmr[t] = fill_cols ? map_axis(IW + t, IW, mode) - cw.gxb : 0;
+    }
+    char *obase = c.out.data + (int64_t)b * c.out.bstride;
+    const int roi_x0 = c.roi_x0, roi_x1 = c.roi_x0 + c.roi_w;
+    const int ox = cw.ox;
+    const bool out_lane = lane >= 1 && lane <= 30 && ox + PX > roi_x0 && ox < roi_x1;
+    const bool ovec = out_lane && ox >= roi_x0 && ox + PX <= roi_x1 &&
+                      (((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) %
+                        (sizeof(TO) * PX > 16 ? 16 : sizeof(TO) * PX)) == 0);
+    const T *lrow = ring + PAD + lane * PX;                      // gather base in slot 0
+    char *orow = obase + (int64_t)cw.y0 * c.out.stride;          // output row of the next output
+    A h1[P1][PX], h2[P2][PX];
+    int slot = 0, islot = PD;                                    // slot of row k, of row k + PD
+    // Register rings of P1 (pass 1) and P2 (pass 2) rows with compile-time slot
+    // indices: the SIMPLE loop is unrolled by the common period of both; the
+    // general loop (edge warps, larger code) by P1 only, with pass 2 as a
+    // shift register (h2[P2-1] newest) so that its body stays short (I-cache).
+    constexpr int UNR = SIMPLE ? (P1 == P2 ? P1 : P1 * P2) : P1;
+    constexpr bool H2RING = UNR % P2 == 0;
+#pragma unroll 1
+    for (int k0 = 0; k0 < nsteps; k0 += UNR) {
+#pragma unroll
+        for (int i = 0; i < UNR; ++i) {
+            const int k = k0 + i;
+            if (k >= nsteps) break;
+            // row k has landed once at most PD - 1 younger groups are pending;
+            // after the barrier every lane is also done with slot k - 1,
+            // which takes row k + PD
+            asm volatile("cp.async.wait_group %0;" ::"n"(PD - 1) : "memory");
+            __syncwarp();
+            issue(k + PD, islot, pre);
+            pre += sstride;
+            islot = islot + 1 == NS ? 0 : islot + 1;
+            if (!SIMPLE) {
+                int r;
+                const int iy = iy0 + k;
+                const bool rok = (unsigned)iy < (unsigned)g.H || chain_row_outside(iy, g, mode, r);
+                if (fill_cols || !rok) {
+                    chain_fill_row<T>(ring + slot * SW, lane, ix0, IW, cm, rok, cval);
+                    __syncwarp();
+                }
+            }
+            // ---- pass 1, horizontal
+            {
+                A v[PX + 2 * R1];
+                chain_gather<T, R1, A>(lrow + slot * SW, v);
+#pragma unroll
+                for (int j = 0; j < PX; ++j) h1[i % P1][j] = sep_h<A, R1>(p.s1, v + j);
+            }
+            slot = slot + 1 == NS ? 0 : slot + 1;
+            if (k < 2 * R1) continue;
+            // ---- pass 1, vertical: G row k - 2 R1 (quantised like a u8 pass)
+            A G[PX];
+#pragma unroll
+            for (int j = 0; j < PX; ++j) {
+                A col[P1];
+#pragma unroll
+                for (int t = 0; t < P1; ++t) col[t] = h1[(i + 1 + t) % P1][j];
+                G[j] = (A)to_g<A, T>(sep_v<A, R1>(p.s1, col), p.s1.shift);
+            }
+            if (fill_cols) {                                         // pass 2's boundary on G
+                const int gx = cw.gxb + PX * lane;
+                if (mode == M_CONSTANT) {
+#pragma unroll
+                    for (int j = 0; j < PX; ++j)
+                        if ((unsigned)(gx + j) >= (unsigned)IW) G[j] = (A)cval;
+                } else {
+                    A lv[R2], rv[R2];
+#pragma unroll
+                    for (int t = 0; t < R2; ++t) {
+                        lv[t] = chain_frame_value<A, PX>(G, gml[t]);
+                        rv[t] = chain_frame_value<A, PX>(G, gmr[t]);
+                    }
+#pragma unroll
+                    for (int j = 0; j < PX; ++j)
+#pragma unroll
+                        for (int t = 0; t < R2; ++t) {
+                            if (gx + j == -1 - t) G[j] = lv[t];
+                            if (gx + j == IW + t) G[j] = rv[t];
+                        }
+                }
+            }
+            // ---- pass 2, horizontal: the R2 G columns of each neighbour lane by shuffles
+            const int i2 = H2RING ? (((i - 2 * R1) % P2) + P2) % P2 : P2 - 1;   // slot of this G row
+            if (!H2RING) {
+#pragma unroll
+                for (int t = 0; t + 1 < P2; ++t)
+#pragma unroll
+                    for (int j = 0; j < PX; ++j) h2[t][j] = h2[t + 1][j];
+            }
+            {
+                A v2[PX + 2 * R2];
+#pragma unroll
+                for (int j = 0; j < PX; ++j) v2[R2 + j] = G[j];
+#pragma unroll
+                for (int t = 0; t < R2; ++t) {
+                    v2[t] = __shfl_up_sync(0xffffffffu, G[PX - R2 + t], 1);
+                    v2[R2 + PX + t] = __shfl_down_sync(0xffffffffu, G[t], 1);
+                }
+#pragma unroll
+                for (int j = 0; j < PX; ++j) h2[i2][j] = sep_h<A, R2>(p.s2, v2 + j);
+            }
+            if (k < 2 * (R1 + R2)) continue;
+            // ---- pass 2, vertical: output row
+            A out[PX];
+#pragma unroll
+            for (int j = 0; j < PX; ++j) {
+                A col[P2];
+#pragma unroll
+                for (int t = 0; t < P2; ++t) col[t] = h2[H2RING ? (i2 + 1 + t) % P2 : t][j];   // rows o .. o + 2 R2
+                out[j] = sep_v<A, R2>(p.s2, col);
+            }
+            if (ovec) store_row<TO, PX>(orow, ox, roi_x1, true, out, p.s2.shift);
+            else if (!SIMPLE && out_lane) store_row_masked<TO, PX>(orow, ox, roi_x0, roi_x1, out, p.s2.shift);
+            orow += c.out.stride;
+        }
+    }
+    asm volatile("cp.async.wait_all;" ::: "memory");
+}
+
+template <typename T, typename TO, int R1, int R2>
+__device__ __forceinline__ void chain_stream_warp(const ConvChain &p, int b, int w,
+                                                  unsigned char *wsmem)
+{
+    using S = chain::SShape<T>;
+    const Common &c = p.s1.c;
+    const ChainPlan &pl = p.plan;
+    const Geom &g = c.in;
+    const int lane = threadIdx.x & 31;
+    const int f = w % pl.nframes, seg = w / pl.nframes;
+    ChainWarp cw;
+    cw.y0 = pl.sy0 + seg * pl.T;
+    if (seg >= pl.nseg || cw.y0 >= pl.sy1) return;               // warp-uniform
+    const int y1 = min(cw.y0 + pl.T, pl.sy1);
+    const int ox0 = pl.ox_base + f * S::OWS;       // output column of lane 1, element 0
+    cw.gxb = ox0 + c.off_x - S::PX;                // input column of lane 0's first G column
+    cw.ix0 = cw.gxb - S::PAD;                      // input column of smem column 0
+    cw.ox = ox0 + S::PX * (lane - 1);
+    cw.iy0 = cw.y0 + c.off_y - R2 - R1;
+    cw.nsteps = (y1 - cw.y0) + 2 * (R1 + R2);
+    cw.col_edge = cw.ix0 < 0 || cw.ix0 + S::SW > g.W;
+    cw.rows_inside = cw.iy0 >= 0 && cw.iy0 + cw.nsteps <= g.H;
+    // output columns partly outside the iteration space also take the general path
+    const bool roi_inner = ox0 >= c.roi_x0 && ox0 + S::OWS <= c.roi_x0 + c.roi_w;
+    if (cw.col_edge) {
+        int *cm = reinterpret_cast<int *>(wsmem + S::RING_BYTES);
+        for (int i = lane; i < S::SW; i += 32) {
+            int col;
+            cm[i] = resolve_col(cw.ix0 + i, g, c.mode, col) ? col : -1;
+        }
+        __syncwarp();
+    }
+    if (!cw.col_edge && cw.rows_inside && roi_inner)
+        chain_stream_run<T, TO, R1, R2, true>(p, b, cw, wsmem);
+    else
+        chain_stream_run<T, TO, R1, R2, false>(p, b, cw, wsmem);
+}
+
+template <typename T, typename TO, int R1, int R2>
+__global__ void __launch_bounds__(chain::NT) conv_chain_stream_kernel(const __grid_constant__ ConvChain p)
+{
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ __align__(8) uint64_t bar;
+    const ChainPlan &pl = p.plan;
+    const int b = blockIdx.z;
+    if ((int)blockIdx.x < pl.stream_ctas) {                      // block-uniform
+        const int warp = threadIdx.x >> 5;
+        chain_stream_warp<T, TO, R1, R2>(p, b, blockIdx.x * chain::NW + warp,
+                                         smem_raw + warp * chain::SShape<T>::WARP_BYTES);
+        return;
+    }
+    const Common &c = p.s1.c;
+    const int t = blockIdx.x - pl.stream_ctas;
+    const int ty = t / pl.ntx, tx = t - ty * pl.ntx;
+    const int tx0 = c.roi_x0 + tx * chain::Shape<T>::OW;
+    int ty0, ry1;
+    if (ty < pl.top_rows) { ty0 = c.roi_y0 + ty * chain::TSB; ry1 = pl.sy0; }
+    else { ty0 = pl.sy1 + (ty - pl.top_rows) * chain::TSB; ry1 = c.roi_y0 + c.roi_h; }
+    chain_tile<T, TO, R1, R2, chain::TSB>(p, b, tx0, ty0, ry1, smem_raw, bar);
+}
+
 namespace {
 
 template <typename T, typename TO, int R1, int R2, int TS>
@@ -361,14 +718,95 @@ cudaError_t launch_chain_rr(const ConvChain &p, cudaStream_t stream)
     }
 }
 
+// Row-streaming launch (conv_chain_stream_kernel) when the geometry allows it:
+// 16-B aligned input rows, chunk-aligned frames (W and off_x multiples of 16 B),
+// outputs that read the image through their own column (roi + off_x inside the
+// image, so every G column outside it is within R2 of an edge), images at least
+// two frames wide and enough streamed rows.  Rows per warp T from the wave
+// model of the pair kernel: cost(T) = waves(T) x (T + warm-up rows).
+// T >= 16 (measured best).  Returns false when not selected or not eligible.
+template <typename T, typename TO, int R1, int R2>
+bool launch_chain_stream(const ConvChain &p0, cudaStream_t stream, cudaError_t &err)
+{
+    using S = chain::SShape<T>;
+    // opt-in (LOP_CHAIN_STREAM=1): measured slower than the tile kernel on B200
+    // (DESIGN.md §6 conv_chain, profiles/r01_session4/chain_stream.txt)
+    const char *env = std::getenv("LOP_CHAIN_STREAM");
+    if (!env || std::atoi(env) == 0) return false;
+    const Common &c = p0.s1.c;
+    const Geom &g = c.in;
+    constexpr int V16 = S::V16;
+    if (((reinterpret_cast<uintptr_t>(g.data) | (uintptr_t)g.stride | (uintptr_t)g.bstride) & 15) ||
+        g.W % V16 || ((c.off_x % V16) + V16) % V16 || g.W < 2 * S::FW)
+        return false;
+    if (c.roi_x0 + c.off_x < 0 || c.roi_x0 + c.roi_w - 1 + c.off_x > g.W - 1) return false;
+    const int sy0 = std::max(c.roi_y0, R2 - c.off_y);
+    const int sy1 = std::min(c.roi_y0 + c.roi_h, g.GH - R2 - c.off_y);
+    if (sy1 - sy0 < 16) return false;
+    static int resident = 0;
+    constexpr size_t smem_stream = (size_t)chain::NW * S::WARP_BYTES;
+    using TS = chain::Shape<T>;
+    constexpr size_t smem_tile = (size_t)(chain::TSB + 2 * R1 + 2 * R2) * TS::ISW * sizeof(T) +
+                                 (size_t)(chain::TSB + 2 * R2) * TS::GW * sizeof(T);
+    constexpr size_t smem = smem_stream > smem_tile ? smem_stream : smem_tile;
+    auto kern = conv_chain_stream_kernel<T, TO, R1, R2>;
+    if (!resident) {
+        int dev = 0, sms = 0, per_sm = 0;
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e == cudaSuccess) e = cudaGetDevice(&dev);
+        if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, chain::NT, smem);
+        if (e != cudaSuccess) { err = e; return true; }
+        resident = std::max(1, sms * per_sm);
+    }
+    ConvChain p = p0;
+    ChainPlan &pl = p.plan;
+    pl.sy0 = sy0;
+    pl.sy1 = sy1;
+    pl.ox_base = c.roi_x0 & ~(V16 - 1);
+    pl.nframes = (c.roi_x0 + c.roi_w - pl.ox_base + S::OWS - 1) / S::OWS;
+    const int rows = sy1 - sy0, warm = 2 * (R1 + R2);
+    int tr = 0;
+    if (const char *env = std::getenv("LOP_CHAIN_ROWS")) tr = std::atoi(env);
+    if (tr <= 0) {
+        double best = 0;
+        for (int t = 16; t <= rows; ++t) {
+            const int64_t segs = (rows + t - 1) / t;
+            const int64_t ctas = (segs * pl.nframes + chain::NW - 1) / chain::NW * c.batch;
+            const double cost = (double)((ctas + resident - 1) / resident) * (t + warm);
+            if (tr == 0 || cost < best) { best = cost; tr = t; }
+            if (segs == 1) break;
+        }
+        if (tr == 0) tr = rows;
+    }
+    pl.T = tr;
+    pl.nseg = (rows + tr - 1) / tr;
+    pl.stream_ctas = (pl.nseg * pl.nframes + chain::NW - 1) / chain::NW;
+    pl.ntx = (c.roi_w + TS::OW - 1) / TS::OW;
+    pl.top_rows = (sy0 - c.roi_y0 + chain::TSB - 1) / chain::TSB;
+    pl.bot_rows = (c.roi_y0 + c.roi_h - sy1 + chain::TSB - 1) / chain::TSB;
+    dim3 grid((unsigned)(pl.stream_ctas + pl.ntx * (pl.top_rows + pl.bot_rows)), 1, c.batch);
+    kern<<<grid, chain::NT, smem, stream>>>(p);
+    err = cudaGetLastError();
+    return true;
+}
+
+template <typename T, typename TO, int R1, int R2>
+cudaError_t launch_chain_any(const ConvChain &p, cudaStream_t stream)
+{
+    cudaError_t e = cudaSuccess;
+    if (launch_chain_stream<T, TO, R1, R2>(p, stream, e)) return e;
+    return launch_chain_rr<T, TO, R1, R2>(p, stream);
+}
+
 template <typename T, typename TO>
 cudaError_t launch_chain_t(const ConvChain &p, cudaStream_t stream)
 {
     const int r1 = p.s1.c.rx, r2 = p.s2.c.rx;
-    if (r1 == 1 && r2 == 1) return launch_chain_rr<T, TO, 1, 1>(p, stream);
-    if (r1 == 1 && r2 == 2) return launch_chain_rr<T, TO, 1, 2>(p, stream);
-    if (r1 == 2 && r2 == 1) return launch_chain_rr<T, TO, 2, 1>(p, stream);
-    if (r1 == 2 && r2 == 2) return launch_chain_rr<T, TO, 2, 2>(p, stream);
+    if (r1 == 1 && r2 == 1) return launch_chain_any<T, TO, 1, 1>(p, stream);
+    if (r1 == 1 && r2 == 2) return launch_chain_any<T, TO, 1, 2>(p, stream);
+    if (r1 == 2 && r2 == 1) return launch_chain_any<T, TO, 2, 1>(p, stream);
+    if (r1 == 2 && r2 == 2) return launch_chain_any<T, TO, 2, 2>(p, stream);
     return cudaErrorNotSupported;
 }
 

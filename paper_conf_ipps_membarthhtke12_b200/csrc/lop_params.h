@@ -103,9 +103,22 @@ struct ConvSep {
 // stages with the same boundary condition; the intermediate image never
 // leaves shared memory.  Intermediate of the u8 path is quantised to u8
 // exactly like a lop_convolve_execute u8 -> u8 pass.
+// Row-streaming plan of the fused chain (conv_chain.cu, set by the launcher):
+// warps stream output rows [sy0, sy1) in frames of 32 lanes; the rows above
+// and below (where pass 2 reads G outside the image) are band tiles of the
+// tile kernel in the same launch.
+struct ChainPlan {
+    int32_t sy0, sy1;            // streamed output rows
+    int32_t T, nseg, nframes;    // rows per warp, row segments, frames across
+    int32_t ox_base;             // output column of frame 0, lane 1, element 0
+    int32_t stream_ctas;         // CTAs of streaming warps (per image)
+    int32_t ntx;                 // band tiles across
+    int32_t top_rows, bot_rows;  // band tile rows above / below the streamed rows
+};
 struct ConvChain {
     ConvSep s1, s2;          // s1.c holds the launch geometry
     int32_t kind;            // 0: f32 -> f32 -> f32; 1: u8 -> u8 -> u8; 2: u8 -> u8 -> i32
+    ChainPlan plan;
 };
 
 }  // namespace lop

@@ -298,10 +298,16 @@ def test_conv_tile_configs(lop, cfg, monkeypatch):
 
 @pytest.mark.parametrize("rows,cols,shift",[([1, 2, 1], [1, 1, 1], 4), ([3, 0, 2, 1, 1], [1, 4, 6, 4, 1], 8),
                                              ([1, 1, 1, 1, 1, 1, 1], [2, 1, 0, 1, 2, 1, 1], 6),
-                                             ([0, 1, 0], [0, 0, 1], 0)])
+                                             ([0, 1, 0], [0, 0, 1], 0),
+                                             # palindromic factors (SW_SYM), shift 8 (SW_SH8)
+                                             ([2, 4, 2], [4, 8, 4], 8),
+                                             ([1, 1, 1, 2, 1, 1, 1], [1, 2, 3, 4, 3, 2, 1], 8),
+                                             ([1, 2, 2, 2, 1], [1, 1, 1, 1, 1], 6),
+                                             ([1, 4, 6, 4, 1], [1, 4, 6, 4, 1], 9)])
 def test_conv_u8_swar_masks(lop, conv_variant, rows, cols, shift):
     """Non-negative separable u8 masks that fit 16-bit lanes take the SWAR path
-    (two exact MACs per IMAD); bit-exact against the oracle in every mode."""
+    (two exact MACs per IMAD; palindromic factors pre-add mirrored taps, shift 8
+    packs by byte permutes); bit-exact against the oracle in every mode."""
     mi = np.outer(np.array(cols), np.array(rows)).astype(np.int32)
     u8 = synthetic.uniform_u8(77, 301, seed=sum(rows) * 7 + shift)
     for mode in MODES:
@@ -309,6 +315,23 @@ def test_conv_u8_swar_masks(lop, conv_variant, rows, cols, shift):
         refq, valid = oracle.convolve_u8(u8.numpy(), mi, shift, mode, cval=250)
         sel = valid if mode == "undefined" else slice(None)
         assert (q[sel] == refq[sel]).all(), mode
+
+
+@pytest.mark.parametrize("swar", ["1", "auto"])
+@pytest.mark.parametrize("size", [3, 5])
+def test_conv_u8_swar_variants_bit_identical(lop, swar, size, monkeypatch):
+    """The SWAR variants (plain: LOP_CONV_SWAR=1; palindromic / shift-8: auto)
+    give the oracle's bits on multi-tile images with ragged tails and frames."""
+    if swar != "auto":
+        monkeypatch.setenv("LOP_CONV_SWAR", swar)
+    u = torch.stack([synthetic.uniform_u8(203, 2085, seed=s + 40) for s in range(2)])
+    gm, k = oracle.gaussian_mask(size)
+    for mode in MODES:
+        q = lop.gaussian(u.cuda(), size, mode, constant=201).cpu().numpy()
+        for i in range(2):
+            refq, valid = oracle.convolve_u8(u[i].numpy(), gm, k, mode, cval=201)
+            sel = valid if mode == "undefined" else slice(None)
+            assert (q[i][sel] == refq[sel]).all(), (mode, i)
 
 
 @pytest.mark.parametrize("msize", [(3, 5), (7, 1), (1, 9), (11, 11), (15, 3)])
@@ -551,3 +574,53 @@ def test_chain_roi_offset_and_validation(lop):
         lop.convolve_chain(img, np.random.rand(3, 3).astype(np.float32), sx)
     with pytest.raises(lop.LopError):
         lop.convolve_chain(img, np.ones((7, 7), np.float32), sx)
+
+
+@pytest.mark.parametrize("rows", ["auto", "8", "13"])
+@pytest.mark.parametrize("mode", MODES)
+def test_chain_stream_equals_tiles(lop, rows, mode, monkeypatch):
+    """The row-streaming fused chain (warp frames, register rings, G neighbours
+    by shuffle; band tiles for the top/bottom rows) == the tile kernel
+    (LOP_CHAIN_STREAM=0) == two passes, bit for bit: f32 and u8 frames wide
+    enough for the streaming path, ragged last frame and row segment
+    (LOP_CHAIN_ROWS = rows per warp), every mode."""
+    if rows != "auto":
+        monkeypatch.setenv("LOP_CHAIN_ROWS", rows)
+    f = torch.stack([synthetic.uniform(67, 1032, seed=s + 70) for s in range(2)]).cuda()
+    u = torch.stack([synthetic.uniform_u8(67, 1040, seed=s + 80) for s in range(2)]).cuda()
+    for x, pairs, cval in ((f, _chain_pairs("f32"), 0.25), (u, _chain_pairs("u8"), 99)):
+        for m1, k1, m2, k2 in pairs:
+            for odt in ((None,) if x.dtype == torch.float32 else (torch.uint8, torch.int32)):
+                kw = dict(constant=cval, shift1=k1, shift2=k2, out_dtype=odt)
+                monkeypatch.setenv("LOP_CHAIN_STREAM", "1")
+                fused = lop.convolve_chain(x, m1, m2, mode, **kw)
+                monkeypatch.setenv("LOP_CHAIN_STREAM", "0")
+                tiles = lop.convolve_chain(x, m1, m2, mode, **kw)
+                assert torch.equal(fused, tiles), (mode, x.dtype, odt)
+                if mode != "undefined":
+                    mid = lop.convolve(x, m1, mode, constant=cval, shift=k1)
+                    two = lop.convolve(mid, m2, mode, constant=cval, shift=k2, out_dtype=odt)
+                    assert torch.equal(fused, two), (mode, x.dtype, odt)
+    monkeypatch.delenv("LOP_CHAIN_STREAM")
+
+
+@pytest.mark.parametrize("mode", ["clamp", "repeat", "mirror", "constant"])
+@pytest.mark.parametrize("roi,offset", [((16, 5, 400, 50), (-8, 3)), ((20, 9, 700, 41), (8, -2)),
+                                        ((3, 0, 1029, 60), (0, 0))])
+def test_chain_stream_roi_offset(lop, mode, roi, offset, monkeypatch):
+    """Streaming chain with iteration spaces and accessor offsets that keep the
+    streaming path eligible: same bits as the tile kernel inside the ROI, the
+    rest of the output untouched."""
+    for x, m1, m2 in ((synthetic.angio(64, 1032, seed=5).cuda(), *(_chain_pairs("f32")[0][0::2])),):
+        outs = []
+        for st in ("1", "0"):
+            monkeypatch.setenv("LOP_CHAIN_STREAM", st)
+            o = torch.full_like(x, -7.0)
+            lop.convolve_chain(x, m1, m2, mode, constant=0.5, out=o, roi=roi, offset=offset)
+            outs.append(o)
+        assert torch.equal(outs[0], outs[1]), (mode, roi, offset)
+        x0, y0, w, h = roi
+        inside = torch.zeros_like(x, dtype=torch.bool)
+        inside[y0:y0 + h, x0:x0 + w] = True
+        assert bool((outs[0][~inside] == -7.0).all())
+    monkeypatch.delenv("LOP_CHAIN_STREAM")
