@@ -318,6 +318,7 @@ __global__ void __launch_bounds__(tiled::NT, 3) bilateral_tiled_kernel(const __g
         load_row<NV>(rowv + (2 * ry + 1) * (SW / 4), v);
         load_row<MV>(mrow + 2 * ry * MV, m);
         mask_row<RX, S::VOFF, SC>(v, cen1, m, nk, d1, p1);                  // yf = 2ry of r0+1
+        if (x_out >= c.roi_x0 + c.roi_w) continue;   // no division for columns past the ROI
         float res[4];
 #pragma unroll
         for (int j = 0; j < 4; ++j)
@@ -407,6 +408,7 @@ __global__ void __launch_bounds__(tiled::NT, 3) bilateral_sep_kernel(const __gri
         // staged row 2ry+1: last window row of output r0+1
         load_row<NV>(rowv + (2 * ry + 1) * (SW / 4), v);
         sep_row<RX, S::VOFF, NP, SC>(v, cen1, p.lx, nk, scy[2 * ry], d1, p1);
+        if (x_out >= c.roi_x0 + c.roi_w) continue;   // no division for columns past the ROI
         float res[4];
 #pragma unroll
         for (int j = 0; j < 4; ++j)
@@ -602,14 +604,19 @@ __device__ __forceinline__ void cp_async4(void *smem_dst, const void *gsrc)
 
 // Column map of a warp's frame, resolved once per kernel (columns do not
 // change from row to row): cm[i] = input column read for smem column i, or -1
-// where CONSTANT substitutes the constant (Table I).
+// where CONSTANT substitutes the constant (Table I).  Columns no
+// stored output reads (beyond the iteration space's footprint, e.g. the part
+// of the last strip past the image edge) are -1 too: they are not fetched
+// (their value only reaches outputs that are not stored).
 template <int SW>
 __device__ __forceinline__ void pair_colmap(const Common &c, int ix0, int *cm, int lane)
 {
+    const int lo = c.roi_x0 + c.off_x - c.rx, hi = c.roi_x0 + c.roi_w - 1 + c.off_x + c.rx;
 #pragma unroll
     for (int i = lane; i < SW; i += 32) {
         int col;
-        cm[i] = resolve_col(ix0 + i, c.in, c.mode, col) ? col : -1;
+        const int ix = ix0 + i;
+        cm[i] = ix >= lo && ix <= hi && resolve_col(ix, c.in, c.mode, col) ? col : -1;
     }
 }
 
@@ -723,8 +730,9 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
     for (int k = 0; k <= R; ++k)
 #pragma unroll
         for (int j = 0; j < 4; ++j) D[k][j] = P[k][j] = 0.0f;
-    const bool out_lane = lane >= HLN && lane < 32 - HLN;
     const int x_out = ox0 + 4 * (lane - HLN);
+    const bool store_lane = lane >= HLN && lane < 32 - HLN && x_out < c.roi_x0 + c.roi_w &&
+                            x_out + 3 >= c.roi_x0;
     int slot0 = 0;                                               // ring slot of row s
 #pragma unroll 1
     for (int s = y0 - R; s < yend; ++s) {
@@ -785,11 +793,15 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
             fold4(cy, rd, rp, D[0], P[0]);
             fold4(cy, qd, qp, D[R], P[R]);
         }
-        if (s >= y0 && out_lane) {
+        // lanes of the frame outside the iteration space skip the division as well:
+        // an out-of-image pixel under CONSTANT 0 has P = 0 there, which sends
+        // __fdiv_rn to its slow path (the right edge strip then set the kernel's
+        // tail: CONSTANT 0 was 4.4 % slower than the other modes)
+        if (s >= y0 && store_lane) {
             float res[4];
 #pragma unroll
             for (int j = 0; j < 4; ++j) res[j] = bilateral_finish_scaled(D[0][j], P[0][j], p.inv_alpha);
-            if (x_out < c.roi_x0 + c.roi_w) {
+            {
                 if (x_out >= c.roi_x0) {
                     store4(c, b, s, x_out, res);
                 } else {                                         // group straddling the ROI start
