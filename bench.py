@@ -414,7 +414,8 @@ def extras(lop, synthetic, dev, stream, peaks):
 
 
 def conv_extras(lop, synthetic, dev, stream, hbm, img, timed):
-    """Gaussian 5x5 / Sobel 3x3 on 4096^2 f32 and u8 (BASELINE config 3): HBM roofline."""
+    """Gaussian 5x5 / Sobel 3x3 on 4096^2 f32 and u8 (BASELINE config 3), the fused chain and
+    the local MIN / MAX operators: HBM roofline."""
     import numpy as np
     import torch
     sets = 8
@@ -452,6 +453,10 @@ def conv_extras(lop, synthetic, dev, stream, hbm, img, timed):
          lambda k, s: lop.convolve(lop.convolve(u_in[k], gi, "clamp", shift=gk, out=mid_u,
                                                 stream=s), sxi, "clamp", out=i_out[k], stream=s),
          5)]
+    # local MIN / MAX (Listing 9 convolve(mask, MIN/MAX, ...)): erosion / dilation
+    cases += [
+        ("erode5x5_u8", lambda k, s: lop.erode(u_in[k], 5, "clamp", out=u_out[k], stream=s), 2),
+        ("dilate3x3_f32", lambda k, s: lop.dilate(f_in[k], 3, "clamp", out=f_out[k], stream=s), 8)]
     res = {}
     H, W = img.shape
     for name, fn, bpp in cases:

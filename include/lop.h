@@ -171,6 +171,21 @@ lop_status lop_convolve_chain_execute(const lop_iteration_space *is, const lop_a
                                       const lop_mask *first, const lop_mask *second,
                                       void *cuda_stream);
 
+/* Local reduction over a mask domain -- Listing 9's
+ * convolve(mask, <reduction>, f) (L956-L967) with the MIN / MAX reductions
+ * (grey-value erosion / dilation with a structuring element):
+ *   out(x,y) = min (or max) of Read(x+xf, y+yf) over the taps with M(xf,yf) != 0
+ * LOP_REDUCE_SUM is the paper's SUM form and equals lop_convolve_execute
+ * (the mask's values are then the weights).
+ * Images: F32 -> F32 (mask F32) or U8 -> U8 (mask I32); only whether a
+ * coefficient is zero matters for MIN / MAX, and at least one must be non-zero
+ * (LOP_ERR_INVALID otherwise).  Window: odd, up to 63 x 63, equal to the
+ * BoundaryCondition's; boundary modes as for every local operator (Table I).
+ * Exact: every output is an input value or the constant. */
+typedef enum { LOP_REDUCE_SUM = 0, LOP_REDUCE_MIN = 1, LOP_REDUCE_MAX = 2 } lop_reduce_op;
+lop_status lop_reduce_execute(const lop_iteration_space *is, const lop_accessor *in,
+                              const lop_mask *domain, int32_t op, void *cuda_stream);
+
 /* Mask builders (host only).
  * lop_mask_closeness: Eq. (1), float coefficients (Listing 4's mask[]).
  * lop_mask_gaussian:  binomial size x size (size odd; 1..11 for LOP_I32, 1..31

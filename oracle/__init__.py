@@ -78,6 +78,10 @@ def _load():
                                                    i64, i64, vp, vp]
             lib.oracle_convolve_u8_sum_points.argtypes = [vp, i64, i64, i64, vp, i32, i32, i32,
                                                           i64, vp, vp, i64, vp, vp]
+            lib.oracle_reduce_f32.argtypes = [vp, i64, i64, i64, vp, i32, i32, i32, i32, dbl,
+                                              i64, i64, vp, vp]
+            lib.oracle_reduce_u8.argtypes = [vp, i64, i64, i64, vp, i32, i32, i32, i32, i64,
+                                             i64, i64, vp, vp]
             lib.oracle_quantize.argtypes = [i64, i32, i32]
             lib.oracle_quantize.restype = i64
             lib.oracle_bilateral_f32.argtypes = [vp, i64, i64, i64, vp, i32, i32, dbl, dbl,
@@ -201,6 +205,26 @@ def convolve_u8_sum_points(img, mask, mode, xs, ys, cval=0):
                                           _ptr(mask), mask.shape[1], mask.shape[0],
                                           _mode(mode), int(cval), _ptr(xs), _ptr(ys), len(xs),
                                           _ptr(out), _ptr(valid))
+    return out, valid.astype(bool)
+
+
+_REDUCE_OPS = {"min": 1, "max": 2}
+
+
+def reduce(img, domain, op, mode, cval=0.0, rows=None):
+    """Listing 9's convolve(mask, op, ...) with op "min" / "max" over the taps
+    where ``domain`` is non-zero.  float32 image -> (out f64, valid);
+    uint8 image -> (out int64, valid)."""
+    u8 = np.asarray(img).dtype == np.uint8
+    img, stride = _img(img, np.uint8 if u8 else np.float32)
+    dom = np.ascontiguousarray(np.asarray(domain) != 0, np.int32)
+    H, W = img.shape
+    y0, y1 = (0, H) if rows is None else rows
+    out = np.empty((y1 - y0, W), np.int64 if u8 else np.float64)
+    valid = np.empty((y1 - y0, W), np.uint8)
+    fn = _load().oracle_reduce_u8 if u8 else _load().oracle_reduce_f32
+    fn(_ptr(img), W, H, stride, _ptr(dom), dom.shape[1], dom.shape[0], _REDUCE_OPS[op],
+       _mode(mode), int(cval) if u8 else float(cval), y0, y1, _ptr(out), _ptr(valid))
     return out, valid.astype(bool)
 
 

@@ -249,6 +249,77 @@ void oracle_convolve_u8_sum_points(const uint8_t *img, int64_t W, int64_t H, int
         out[i] = conv_px_u8(img, W, H, stride, mask, mw, mh, mode, cval, xs[i], ys[i], &valid[i]);
 }
 
+/* ------------------------------------------------------------------ */
+/* Local reduction over a mask domain: Listing 9's                      */
+/*   output() = convolve(cMask, <reduction>, [&] () { ... })            */
+/* with the MIN / MAX reductions (grey-value       */
+/* erosion / dilation; the SUM form is the convolution above).  The     */
+/* domain is the set of taps whose mask coefficient is non-zero; taps   */
+/* are visited yf outer, xf inner, each read through Read() with the    */
+/* boundary mode.  op: 1 = min, 2 = max.                                */
+/* ------------------------------------------------------------------ */
+static double reduce_px_f32(const float *img, int64_t W, int64_t H, int64_t stride,
+                            const int32_t *dom, int mw, int mh, int op, int mode, double cval,
+                            int64_t x, int64_t y, uint8_t *valid)
+{
+    int m = mw / 2, n = mh / 2, undef = 0, first = 1;
+    double acc = 0.0;
+    for (int yf = -n; yf <= n; ++yf)
+        for (int xf = -m; xf <= m; ++xf) {
+            if (!dom[(yf + n) * mw + (xf + m)])
+                continue;
+            double v = read_f32(img, W, H, stride, x + xf, y + yf, mode, cval, &undef);
+            if (first || (op == 1 ? v < acc : v > acc))
+                acc = v;
+            first = 0;
+        }
+    *valid = (uint8_t)!undef;
+    return acc;
+}
+
+static int64_t reduce_px_u8(const uint8_t *img, int64_t W, int64_t H, int64_t stride,
+                            const int32_t *dom, int mw, int mh, int op, int mode, int64_t cval,
+                            int64_t x, int64_t y, uint8_t *valid)
+{
+    int m = mw / 2, n = mh / 2, undef = 0, first = 1;
+    int64_t acc = 0;
+    for (int yf = -n; yf <= n; ++yf)
+        for (int xf = -m; xf <= m; ++xf) {
+            if (!dom[(yf + n) * mw + (xf + m)])
+                continue;
+            int64_t v = read_u8(img, W, H, stride, x + xf, y + yf, mode, cval, &undef);
+            if (first || (op == 1 ? v < acc : v > acc))
+                acc = v;
+            first = 0;
+        }
+    *valid = (uint8_t)!undef;
+    return acc;
+}
+
+void oracle_reduce_f32(const float *img, int64_t W, int64_t H, int64_t stride,
+                       const int32_t *dom, int mw, int mh, int op, int mode, double cval,
+                       int64_t y0, int64_t y1, double *out, uint8_t *valid)
+{
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t y = y0; y < y1; ++y)
+        for (int64_t x = 0; x < W; ++x) {
+            int64_t o = (y - y0) * W + x;
+            out[o] = reduce_px_f32(img, W, H, stride, dom, mw, mh, op, mode, cval, x, y, &valid[o]);
+        }
+}
+
+void oracle_reduce_u8(const uint8_t *img, int64_t W, int64_t H, int64_t stride,
+                      const int32_t *dom, int mw, int mh, int op, int mode, int64_t cval,
+                      int64_t y0, int64_t y1, int64_t *out, uint8_t *valid)
+{
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t y = y0; y < y1; ++y)
+        for (int64_t x = 0; x < W; ++x) {
+            int64_t o = (y - y0) * W + x;
+            out[o] = reduce_px_u8(img, W, H, stride, dom, mw, mh, op, mode, cval, x, y, &valid[o]);
+        }
+}
+
 /* Output quantisation of the integer sum (reading c12): rounding half-up by
  * (S + 2^(k-1)) >> k (arithmetic shift = floor), then for u8 outputs
  * saturation to [0, 255]; i32 outputs keep the shifted value. */

@@ -185,6 +185,33 @@ def convolve_chain(x: torch.Tensor, first, second, mode="clamp", constant=0.0, s
                         is_, acc, ctypes.byref(m1), ctypes.byref(m2), s))
 
 
+_REDUCE = {"sum": _lib.LOP_REDUCE_SUM, "min": _lib.LOP_REDUCE_MIN, "max": _lib.LOP_REDUCE_MAX}
+
+
+def reduce(x: torch.Tensor, domain, op="min", mode="clamp", constant=0.0, out=None, roi=None,
+           offset=(0, 0), stream=None, band=(0, 0, 0, 0)) -> torch.Tensor:
+    """Local reduction over a mask domain, Listing 9's convolve(mask, <op>, f):
+    op "min" / "max" over the taps where ``domain`` is non-zero (erosion /
+    dilation), "sum" = convolve(x, domain).  float32 or uint8 images."""
+    mdt = _lib.LOP_F32 if x.dtype == torch.float32 else _lib.LOP_I32
+    marr, m = _host_mask(domain, mdt)
+    if out is None:
+        out = torch.empty_like(x)
+    return _execute("reduce", x, out, mode, constant, (m.size_x, m.size_y), roi, offset, stream,
+                    band, lambda is_, acc, s: lib.lop_reduce_execute(is_, acc, ctypes.byref(m),
+                                                                     _REDUCE[op], s))
+
+
+def erode(x: torch.Tensor, size: int = 3, mode="clamp", constant=0.0, **kw) -> torch.Tensor:
+    """Grey-value erosion with a full size x size window (local MIN)."""
+    return reduce(x, np.ones((size, size)), "min", mode, constant, **kw)
+
+
+def dilate(x: torch.Tensor, size: int = 3, mode="clamp", constant=0.0, **kw) -> torch.Tensor:
+    """Grey-value dilation with a full size x size window (local MAX)."""
+    return reduce(x, np.ones((size, size)), "max", mode, constant, **kw)
+
+
 def gaussian(x: torch.Tensor, size: int = 5, mode="clamp", constant=0.0, **kw) -> torch.Tensor:
     """Binomial Gaussian (Tables VIII-IX; reading c11): f32 -> f32, u8 -> u8."""
     if x.dtype == torch.float32:

@@ -16,6 +16,7 @@ LOP_OK, LOP_ERR_INVALID, LOP_ERR_UNSUPPORTED, LOP_ERR_CUDA = 0, -1, -2, -3
 LOP_U8, LOP_I32, LOP_F32 = 0, 1, 2
 LOP_UNDEFINED, LOP_CLAMP, LOP_REPEAT, LOP_MIRROR, LOP_CONSTANT = 0, 1, 2, 3, 4
 LOP_VARIANT_AUTO, LOP_VARIANT_GENERIC, LOP_VARIANT_TILED = 0, 1, 2
+LOP_REDUCE_SUM, LOP_REDUCE_MIN, LOP_REDUCE_MAX = 0, 1, 2
 
 c_i32, c_i64, c_dbl, c_flt, c_vp = (ctypes.c_int32, ctypes.c_int64, ctypes.c_double,
                                     ctypes.c_float, ctypes.c_void_p)
@@ -59,6 +60,9 @@ SIGNATURES = {
     "lop_convolve_chain_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
                                            ctypes.POINTER(lop_accessor), ctypes.POINTER(lop_mask),
                                            ctypes.POINTER(lop_mask), c_vp]),
+    "lop_reduce_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
+                                   ctypes.POINTER(lop_accessor), ctypes.POINTER(lop_mask),
+                                   c_i32, c_vp]),
     "lop_mask_closeness": (c_i32, [c_flt, c_i32, c_i32, c_vp]),
     "lop_mask_gaussian": (c_i32, [c_i32, c_i32, c_vp, ctypes.POINTER(c_i32)]),
     "lop_mask_sobel": (c_i32, [c_i32, c_i32, c_vp]),

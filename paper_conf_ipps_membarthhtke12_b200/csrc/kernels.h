@@ -18,6 +18,9 @@ cudaError_t launch_conv_tiled(const ConvGeneric &p, cudaStream_t stream);
 bool conv_tiled_supported(const ConvGeneric &p);
 // Exact separable factorisation (false if the mask is not rank 1 / too large).
 bool conv_factor(const ConvGeneric &p, ConvSep &s);
+// Local MIN / MAX over a mask domain (reduce.cu): tiled separable kernel for
+// full windows up to 9x9, generic kernel otherwise.
+cudaError_t launch_reduce(const ReduceParams &p, bool allow_tiled, cudaStream_t stream);
 // Fused two-stage convolution; cudaErrorNotSupported if no instance matches.
 cudaError_t launch_conv_chain(const ConvChain &p, cudaStream_t stream);
 

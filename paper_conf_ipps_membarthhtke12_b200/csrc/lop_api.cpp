@@ -453,6 +453,58 @@ lop_status lop_convolve_execute(const lop_iteration_space *is, const lop_accesso
     return launched(lop::launch_conv_generic(p, stream), "conv_generic launch");
 }
 
+// ------------------------------------------------ local MIN / MAX reduction
+lop_status lop_reduce_execute(const lop_iteration_space *is, const lop_accessor *in,
+                              const lop_mask *domain, int32_t op, void *cuda_stream)
+{
+    if (op == LOP_REDUCE_SUM) return lop_convolve_execute(is, in, domain, cuda_stream);
+    if (op != LOP_REDUCE_MIN && op != LOP_REDUCE_MAX)
+        return fail(LOP_ERR_INVALID, "unknown reduction %d (SUM, MIN, MAX)", op);
+    Prepared pp;
+    lop_status st = prepare(is, in, pp);
+    if (st) return st;
+    const lop::Common &c = pp.c;
+    if (!domain || !domain->coeffs) return fail(LOP_ERR_INVALID, "domain mask is NULL");
+    const int sx = 2 * c.rx + 1, sy = 2 * c.ry + 1;
+    if (domain->size_x != sx || domain->size_y != sy)
+        return fail(LOP_ERR_INVALID, "domain %d x %d != window %d x %d", domain->size_x,
+                    domain->size_y, sx, sy);
+    const int32_t idt = in->bc->image.dtype, odt = is->image.dtype;
+    static thread_local lop::ReduceParams p;
+    p.c = c;
+    p.op = op == LOP_REDUCE_MIN ? lop::RED_MIN : lop::RED_MAX;
+    if (idt == LOP_F32 && odt == LOP_F32) {
+        if (domain->dtype != LOP_F32) return fail(LOP_ERR_INVALID, "F32 images need an F32 domain mask");
+        p.u8 = 0;
+    } else if (idt == LOP_U8 && odt == LOP_U8) {
+        if (domain->dtype != LOP_I32) return fail(LOP_ERR_INVALID, "U8 images need an I32 domain mask");
+        p.u8 = 1;
+    } else {
+        return fail(LOP_ERR_INVALID, "unsupported dtype combination %d -> %d (F32->F32, U8->U8)",
+                    idt, odt);
+    }
+    int taps = 0;
+    for (int yf = 0; yf < sy; ++yf) {
+        uint64_t bits = 0;
+        for (int xf = 0; xf < sx; ++xf) {
+            const bool on = domain->dtype == LOP_F32
+                                ? static_cast<const float *>(domain->coeffs)[yf * sx + xf] != 0.0f
+                                : static_cast<const int32_t *>(domain->coeffs)[yf * sx + xf] != 0;
+            if (on) { bits |= 1ull << xf; ++taps; }
+        }
+        p.dom[yf] = bits;
+    }
+    if (!taps) return fail(LOP_ERR_INVALID, "domain mask has no non-zero coefficient");
+    p.full = taps == sx * sy;
+    const int32_t variant = g_variant;
+    const bool tiled_ok = p.full && c.rx == c.ry && c.rx >= 1 && c.rx <= 4;
+    if (variant == LOP_VARIANT_TILED && !tiled_ok)
+        return fail(LOP_ERR_UNSUPPORTED, "no tiled reduction instance for this domain");
+    return launched(lop::launch_reduce(p, variant != LOP_VARIANT_GENERIC,
+                                       static_cast<cudaStream_t>(cuda_stream)),
+                    "reduce launch");
+}
+
 // ------------------------------------------------- fused two-stage operator
 namespace {
 // One stage's mask -> exact separable factors (reusing the convolution path).

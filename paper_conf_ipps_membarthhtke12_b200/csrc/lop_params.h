@@ -103,6 +103,18 @@ struct ConvSep {
 // stages with the same boundary condition; the intermediate image never
 // leaves shared memory.  Intermediate of the u8 path is quantised to u8
 // exactly like a lop_convolve_execute u8 -> u8 pass.
+// Local reduction over a mask domain (Listing 9's convolve(mask, <reduction>, f)
+// with the MIN / MAX reductions; reduce.cu): out = min / max of Read(x+xf, y+yf)
+// over the taps where the mask is non-zero.  dom[yf + ry] bit (xf + rx) = tap.
+enum ReduceOp { RED_MIN = 1, RED_MAX = 2 };
+struct ReduceParams {
+    Common c;
+    int32_t op;                      // RED_MIN / RED_MAX
+    int32_t u8;                      // 1: u8 -> u8, 0: f32 -> f32
+    int32_t full;                    // domain is the whole window (separable)
+    uint64_t dom[2 * kMaxRadius + 1];
+};
+
 // Row-streaming plan of the fused chain (conv_chain.cu, set by the launcher):
 // warps stream output rows [sy0, sy1) in frames of 32 lanes; the rows above
 // and below (where pass 2 reads G outside the image) are band tiles of the

@@ -1,0 +1,242 @@
+// reduce.cu -- local MIN / MAX reductions over a mask domain: the
+// convolve(mask, <reduction>, f) form of Listing 9 (the
+// paper writes it with the SUM reduction, which is lop_convolve_execute) with
+// the reductions MIN and MAX -- grey-value erosion / dilation with a
+// structuring element, a local operator in the paper's sense (every output a
+// reduction over a (2m+1)x(2n+1) window, L274-L282) with the same boundary
+// handling (Table I).  Exact for f32 and u8: the result is one of
+// the input values (or the constant), whatever the evaluation order.
+//
+//  * reduce_tiled_kernel<T, OP, R>: full square windows up to 9x9 -- the
+//    domain is a rectangle, so min/max is separable (row reduction, then
+//    column reduction).  Tile staging as the convolution kernels (stage.cuh:
+//    one cp.async.bulk per row, boundary resolved at staging time).  u8: four
+//    pixels per instruction with the byte-SIMD __vminu4 / __vmaxu4 on funnel-
+//    shifted words; f32: FMNMX per pixel.  HBM-bound (2 or 8 bytes per pixel).
+//  * reduce_generic_kernel: any domain up to 63x63 (one bit per tap), one
+//    thread per output pixel, per-tap boundary resolution.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "boundary.cuh"
+#include "kernels.h"
+#include "lop_params.h"
+#include "stage.cuh"
+
+namespace lop {
+
+namespace red {
+constexpr int NT = 128;
+template <typename T> struct Shape {
+    static constexpr int PX = sizeof(T) == 4 ? 4 : 8;        // columns per thread
+    static constexpr int TWE = NT * PX;                      // tile width (elements)
+    static constexpr int PADE = 16 / (int)sizeof(T);         // 16-B pad each side (>= R)
+    static constexpr int SWE = TWE + 2 * PADE;               // smem row pitch
+    static constexpr int TS = sizeof(T) == 4 ? 8 : 16;       // output rows per tile
+};
+}  // namespace red
+
+template <int OP> __device__ __forceinline__ float red_f(float a, float b)
+{
+    return OP == RED_MIN ? fminf(a, b) : fmaxf(a, b);
+}
+template <int OP> __device__ __forceinline__ uint32_t red_u4(uint32_t a, uint32_t b)
+{
+    return OP == RED_MIN ? __vminu4(a, b) : __vmaxu4(a, b);
+}
+
+template <typename T, int OP, int R>
+__global__ void __launch_bounds__(red::NT) reduce_tiled_kernel(const __grid_constant__ ReduceParams p)
+{
+    using S = red::Shape<T>;
+    constexpr int PX = S::PX, SWE = S::SWE, PADE = S::PADE, TS = S::TS, P = 2 * R + 1;
+    static_assert(R >= 1 && R <= 4, "halo must fit the 16-B pad");
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ __align__(8) uint64_t bar;
+    T *tile = reinterpret_cast<T *>(smem_raw);
+    const Common &c = p.c;
+    const int b = blockIdx.z;
+    const int tx0 = c.roi_x0 + blockIdx.x * S::TWE, ty0 = c.roi_y0 + blockIdx.y * TS;
+    const int roi_x1 = c.roi_x0 + c.roi_w;
+    const int nrows = min(TS, c.roi_y0 + c.roi_h - ty0), srows = nrows + 2 * R;
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&bar)));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    stage_rows<T, SWE, red::NT>(c, b, tx0 + c.off_x - PADE, ty0 + c.off_y - R, srows, tile, &bar);
+    __syncthreads();
+    mbar_wait(&bar, 0);
+
+    const int ox0 = tx0 + threadIdx.x * PX;
+    if (ox0 >= roi_x1) return;
+    char *obase = c.out.data + (int64_t)b * c.out.bstride + (int64_t)ty0 * c.out.stride;
+    const bool ovec = (ox0 + PX <= roi_x1) && (ox0 % PX == 0) &&
+                      (((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) %
+                        (sizeof(T) * PX)) == 0);
+    const T *tcol = tile + PADE + threadIdx.x * PX;
+    if constexpr (sizeof(T) == 1) {
+        uint32_t h[P][2];                                        // row reductions, ring
+#pragma unroll
+        for (int k = 0; k < TS + 2 * R; ++k) {
+            if (k >= srows) break;
+            const uint8_t *rp = reinterpret_cast<const uint8_t *>(tcol) + k * SWE;
+            const uint2 cv = *reinterpret_cast<const uint2 *>(rp);
+            const uint32_t W[4] = {*reinterpret_cast<const uint32_t *>(rp - 4), cv.x, cv.y,
+                                   *reinterpret_cast<const uint32_t *>(rp + 8)};
+#pragma unroll
+            for (int w = 0; w < 2; ++w) {                        // output words: bytes 4w .. 4w+3
+                uint32_t m = W[w + 1];
+#pragma unroll
+                for (int s = 1; s <= R; ++s) {
+                    m = red_u4<OP>(m, __funnelshift_rc(W[w + 1], W[w + 2], 8 * s));       // bytes +s (s = 4: W[w+2])
+                    m = red_u4<OP>(m, __funnelshift_rc(W[w], W[w + 1], 32 - 8 * s));      // bytes -s (s = 4: W[w])
+                }
+                h[k % P][w] = m;
+            }
+            const int o = k - 2 * R;
+            if (o < 0) continue;
+            uint32_t q[2];
+#pragma unroll
+            for (int w = 0; w < 2; ++w) {
+                uint32_t m = h[o % P][w];
+#pragma unroll
+                for (int t = 1; t < P; ++t) m = red_u4<OP>(m, h[(o + t) % P][w]);
+                q[w] = m;
+            }
+            uint8_t *op = reinterpret_cast<uint8_t *>(obase + (int64_t)o * c.out.stride) + ox0;
+            if (ovec) {
+                *reinterpret_cast<uint2 *>(op) = make_uint2(q[0], q[1]);
+            } else {
+#pragma unroll
+                for (int j = 0; j < 8; ++j)
+                    if (ox0 + j < roi_x1) op[j] = (uint8_t)(q[j >> 2] >> (8 * (j & 3)));
+            }
+        }
+    } else {
+        float h[P][PX];
+#pragma unroll
+        for (int k = 0; k < TS + 2 * R; ++k) {
+            if (k >= srows) break;
+            const float *rp = reinterpret_cast<const float *>(tcol) + k * SWE;
+            const float4 cv = *reinterpret_cast<const float4 *>(rp);
+            const float4 l = *reinterpret_cast<const float4 *>(rp - 4);
+            const float4 r = *reinterpret_cast<const float4 *>(rp + 4);
+            const float v[12] = {l.x, l.y, l.z, l.w, cv.x, cv.y, cv.z, cv.w, r.x, r.y, r.z, r.w};
+#pragma unroll
+            for (int j = 0; j < PX; ++j) {
+                float m = v[4 + j];
+#pragma unroll
+                for (int s = 1; s <= R; ++s) m = red_f<OP>(red_f<OP>(m, v[4 + j - s]), v[4 + j + s]);
+                h[k % P][j] = m;
+            }
+            const int o = k - 2 * R;
+            if (o < 0) continue;
+            float q[PX];
+#pragma unroll
+            for (int j = 0; j < PX; ++j) {
+                float m = h[o % P][j];
+#pragma unroll
+                for (int t = 1; t < P; ++t) m = red_f<OP>(m, h[(o + t) % P][j]);
+                q[j] = m;
+            }
+            float *op = reinterpret_cast<float *>(obase + (int64_t)o * c.out.stride) + ox0;
+            if (ovec) {
+                *reinterpret_cast<float4 *>(op) = make_float4(q[0], q[1], q[2], q[3]);
+            } else {
+#pragma unroll
+                for (int j = 0; j < PX; ++j)
+                    if (ox0 + j < roi_x1) op[j] = q[j];
+            }
+        }
+    }
+}
+
+template <int OP>
+__global__ void __launch_bounds__(256) reduce_generic_kernel(const __grid_constant__ ReduceParams p)
+{
+    const Common &c = p.c;
+    const int ox = c.roi_x0 + blockIdx.x * blockDim.x + threadIdx.x;
+    const int oy = c.roi_y0 + blockIdx.y * blockDim.y + threadIdx.y;
+    const int b = blockIdx.z;
+    if (ox >= c.roi_x0 + c.roi_w || oy >= c.roi_y0 + c.roi_h) return;
+    const int ix = ox + c.off_x, iy = oy + c.off_y;
+    char *orow = c.out.data + (int64_t)b * c.out.bstride + (int64_t)oy * c.out.stride;
+    float mf = 0.f;
+    uint32_t mi = 0;
+    bool first = true;
+    for (int yf = -c.ry; yf <= c.ry; ++yf) {
+        uint64_t bits = p.dom[yf + c.ry];
+        if (!bits) continue;
+        int row;
+        const bool row_ok = resolve_row(iy + yf, c.in, c.mode, row);
+        while (bits) {
+            const int xf = __ffsll((long long)bits) - 1 - c.rx;
+            bits &= bits - 1;
+            int col;
+            const bool ok = row_ok && resolve_col(ix + xf, c.in, c.mode, col);
+            if (p.u8) {
+                const uint32_t v = ok ? (uint32_t)__ldg(row_ptr<uint8_t>(c.in, b, row) + col)
+                                      : (uint32_t)c.cval_i;
+                mi = first ? v : (OP == RED_MIN ? min(mi, v) : max(mi, v));
+            } else {
+                const float v = ok ? __ldg(row_ptr<float>(c.in, b, row) + col) : c.cval_f;
+                mf = first ? v : red_f<OP>(mf, v);
+            }
+            first = false;
+        }
+    }
+    if (p.u8) reinterpret_cast<uint8_t *>(orow)[ox] = (uint8_t)mi;
+    else reinterpret_cast<float *>(orow)[ox] = mf;
+}
+
+namespace {
+
+template <typename T, int OP, int R>
+cudaError_t launch_tiled_r(const ReduceParams &p, cudaStream_t stream)
+{
+    using S = red::Shape<T>;
+    const size_t smem = (size_t)(S::TS + 2 * R) * S::SWE * sizeof(T);
+    static bool configured = false;
+    if (!configured && smem > 48 * 1024) {
+        cudaError_t e = cudaFuncSetAttribute(reduce_tiled_kernel<T, OP, R>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        configured = true;
+    }
+    dim3 grid((p.c.roi_w + S::TWE - 1) / S::TWE, (p.c.roi_h + S::TS - 1) / S::TS, p.c.batch);
+    reduce_tiled_kernel<T, OP, R><<<grid, red::NT, smem, stream>>>(p);
+    return cudaGetLastError();
+}
+
+template <typename T, int OP>
+cudaError_t launch_tiled_op(const ReduceParams &p, cudaStream_t stream)
+{
+    switch (p.c.rx) {
+    case 1: return launch_tiled_r<T, OP, 1>(p, stream);
+    case 2: return launch_tiled_r<T, OP, 2>(p, stream);
+    case 3: return launch_tiled_r<T, OP, 3>(p, stream);
+    case 4: return launch_tiled_r<T, OP, 4>(p, stream);
+    default: return cudaErrorNotSupported;
+    }
+}
+
+}  // namespace
+
+cudaError_t launch_reduce(const ReduceParams &p, bool allow_tiled, cudaStream_t stream)
+{
+    const bool tiled = allow_tiled && p.full && p.c.rx == p.c.ry && p.c.rx >= 1 && p.c.rx <= 4;
+    if (tiled) {
+        if (p.u8) return p.op == RED_MIN ? launch_tiled_op<uint8_t, RED_MIN>(p, stream)
+                                         : launch_tiled_op<uint8_t, RED_MAX>(p, stream);
+        return p.op == RED_MIN ? launch_tiled_op<float, RED_MIN>(p, stream)
+                               : launch_tiled_op<float, RED_MAX>(p, stream);
+    }
+    dim3 block(32, 8);
+    dim3 grid((p.c.roi_w + 31) / 32, (p.c.roi_h + 7) / 8, p.c.batch);
+    if (p.op == RED_MIN) reduce_generic_kernel<RED_MIN><<<grid, block, 0, stream>>>(p);
+    else reduce_generic_kernel<RED_MAX><<<grid, block, 0, stream>>>(p);
+    return cudaGetLastError();
+}
+
+}  // namespace lop

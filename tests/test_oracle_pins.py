@@ -402,3 +402,72 @@ def test_bilateral_window_larger_than_image():
         c = oracle.closeness_mask(3.0, 13)
         ref = ndi.correlate(img.astype(np.float64), c / c.sum(), mode=SCIPY_MODE[mode])
         np.testing.assert_allclose(out, ref, rtol=0, atol=1e-9)
+
+
+# ------------------------------------------- local MIN / MAX (Listing 9) ----
+
+def _domain(rng, msize, kind):
+    if kind == "full":
+        return np.ones((msize[1], msize[0]), np.int32)
+    d = (rng.random((msize[1], msize[0])) < 0.5).astype(np.int32)   # asymmetric, holes
+    d[rng.integers(0, msize[1]), rng.integers(0, msize[0])] = 7     # at least one tap
+    return d
+
+
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("op", ["min", "max"])
+@pytest.mark.parametrize("shape,msize,kind", [((17, 13), (3, 3), "full"), ((9, 11), (5, 3), "random"),
+                                              ((6, 5), (1, 7), "random"), ((4, 4), (9, 9), "full"),
+                                              ((3, 8), (7, 5), "random"), ((1, 1), (3, 3), "full")])
+def test_reduce_matches_scipy_rank_filters(mode, op, shape, msize, kind):
+    """oracle.reduce (Listing 9 convolve(mask, MIN/MAX, ...)) == scipy.ndimage
+    minimum_filter / maximum_filter with the mask's non-zero taps as footprint,
+    f32 and u8, every defined mode, windows larger than the image, asymmetric
+    domains with holes (a transposed or flipped domain fails)."""
+    rng = _rng(zlib.crc32(repr(("reduce", mode, op, shape, msize, kind)).encode()))
+    dom = _domain(rng, msize, kind)
+    fn = ndi.minimum_filter if op == "min" else ndi.maximum_filter
+    img = rng.random(shape).astype(np.float32)
+    out, valid = oracle.reduce(img, dom, op, mode, 0.4375)
+    ref = fn(img.astype(np.float64), footprint=dom != 0, mode=SCIPY_MODE[mode], cval=0.4375)
+    assert valid.all() and np.array_equal(out, ref)
+    u8 = rng.integers(0, 256, shape).astype(np.uint8)
+    out, valid = oracle.reduce(u8, dom, op, mode, 77)
+    ref = fn(u8.astype(np.int64), footprint=dom != 0, mode=SCIPY_MODE[mode], cval=77)
+    assert valid.all() and np.array_equal(out, ref)
+
+
+@pytest.mark.parametrize("mode", MODES)
+def test_reduce_invariants(mode):
+    """Erosion <= image <= dilation for domains holding the centre; MIN/MAX
+    duality under negation (f32) and 255 - x (u8, constant mapped too); a
+    constant image is a fixed point (constant mode with the same constant)."""
+    rng = _rng(11)
+    img = rng.random((23, 19)).astype(np.float32)
+    dom = _domain(rng, (5, 7), "random")
+    dom[3, 2] = 1                                                     # centre tap
+    lo, _ = oracle.reduce(img, dom, "min", mode, 0.25)
+    hi, _ = oracle.reduce(img, dom, "max", mode, 0.25)
+    if mode != "undefined":
+        assert (lo <= img).all() and (img <= hi).all()
+        neg, _ = oracle.reduce(-img, dom, "min", mode, -0.25)
+        assert np.array_equal(-neg, hi)
+        u8 = rng.integers(0, 256, (23, 19)).astype(np.uint8)
+        a, _ = oracle.reduce(u8, dom, "max", mode, 40)
+        b, _ = oracle.reduce((255 - u8).astype(np.uint8), dom, "min", mode, 215)
+        assert np.array_equal(a, 255 - b)
+    flat = np.full((8, 9), 0.625, np.float32)
+    out, _ = oracle.reduce(flat, dom, "min", mode, 0.625)
+    assert (out == 0.625).all()
+
+
+def test_reduce_undefined_valid_region():
+    rng = _rng(12)
+    img = rng.random((12, 15)).astype(np.float32)
+    dom = np.ones((3, 5), np.int32)
+    out, valid = oracle.reduce(img, dom, "max", "undefined")
+    exp = np.zeros_like(valid)
+    exp[1:-1, 2:-2] = True
+    assert np.array_equal(valid, exp)
+    ref, _ = oracle.reduce(img, dom, "max", "clamp")
+    assert np.array_equal(out[valid], ref[valid])

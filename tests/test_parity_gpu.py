@@ -624,3 +624,81 @@ def test_chain_stream_roi_offset(lop, mode, roi, offset, monkeypatch):
         inside[y0:y0 + h, x0:x0 + w] = True
         assert bool((outs[0][~inside] == -7.0).all())
     monkeypatch.delenv("LOP_CHAIN_STREAM")
+
+
+# ----------------------------------------- local MIN / MAX (Listing 9) ----
+
+def _red_domain(rng, size, kind):
+    sx, sy = size
+    if kind == "full":
+        return np.ones((sy, sx), np.int32)
+    d = (rng.random((sy, sx)) < 0.5).astype(np.int32)
+    d[sy // 2, 0] = 3
+    return d
+
+
+@pytest.mark.parametrize("shape", SHAPES)
+@pytest.mark.parametrize("mode", MODES)
+def test_reduce_small_shapes(lop, conv_variant, shape, mode):
+    """Local MIN / MAX (erosion / dilation) == the oracle bit for bit: full
+    square windows (tiled byte-SIMD / FMNMX kernel) and asymmetric domains with
+    holes (generic kernel), f32 and u8, ragged tails, images smaller than the
+    window."""
+    H, W = shape
+    rng = np.random.default_rng(H * 101 + W)
+    img = synthetic.uniform(H, W, seed=H * 31 + W + 5)
+    u8 = synthetic.uniform_u8(H, W, seed=H * 37 + W + 5)
+    for size, kind in (((3, 3), "full"), ((5, 5), "full"), ((9, 9), "full"), ((5, 3), "random"),
+                       ((7, 7), "random")):
+        dom = _red_domain(rng, size, kind)
+        if conv_variant == "tiled" and kind != "full":
+            continue
+        for op in ("min", "max"):
+            out = lop.reduce(img.cuda(), dom.astype(np.float32), op, mode, constant=0.5).cpu().numpy()
+            ref, valid = oracle.reduce(img.numpy(), dom, op, mode, 0.5)
+            sel = valid if mode == "undefined" else slice(None)
+            assert np.array_equal(out[sel].astype(np.float64), ref[sel]), (size, kind, op)
+            q = lop.reduce(u8.cuda(), dom, op, mode, constant=201).cpu().numpy()
+            refq, valid = oracle.reduce(u8.numpy(), dom, op, mode, 201)
+            sel = valid if mode == "undefined" else slice(None)
+            assert np.array_equal(q[sel].astype(np.int64), refq[sel]), (size, kind, op)
+
+
+@pytest.mark.parametrize("mode", ["clamp", "repeat", "mirror", "constant"])
+def test_reduce_4096_full_bit_exact(lop, mode):
+    """Erosion 5x5 (u8) and dilation 3x3 (f32) at BASELINE config-3 size, every
+    output compared with the oracle."""
+    img = synthetic.angio(4096, 4096, seed=synthetic.config_seed(3), device="cuda")
+    u8 = synthetic.to_u8(img)
+    q = lop.erode(u8, 5, mode, constant=17).cpu().numpy()
+    refq, _ = oracle.reduce(u8.cpu().numpy(), np.ones((5, 5)), "min", mode, 17)
+    assert np.array_equal(q.astype(np.int64), refq)
+    f = lop.dilate(img, 3, mode, constant=0.75).cpu().numpy()
+    ref, _ = oracle.reduce(img.cpu().numpy(), np.ones((3, 3)), "max", mode, 0.75)
+    assert np.array_equal(f.astype(np.float64), ref)
+
+
+def test_reduce_roi_offset_frames_and_validation(lop):
+    frames = torch.stack([synthetic.uniform_u8(70, 1100, seed=s) for s in range(3)]).cuda()
+    full = lop.erode(frames, 5, "mirror")
+    for i in range(3):
+        ref, _ = oracle.reduce(frames[i].cpu().numpy(), np.ones((5, 5)), "min", "mirror")
+        assert np.array_equal(full[i].cpu().numpy().astype(np.int64), ref)
+    out = torch.full_like(frames, 9)
+    lop.reduce(frames, np.ones((5, 5), np.int32), "min", "mirror", out=out, roi=(13, 7, 900, 50))
+    assert torch.equal(out[:, 7:57, 13:913], full[:, 7:57, 13:913])
+    assert bool((out[:, :7] == 9).all()) and bool((out[:, :, 913:] == 9).all())
+    img = synthetic.uniform(40, 300, seed=3).cuda()
+    off = lop.reduce(img, np.ones((3, 3), np.float32), "max", "clamp", offset=(3, -2))
+    ref, _ = oracle.reduce(img.cpu().numpy(), np.ones((3, 3)), "max", "clamp")
+    # offset (3, -2): output (x, y) reads the window around input (x + 3, y - 2)
+    ys, xs = np.mgrid[0:40, 0:300]
+    exp = ref[np.clip(ys - 2, 0, 39), np.clip(xs + 3, 0, 299)]
+    inner = (ys >= 3) & (xs < 300 - 4)
+    assert np.array_equal(off.cpu().numpy()[inner].astype(np.float64), exp[inner])
+    s = lop.reduce(img, np.ones((3, 3), np.float32), "sum", "clamp")
+    assert torch.equal(s, lop.convolve(img, np.ones((3, 3), np.float32), "clamp"))
+    with pytest.raises(lop.LopError, match="no non-zero"):
+        lop.reduce(img, np.zeros((3, 3), np.float32), "min")
+    with pytest.raises(KeyError):
+        lop.reduce(img, np.ones((3, 3), np.float32), "median")
