@@ -147,6 +147,70 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
     }
 }
 
+// f32 separable pass with sm_100 packed FP32 for the vertical half: the ring
+// holds the horizontal sums of two adjacent columns as a register pair, so
+// (o[j], o[j+1]) = c0 (h[o][j], h[o][j+1]) + sum_t c[t] (...) is one FMUL2 /
+// FFMA2 per tap with the coefficient as a broadcast pair.  Each lane performs
+// exactly the scalar operation of its column (same operands, same order,
+// round-to-nearest), so the result is the scalar kernel's bit for bit.
+template <int R, int TS>
+__device__ __forceinline__ void conv_f32_packed(const ConvSep &p, const float *tcol, int srows,
+                                                char *orow0, int64_t ostride, int ox0, int roi_x1,
+                                                bool ovec)
+{
+    constexpr int SWE = TileShape<float>::SWE;
+    constexpr int P = 2 * R + 1;
+    float2 h[P][2];                                                 // (h0,h1), (h2,h3) ring
+#pragma unroll
+    for (int k = 0; k < TS + 2 * R; ++k) {
+        if (k >= srows) break;
+        const float *rp = tcol + k * SWE;
+        float v[4 + 2 * R];
+        const float4 cv = *reinterpret_cast<const float4 *>(rp);
+        v[R + 0] = cv.x; v[R + 1] = cv.y; v[R + 2] = cv.z; v[R + 3] = cv.w;
+        if constexpr (R > 0) {
+            const float4 l = *reinterpret_cast<const float4 *>(rp - 4);
+            const float4 r = *reinterpret_cast<const float4 *>(rp + 4);
+            const float lv[4] = {l.x, l.y, l.z, l.w}, rv[4] = {r.x, r.y, r.z, r.w};
+#pragma unroll
+            for (int j = 0; j < R; ++j) {
+                v[j] = lv[4 - R + j];
+                v[R + 4 + j] = rv[j];
+            }
+        }
+        // horizontal: scalar (packing it would need a register pair per odd shift),
+        // results written straight into the pair registers of the ring
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            float a = __fmul_rn(p.rf[0], v[j]);
+#pragma unroll
+            for (int t = 1; t <= 2 * R; ++t) a = __fmaf_rn(p.rf[t], v[j + t], a);
+            if (j & 1) h[k % P][j >> 1].y = a;
+            else h[k % P][j >> 1].x = a;
+        }
+        const int o = k - 2 * R;
+        if (o < 0) continue;
+        float2 out[2];
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+            float2 a = __fmul2_rn(h[o % P][q], make_float2(p.cf[0], p.cf[0]));
+#pragma unroll
+            for (int t = 1; t <= 2 * R; ++t)
+                a = __ffma2_rn(h[(o + t) % P][q], make_float2(p.cf[t], p.cf[t]), a);
+            out[q] = a;
+        }
+        float *op = reinterpret_cast<float *>(orow0 + (int64_t)o * ostride) + ox0;
+        if (ovec) {
+            *reinterpret_cast<float4 *>(op) = make_float4(out[0].x, out[0].y, out[1].x, out[1].y);
+        } else {
+            const float w[4] = {out[0].x, out[0].y, out[1].x, out[1].y};
+#pragma unroll
+            for (int j = 0; j < 4; ++j)
+                if (ox0 + j < roi_x1) op[j] = w[j];
+        }
+    }
+}
+
 // Tile geometry of tile index `t` (row-major over column tiles, row tiles, frames).
 struct ConvTile {
     int b, tx0, ty0, nrows;
@@ -206,6 +270,11 @@ __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &c
     if constexpr (SWAR != 0) {
         conv_u8_swar<R, TS, SWAR>(p, reinterpret_cast<const uint8_t *>(tcol), srows,
                         obase + (int64_t)ty0 * c.out.stride, c.out.stride, ox0, roi_x1, ovec);
+        return;
+    }
+    if constexpr (F) {
+        conv_f32_packed<R, TS>(p, reinterpret_cast<const float *>(tcol), srows,
+                               obase + (int64_t)ty0 * c.out.stride, c.out.stride, ox0, roi_x1, ovec);
         return;
     }
     A h[2 * RY + 1][PX];                                          // horizontal sums, ring

@@ -42,5 +42,31 @@ band = buf[6:106]
 lop.bilateral(band, 3.0, 0.1, "clamp", band=(6, 6, 40, 300))
 lop.gaussian(band, 5, "repeat", band=(6, 6, 40, 300))
 n += 6
+# session 4: SWAR variants, local MIN / MAX, fused chains (tile and row-streaming)
+for H, W in ((13, 17), (70, 257), (67, 1040)):
+    img = synthetic.uniform(H, W, seed=H + 3 * W).cuda()
+    u8 = synthetic.uniform_u8(H, W, seed=H * 7 + W).cuda()
+    for mode in MODES:
+        for v in ("generic", "tiled"):
+            lop.set_variant(v)
+            lop.erode(u8, 9, mode, constant=5)
+            lop.dilate(img, 3, mode, constant=0.5)
+            if v == "generic":
+                lop.reduce(u8, [[0, 1, 0], [1, 1, 1], [0, 1, 1]], "min", mode)
+            n += 3
+        lop.set_variant("auto")
+        lop.gaussian(u8, 3, mode, constant=9)                      # plain SWAR
+        lop.convolve(u8, np.outer([1, 2, 3, 2, 1], [1, 2, 3, 2, 1]).astype(np.int32), mode,
+                     shift=8)                                         # palindromic shift-8 SWAR
+        gf, _ = lop.gaussian_mask(5, np.float32)
+        gi, gk = lop.gaussian_mask(5, np.int32)
+        for st in ("0", "1"):
+            os.environ["LOP_CHAIN_STREAM"] = st
+            lop.convolve_chain(img, gf, lop.sobel_mask(0, np.float32), mode, constant=0.5)
+            lop.convolve_chain(u8, gi, lop.sobel_mask(1, np.int32), mode, constant=9, shift1=gk,
+                               out_dtype=torch.int32)
+            n += 2
+        os.environ.pop("LOP_CHAIN_STREAM")
+        n += 2
 torch.cuda.synchronize()
 print("sanitize probe: %d calls ok" % n)
