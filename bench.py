@@ -457,6 +457,16 @@ def conv_extras(lop, synthetic, dev, stream, hbm, img, timed):
     cases += [
         ("erode5x5_u8", lambda k, s: lop.erode(u_in[k], 5, "clamp", out=u_out[k], stream=s), 2),
         ("dilate3x3_f32", lambda k, s: lop.dilate(f_in[k], 3, "clamp", out=f_out[k], stream=s), 8)]
+    # two local operators + point-operator epilogue in one pass (N3): Sobel magnitude,
+    # against the two Sobel passes alone (whose outputs a third pass would still combine)
+    cases += [
+        ("sobel_magnitude_l2_f32_fused",
+         lambda k, s: lop.sobel_magnitude(f_in[k], "clamp", out=f_out[k], stream=s), 8),
+        ("sobel_x_and_y_f32_two_passes",
+         lambda k, s: (lop.sobel(f_in[k], 0, "clamp", out=f_out[k], stream=s),
+                       lop.sobel(f_in[k], 1, "clamp", out=mid_f, stream=s)), 8),
+        ("sobel_magnitude_l1_u8_i32_fused",
+         lambda k, s: lop.sobel_magnitude(u_in[k], "clamp", out=i_out[k], stream=s), 5)]
     res = {}
     H, W = img.shape
     for name, fn, bpp in cases:

@@ -186,6 +186,24 @@ typedef enum { LOP_REDUCE_SUM = 0, LOP_REDUCE_MIN = 1, LOP_REDUCE_MAX = 2 } lop_
 lop_status lop_reduce_execute(const lop_iteration_space *is, const lop_accessor *in,
                               const lop_mask *domain, int32_t op, void *cuda_stream);
 
+/* Two local operators on one input combined by a point operator, in one pass
+ * (PAPER.md L107-L122 -- point operators after local ones):
+ *   A = Ma (*) I,  B = Mb (*) I   (correlation, as lop_convolve_execute)
+ *   out = sqrt(A^2 + B^2)  (LOP_COMBINE_L2, F32 only; e.g. the Sobel gradient
+ *         magnitude with Ma = Sobel-x, Mb = Sobel-y, Table IX)
+ *       = |A| + |B|        (LOP_COMBINE_L1)
+ *       = A^2 + B^2        (LOP_COMBINE_SUMSQ)
+ * F32 -> F32 (F32 masks; the epilogue in IEEE f32: A*A, B*B, +, sqrt, each
+ * rounded) or U8 -> I32 (I32 masks, shift 0; exact integers).  Both masks
+ * have the BoundaryCondition's size (odd, up to 31 x 31).  When both are
+ * exactly separable and 3x3 or 5x5, A and B are bit-identical to
+ * lop_convolve_execute's results, so out equals the epilogue applied to two
+ * separate passes, without A and B making a round trip through HBM. */
+typedef enum { LOP_COMBINE_L2 = 0, LOP_COMBINE_L1 = 1, LOP_COMBINE_SUMSQ = 2 } lop_combine;
+lop_status lop_convolve2_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                 const lop_mask *a, const lop_mask *b, int32_t combine,
+                                 void *cuda_stream);
+
 /* Mask builders (host only).
  * lop_mask_closeness: Eq. (1), float coefficients (Listing 4's mask[]).
  * lop_mask_gaussian:  binomial size x size (size odd; 1..11 for LOP_I32, 1..31

@@ -208,6 +208,29 @@ def convolve_u8_sum_points(img, mask, mode, xs, ys, cval=0):
     return out, valid.astype(bool)
 
 
+def convolve2(img, mask_a, mask_b, combine, mode, cval=0.0, rows=None):
+    """Two local operators on one input combined by a point operator
+    (PAPER.md L107-L122): A, B = the oracle convolutions
+    above (exact double / integer sums), then, in double (f32 images) or
+    exact integers (u8 images):  "l2" sqrt(A^2 + B^2), "l1" |A| + |B|,
+    "sumsq" A^2 + B^2.  Returns (out, valid)."""
+    if np.asarray(img).dtype == np.uint8:
+        A, va = convolve_u8_sum(img, mask_a, mode, int(cval), rows)
+        B, vb = convolve_u8_sum(img, mask_b, mode, int(cval), rows)
+    else:
+        A, va = convolve_f32(img, mask_a, mode, cval, rows)
+        B, vb = convolve_f32(img, mask_b, mode, cval, rows)
+    if combine == "l2":
+        out = np.sqrt(A.astype(np.float64) ** 2 + B.astype(np.float64) ** 2)
+    elif combine == "l1":
+        out = np.abs(A) + np.abs(B)
+    elif combine == "sumsq":
+        out = A * A + B * B
+    else:
+        raise ValueError(combine)
+    return out, va & vb
+
+
 _REDUCE_OPS = {"min": 1, "max": 2}
 
 

@@ -212,6 +212,35 @@ def dilate(x: torch.Tensor, size: int = 3, mode="clamp", constant=0.0, **kw) -> 
     return reduce(x, np.ones((size, size)), "max", mode, constant, **kw)
 
 
+_COMBINE = {"l2": _lib.LOP_COMBINE_L2, "l1": _lib.LOP_COMBINE_L1, "sumsq": _lib.LOP_COMBINE_SUMSQ}
+
+
+def convolve2(x: torch.Tensor, mask_a, mask_b, combine="l2", mode="clamp", constant=0.0,
+              out=None, roi=None, offset=(0, 0), stream=None) -> torch.Tensor:
+    """Two local operators on one input combined by a point operator, one pass:
+    combine = "l2" sqrt(A^2 + B^2) (float32), "l1" |A| + |B|, "sumsq" A^2 + B^2.
+    float32 -> float32 or uint8 -> int32."""
+    mdt = _lib.LOP_F32 if x.dtype == torch.float32 else _lib.LOP_I32
+    aa, ma = _host_mask(mask_a, mdt)
+    ab, mb = _host_mask(mask_b, mdt)
+    if out is None:
+        out = torch.empty(x.shape, dtype=torch.float32 if x.dtype == torch.float32 else torch.int32,
+                          device=x.device)
+    return _execute("convolve2", x, out, mode, constant, (ma.size_x, ma.size_y), roi, offset,
+                    stream, (0, 0, 0, 0),
+                    lambda is_, acc, s: lib.lop_convolve2_execute(is_, acc, ctypes.byref(ma),
+                                                                  ctypes.byref(mb),
+                                                                  _COMBINE[combine], s))
+
+
+def sobel_magnitude(x: torch.Tensor, mode="clamp", constant=0.0, **kw) -> torch.Tensor:
+    """Sobel gradient magnitude in one pass: sqrt(gx^2 + gy^2) for float32
+    images, |gx| + |gy| (int32) for uint8 images."""
+    dt = np.float32 if x.dtype == torch.float32 else np.int32
+    combine = "l2" if x.dtype == torch.float32 else "l1"
+    return convolve2(x, sobel_mask(0, dt), sobel_mask(1, dt), combine, mode, constant, **kw)
+
+
 def gaussian(x: torch.Tensor, size: int = 5, mode="clamp", constant=0.0, **kw) -> torch.Tensor:
     """Binomial Gaussian (Tables VIII-IX; reading c11): f32 -> f32, u8 -> u8."""
     if x.dtype == torch.float32:

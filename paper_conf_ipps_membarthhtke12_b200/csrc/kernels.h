@@ -21,6 +21,10 @@ bool conv_factor(const ConvGeneric &p, ConvSep &s);
 // Local MIN / MAX over a mask domain (reduce.cu): tiled separable kernel for
 // full windows up to 9x9, generic kernel otherwise.
 cudaError_t launch_reduce(const ReduceParams &p, bool allow_tiled, cudaStream_t stream);
+// Two local operators combined by a point operator (conv_pair.cu); the tiled
+// launcher returns cudaErrorNotSupported when no instance matches.
+cudaError_t launch_conv_pair(const ConvPair &p, cudaStream_t stream);
+cudaError_t launch_conv_pair_generic(const ConvPairGeneric &p, cudaStream_t stream);
 // Fused two-stage convolution; cudaErrorNotSupported if no instance matches.
 cudaError_t launch_conv_chain(const ConvChain &p, cudaStream_t stream);
 

@@ -505,6 +505,93 @@ lop_status lop_reduce_execute(const lop_iteration_space *is, const lop_accessor 
                     "reduce launch");
 }
 
+// -------------------------------- two local operators + point-operator epilogue
+lop_status lop_convolve2_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                 const lop_mask *a, const lop_mask *b, int32_t combine,
+                                 void *cuda_stream)
+{
+    if (combine < LOP_COMBINE_L2 || combine > LOP_COMBINE_SUMSQ)
+        return fail(LOP_ERR_INVALID, "unknown combine %d (L2, L1, SUMSQ)", combine);
+    Prepared pp;
+    lop_status st = prepare(is, in, pp);
+    if (st) return st;
+    const lop::Common &c = pp.c;
+    if (!a || !a->coeffs || !b || !b->coeffs) return fail(LOP_ERR_INVALID, "mask is NULL");
+    const int sx = 2 * c.rx + 1, sy = 2 * c.ry + 1;
+    if (a->size_x != sx || a->size_y != sy || b->size_x != sx || b->size_y != sy)
+        return fail(LOP_ERR_INVALID, "masks must both be the window size %d x %d", sx, sy);
+    if (c.rx > lop::kPairMaxR || c.ry > lop::kPairMaxR)
+        return fail(LOP_ERR_UNSUPPORTED, "window %d x %d larger than 31 x 31", sx, sy);
+    const int32_t idt = in->bc->image.dtype, odt = is->image.dtype;
+    int u8 = 0;
+    if (idt == LOP_F32 && odt == LOP_F32) {
+        if (a->dtype != LOP_F32 || b->dtype != LOP_F32 || a->shift || b->shift)
+            return fail(LOP_ERR_INVALID, "F32 images need F32 masks with shift 0");
+        u8 = 0;
+    } else if (idt == LOP_U8 && odt == LOP_I32) {
+        if (a->dtype != LOP_I32 || b->dtype != LOP_I32 || a->shift || b->shift)
+            return fail(LOP_ERR_INVALID, "U8 images need I32 masks with shift 0");
+        if (combine == LOP_COMBINE_L2)
+            return fail(LOP_ERR_INVALID, "LOP_COMBINE_L2 needs F32 images (U8 -> I32 is exact: L1 or SUMSQ)");
+        u8 = 1;
+        int64_t la = 0, lb = 0;
+        for (int i = 0; i < sx * sy; ++i) {
+            const int32_t va = static_cast<const int32_t *>(a->coeffs)[i];
+            const int32_t vb = static_cast<const int32_t *>(b->coeffs)[i];
+            la += va < 0 ? -(int64_t)va : va;
+            lb += vb < 0 ? -(int64_t)vb : vb;
+        }
+        const int64_t ma = 255 * la, mb = 255 * lb;
+        if (ma * ma + mb * mb >= (1ll << 31))
+            return fail(LOP_ERR_UNSUPPORTED, "integer masks too large: the combined value may overflow int32");
+    } else {
+        return fail(LOP_ERR_INVALID, "unsupported dtype combination %d -> %d (F32->F32, U8->I32)",
+                    idt, odt);
+    }
+    cudaStream_t stream = static_cast<cudaStream_t>(cuda_stream);
+    // tiled: both masks exactly separable (the convolution's own factorisation)
+    static thread_local lop::ConvGeneric g;
+    static thread_local lop::ConvPair tp;
+    bool sep = c.rx == c.ry && c.rx >= 1 && c.rx <= 2 && g_variant != LOP_VARIANT_GENERIC;
+    for (int k = 0; k < 2 && sep; ++k) {
+        const lop_mask *m = k ? b : a;
+        g.c = c;
+        g.kind = u8 ? lop::CONV_U8_I32 : lop::CONV_F32;
+        g.shift = 0;
+        for (int i = 0; i < sx * sy; ++i) {
+            if (u8) g.m.i[i] = static_cast<const int32_t *>(m->coeffs)[i];
+            else g.m.f[i] = static_cast<const float *>(m->coeffs)[i];
+        }
+        lop::ConvSep &s = k ? tp.b : tp.a;
+        sep = lop::conv_factor(g, s);
+        s.c = c;
+        s.kind = g.kind;
+        s.shift = 0;
+    }
+    if (sep) {
+        tp.combine = combine;
+        tp.u8 = u8;
+        cudaError_t e = lop::launch_conv_pair(tp, stream);
+        if (e != cudaErrorNotSupported) return launched(e, "conv_pair launch");
+    }
+    if (g_variant == LOP_VARIANT_TILED)
+        return fail(LOP_ERR_UNSUPPORTED, "no tiled instance for this mask pair");
+    static thread_local lop::ConvPairGeneric gp;
+    gp.c = c;
+    gp.combine = combine;
+    gp.u8 = u8;
+    for (int i = 0; i < sx * sy; ++i) {
+        if (u8) {
+            gp.ia[i] = static_cast<const int32_t *>(a->coeffs)[i];
+            gp.ib[i] = static_cast<const int32_t *>(b->coeffs)[i];
+        } else {
+            gp.ma[i] = static_cast<const float *>(a->coeffs)[i];
+            gp.mb[i] = static_cast<const float *>(b->coeffs)[i];
+        }
+    }
+    return launched(lop::launch_conv_pair_generic(gp, stream), "conv_pair_generic launch");
+}
+
 // ------------------------------------------------- fused two-stage operator
 namespace {
 // One stage's mask -> exact separable factors (reusing the convolution path).

@@ -115,6 +115,25 @@ struct ReduceParams {
     uint64_t dom[2 * kMaxRadius + 1];
 };
 
+// Two local operators on one input, combined by a point operator (conv_pair.cu):
+// out = combine(Ma (*) I, Mb (*) I).  L2: sqrt(a^2 + b^2) (f32), L1: |a| + |b|,
+// SUMSQ: a^2 + b^2.  f32 -> f32 or u8 -> i32.
+enum PairCombine { PAIR_L2 = 0, PAIR_L1 = 1, PAIR_SUMSQ = 2 };
+struct ConvPair {            // both masks exactly separable, same radius <= 2
+    ConvSep a, b;            // a.c holds the launch geometry
+    int32_t combine;
+    int32_t u8;
+};
+constexpr int kPairMaxR = 15;                                 // generic pair: windows up to 31x31
+constexpr int kPairMaxTaps = (2 * kPairMaxR + 1) * (2 * kPairMaxR + 1);
+struct ConvPairGeneric {
+    Common c;
+    int32_t combine;
+    int32_t u8;
+    union { float ma[kPairMaxTaps]; int32_t ia[kPairMaxTaps]; };
+    union { float mb[kPairMaxTaps]; int32_t ib[kPairMaxTaps]; };
+};
+
 // Row-streaming plan of the fused chain (conv_chain.cu, set by the launcher):
 // warps stream output rows [sy0, sy1) in frames of 32 lanes; the rows above
 // and below (where pass 2 reads G outside the image) are band tiles of the

@@ -10,9 +10,10 @@
 //  * reduce_tiled_kernel<T, OP, R>: full square windows up to 9x9 -- the
 //    domain is a rectangle, so min/max is separable (row reduction, then
 //    column reduction).  Tile staging as the convolution kernels (stage.cuh:
-//    one cp.async.bulk per row, boundary resolved at staging time).  u8: four
-//    pixels per instruction with the byte-SIMD __vminu4 / __vmaxu4 on funnel-
-//    shifted words; f32: FMNMX per pixel.  HBM-bound (2 or 8 bytes per pixel).
+//    one cp.async.bulk per row, boundary resolved at staging time).  u8: two
+//    pixels per instruction in 16-bit lanes with the native 3-input
+//    VIMNMX3.U16x2 (pixels q, q+2 per register, as the SWAR convolution);
+//    f32: FMNMX per pixel.  HBM-bound (2 or 8 bytes per pixel).
 //  * reduce_generic_kernel: any domain up to 63x63 (one bit per tap), one
 //    thread per output pixel, per-tap boundary resolution.
 #include <cuda_runtime.h>
@@ -40,9 +41,23 @@ template <int OP> __device__ __forceinline__ float red_f(float a, float b)
 {
     return OP == RED_MIN ? fminf(a, b) : fmaxf(a, b);
 }
-template <int OP> __device__ __forceinline__ uint32_t red_u4(uint32_t a, uint32_t b)
+// u8 pixels in 16-bit lanes: native VIMNMX.U16x2 / VIMNMX3.U16x2 (3-input)
+// on sm_100 (the byte-SIMD __vminu4 is emulated with ~7 instructions).
+template <int OP> __device__ __forceinline__ uint32_t red2(uint32_t a, uint32_t b)
 {
-    return OP == RED_MIN ? __vminu4(a, b) : __vmaxu4(a, b);
+    return OP == RED_MIN ? __vminu2(a, b) : __vmaxu2(a, b);
+}
+template <int OP> __device__ __forceinline__ uint32_t red3(uint32_t a, uint32_t b, uint32_t c)
+{
+    return OP == RED_MIN ? __vimin3_u16x2(a, b, c) : __vimax3_u16x2(a, b, c);
+}
+// reduction of x[0..N-1] with 3-input instructions
+template <int OP, int N> __device__ __forceinline__ uint32_t red_n(const uint32_t *x)
+{
+    uint32_t m = N >= 3 ? red3<OP>(x[0], x[1], x[2]) : (N == 2 ? red2<OP>(x[0], x[1]) : x[0]);
+#pragma unroll
+    for (int i = 3; i < N; i += 2) m = i + 1 < N ? red3<OP>(m, x[i], x[i + 1]) : red2<OP>(m, x[i]);
+    return m;
 }
 
 template <typename T, int OP, int R>
@@ -76,7 +91,9 @@ __global__ void __launch_bounds__(red::NT) reduce_tiled_kernel(const __grid_cons
                         (sizeof(T) * PX)) == 0);
     const T *tcol = tile + PADE + threadIdx.x * PX;
     if constexpr (sizeof(T) == 1) {
-        uint32_t h[P][2];                                        // row reductions, ring
+        // staged words W0..W3 = bytes -4..11 of this thread's 8 columns; sources
+        // S[q + R] = bytes (q, q+2) in the two 16-bit lanes (as conv_u8_swar)
+        uint32_t h[P][4];                                        // lanes (0,2) (1,3) (4,6) (5,7)
 #pragma unroll
         for (int k = 0; k < TS + 2 * R; ++k) {
             if (k >= srows) break;
@@ -84,33 +101,42 @@ __global__ void __launch_bounds__(red::NT) reduce_tiled_kernel(const __grid_cons
             const uint2 cv = *reinterpret_cast<const uint2 *>(rp);
             const uint32_t W[4] = {*reinterpret_cast<const uint32_t *>(rp - 4), cv.x, cv.y,
                                    *reinterpret_cast<const uint32_t *>(rp + 8)};
+            uint32_t E[4], O[4];
 #pragma unroll
-            for (int w = 0; w < 2; ++w) {                        // output words: bytes 4w .. 4w+3
-                uint32_t m = W[w + 1];
-#pragma unroll
-                for (int s = 1; s <= R; ++s) {
-                    m = red_u4<OP>(m, __funnelshift_rc(W[w + 1], W[w + 2], 8 * s));       // bytes +s (s = 4: W[w+2])
-                    m = red_u4<OP>(m, __funnelshift_rc(W[w], W[w + 1], 32 - 8 * s));      // bytes -s (s = 4: W[w])
-                }
-                h[k % P][w] = m;
+            for (int i = 0; i < 4; ++i) {
+                E[i] = __byte_perm(W[i], 0u, 0x4240);
+                O[i] = __byte_perm(W[i], 0u, 0x4341);
             }
+            uint32_t Sx[6 + 2 * R];
+#pragma unroll
+            for (int q = -R; q <= 5 + R; ++q) {
+                const int wi = (q + 4) >> 2, sh = (q + 4) & 3;
+                if (sh == 0) Sx[q + R] = E[wi];
+                else if (sh == 1) Sx[q + R] = O[wi];
+                else if (sh == 2) Sx[q + R] = __byte_perm(E[wi], E[wi + 1], 0x5412);
+                else Sx[q + R] = __byte_perm(O[wi], O[wi + 1], 0x5412);
+            }
+            constexpr int J[4] = {0, 1, 4, 5};
+#pragma unroll
+            for (int jj = 0; jj < 4; ++jj) h[k % P][jj] = red_n<OP, P>(Sx + J[jj]);
             const int o = k - 2 * R;
             if (o < 0) continue;
-            uint32_t q[2];
+            uint32_t q4[4];
 #pragma unroll
-            for (int w = 0; w < 2; ++w) {
-                uint32_t m = h[o % P][w];
+            for (int jj = 0; jj < 4; ++jj) {
+                uint32_t col[P];
 #pragma unroll
-                for (int t = 1; t < P; ++t) m = red_u4<OP>(m, h[(o + t) % P][w]);
-                q[w] = m;
+                for (int t = 0; t < P; ++t) col[t] = h[(o + t) % P][jj];
+                q4[jj] = red_n<OP, P>(col);
             }
+            const uint32_t lo = __byte_perm(q4[0], q4[1], 0x6240), hi = __byte_perm(q4[2], q4[3], 0x6240);
             uint8_t *op = reinterpret_cast<uint8_t *>(obase + (int64_t)o * c.out.stride) + ox0;
             if (ovec) {
-                *reinterpret_cast<uint2 *>(op) = make_uint2(q[0], q[1]);
+                *reinterpret_cast<uint2 *>(op) = make_uint2(lo, hi);
             } else {
 #pragma unroll
                 for (int j = 0; j < 8; ++j)
-                    if (ox0 + j < roi_x1) op[j] = (uint8_t)(q[j >> 2] >> (8 * (j & 3)));
+                    if (ox0 + j < roi_x1) op[j] = (uint8_t)((j < 4 ? lo : hi) >> (8 * (j & 3)));
             }
         }
     } else {

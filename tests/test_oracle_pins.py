@@ -471,3 +471,38 @@ def test_reduce_undefined_valid_region():
     assert np.array_equal(valid, exp)
     ref, _ = oracle.reduce(img, dom, "max", "clamp")
     assert np.array_equal(out[valid], ref[valid])
+
+
+# ---------------------- two local operators + point-operator epilogue (N3) ----
+
+@pytest.mark.parametrize("mode", ["clamp", "mirror"])
+def test_convolve2_sobel_magnitude_on_ramps(mode):
+    """Sobel magnitude of a ramp I = a x + b y: gx = 8a, gy = 8b in the interior
+    (the Sobel ramp pin above), so L2 = 8 sqrt(a^2 + b^2), L1 = 8 (|a| + |b|),
+    SUMSQ = 64 (a^2 + b^2); exact for integer ramps on u8."""
+    sx, sy = oracle.sobel_mask(0), oracle.sobel_mask(1)
+    ys, xs = np.mgrid[0:20, 0:24]
+    a, b = 3, -2
+    u8 = (100 + a * xs + b * ys).astype(np.uint8)
+    l1, _ = oracle.convolve2(u8, sx, sy, "l1", mode)
+    sq, _ = oracle.convolve2(u8, sx, sy, "sumsq", mode)
+    assert (l1[1:-1, 1:-1] == 8 * (abs(a) + abs(b))).all()
+    assert (sq[1:-1, 1:-1] == 64 * (a * a + b * b)).all()
+    f = (0.01 * a * xs + 0.01 * b * ys).astype(np.float32)
+    l2, _ = oracle.convolve2(f, sx.astype(np.float64), sy.astype(np.float64), "l2", mode)
+    gx, _ = oracle.convolve_f32(f, sx.astype(np.float64), mode)
+    gy, _ = oracle.convolve_f32(f, sy.astype(np.float64), mode)
+    np.testing.assert_allclose(l2[1:-1, 1:-1], 0.08 * math.hypot(a, b), rtol=1e-5)
+    np.testing.assert_allclose(l2, np.hypot(gx, gy), rtol=1e-14, atol=1e-15)
+
+
+def test_convolve2_transpose_symmetry():
+    """Swapping the image axes swaps Sobel-x and Sobel-y: the L2 / L1 magnitude
+    of the transposed image is the transposed magnitude (symmetric modes)."""
+    rng = _rng(21)
+    img = rng.random((17, 23)).astype(np.float32)
+    sx, sy = oracle.sobel_mask(0).astype(np.float64), oracle.sobel_mask(1).astype(np.float64)
+    for mode in ("clamp", "mirror", "repeat"):
+        m, _ = oracle.convolve2(img, sx, sy, "l2", mode)
+        mt, _ = oracle.convolve2(np.ascontiguousarray(img.T), sx, sy, "l2", mode)
+        np.testing.assert_allclose(mt, m.T, rtol=0, atol=1e-12)

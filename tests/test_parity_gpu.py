@@ -702,3 +702,103 @@ def test_reduce_roi_offset_frames_and_validation(lop):
         lop.reduce(img, np.zeros((3, 3), np.float32), "min")
     with pytest.raises(KeyError):
         lop.reduce(img, np.ones((3, 3), np.float32), "median")
+
+
+# ------------------ two local operators + point-operator epilogue (N3) ----
+
+def _np_combine(a, b, combine):
+    """The epilogue in the kernel's precision and order (IEEE f32: a*a, b*b, +,
+    sqrt; exact int64 for integers)."""
+    if a.dtype == np.float32:
+        if combine == "l1":
+            return np.abs(a) + np.abs(b)
+        s = a * a + b * b
+        return np.sqrt(s) if combine == "l2" else s
+    a, b = a.astype(np.int64), b.astype(np.int64)
+    return np.abs(a) + np.abs(b) if combine == "l1" else a * a + b * b
+
+
+@pytest.mark.parametrize("shape", [(1, 1), (5, 7), (33, 130), (70, 600), (129, 1031)])
+@pytest.mark.parametrize("mode", MODES)
+def test_convolve2_equals_two_passes_and_oracle(lop, shape, mode):
+    """Fused A/B + epilogue (Sobel magnitude; random separable 5x5 pairs) == the
+    epilogue applied to two lop.convolve passes, bit for bit (tiled kernel),
+    and == the oracle (f32 within 1e-5 x scale, u8 -> i32 exact)."""
+    H, W = shape
+    rng = np.random.default_rng(H * 7 + W)
+    img = synthetic.uniform(H, W, seed=H + 11 * W)
+    u8 = synthetic.uniform_u8(H, W, seed=H * 5 + W)
+    sxf, syf = lop.sobel_mask(0, np.float32), lop.sobel_mask(1, np.float32)
+    sxi, syi = lop.sobel_mask(0, np.int32), lop.sobel_mask(1, np.int32)
+    ra = np.outer(rng.integers(-3, 4, 5), rng.integers(-3, 4, 5)).astype(np.int32)
+    rb = np.outer(rng.integers(-3, 4, 5), rng.integers(-3, 4, 5)).astype(np.int32)
+    # float pairs whose column ratios are powers of two (the float factorisation
+    # is exact, so both take the tiled kernel, as each lop.convolve pass does)
+    fa = np.outer(rng.choice([-4, -2, -1, 1, 2, 4], 5), rng.integers(-8, 9, 5) / 8.0)
+    fb = np.outer(rng.choice([-2, -1, 1, 2], 5), rng.integers(-8, 9, 5) / 4.0)
+    pairs_f = [(sxf, syf), (fa.astype(np.float32), fb.astype(np.float32))]
+    pairs_i = [(sxi, syi), (ra, rb)]
+    for (ma, mb) in pairs_f:
+        for combine in ("l2", "l1", "sumsq"):
+            fused = lop.convolve2(img.cuda(), ma, mb, combine, mode, constant=0.5).cpu().numpy()
+            a = lop.convolve(img.cuda(), ma, mode, constant=0.5).cpu().numpy()
+            b = lop.convolve(img.cuda(), mb, mode, constant=0.5).cpu().numpy()
+            if mode != "undefined":
+                assert np.array_equal(fused, _np_combine(a, b, combine)), (combine, ma.shape)
+            ref, valid = oracle.convolve2(img.numpy(), ma.astype(np.float64), mb.astype(np.float64),
+                                          combine, mode, 0.5)
+            sel = valid if mode == "undefined" else np.ones_like(valid)
+            scale = max(1.0, float(np.abs(ref[sel]).max()) if sel.any() else 1.0)
+            _cmp_float(fused, ref, sel, tol=1e-5 * scale)
+    for (ma, mb) in pairs_i:
+        for combine in ("l1", "sumsq"):
+            fused = lop.convolve2(u8.cuda(), ma, mb, combine, mode, constant=77).cpu().numpy()
+            assert fused.dtype == np.int32
+            ref, valid = oracle.convolve2(u8.numpy(), ma, mb, combine, mode, 77)
+            sel = valid if mode == "undefined" else slice(None)
+            assert np.array_equal(fused[sel].astype(np.int64), ref[sel]), (combine, mode)
+
+
+@pytest.mark.parametrize("mode", ["clamp", "repeat", "constant"])
+def test_convolve2_generic_masks_roi_offset(lop, mode):
+    """Non-separable / 7x7 mask pairs take the generic kernel (2D sums); ROI and
+    accessor offsets; validation."""
+    rng = np.random.default_rng(3)
+    img = synthetic.uniform(45, 140, seed=9)
+    u8 = synthetic.uniform_u8(45, 140, seed=10)
+    ma = rng.standard_normal((7, 7)).astype(np.float32)
+    mb = rng.standard_normal((7, 7)).astype(np.float32)
+    out = lop.convolve2(img.cuda(), ma, mb, "l2", mode, constant=0.3).cpu().numpy()
+    ref, _ = oracle.convolve2(img.numpy(), ma.astype(np.float64), mb.astype(np.float64), "l2",
+                              mode, 0.3)
+    _cmp_float(out, ref, tol=1e-4)
+    ia = rng.integers(-2, 3, (7, 7)).astype(np.int32)     # |A|, |B| <= 255 * 98: A^2 + B^2 fits int32
+    ib = rng.integers(-2, 3, (7, 7)).astype(np.int32)
+    q = lop.convolve2(u8.cuda(), ia, ib, "sumsq", mode, constant=3).cpu().numpy()
+    refq, _ = oracle.convolve2(u8.numpy(), ia, ib, "sumsq", mode, 3)
+    assert np.array_equal(q.astype(np.int64), refq)
+    full = lop.sobel_magnitude(img.cuda(), mode)
+    o = torch.full_like(full, -1.0)
+    lop.convolve2(img.cuda(), lop.sobel_mask(0, np.float32), lop.sobel_mask(1, np.float32), "l2",
+                  mode, out=o, roi=(9, 4, 100, 30))
+    assert torch.equal(o[4:34, 9:109], full[4:34, 9:109]) and bool((o[:4] == -1).all())
+    off = lop.sobel_magnitude(img.cuda(), mode, offset=(2, -1)).cpu().numpy()
+    gx = lop.sobel(img.cuda(), 0, mode, offset=(2, -1)).cpu().numpy()
+    gy = lop.sobel(img.cuda(), 1, mode, offset=(2, -1)).cpu().numpy()
+    assert np.array_equal(off, _np_combine(gx, gy, "l2"))
+    with pytest.raises(lop.LopError, match="L2 needs F32"):
+        lop.convolve2(u8.cuda(), lop.sobel_mask(0, np.int32), lop.sobel_mask(1, np.int32), "l2")
+
+
+def test_sobel_magnitude_4096(lop):
+    """Config-3 size: the u8 Sobel L1 magnitude every output exact; f32 L2 sampled."""
+    img = synthetic.angio(4096, 4096, seed=synthetic.config_seed(3), device="cuda")
+    u8 = synthetic.to_u8(img)
+    q = lop.sobel_magnitude(u8, "mirror").cpu().numpy()
+    ref, _ = oracle.convolve2(u8.cpu().numpy(), oracle.sobel_mask(0), oracle.sobel_mask(1), "l1",
+                              "mirror")
+    assert np.array_equal(q.astype(np.int64), ref)
+    f = lop.sobel_magnitude(img, "clamp").cpu().numpy()
+    gx = lop.sobel(img, 0, "clamp").cpu().numpy()
+    gy = lop.sobel(img, 1, "clamp").cpu().numpy()
+    assert np.array_equal(f, _np_combine(gx, gy, "l2"))
