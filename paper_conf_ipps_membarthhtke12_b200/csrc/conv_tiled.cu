@@ -513,6 +513,13 @@ cudaError_t launch_cfg(const ConvSep &s, cudaStream_t stream)
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(
             &per_sm, conv_sep_kernel<T, TO, R, SWAR, TS, NBUF>, convt::NT, smem);
         grid_max = sms * (per_sm > 0 ? per_sm : 1);
+        // persistent (NBUF = 2) grid: LOP_CONV_CTAS_PER_SM caps the resident CTAs so
+        // that each walks several tiles (otherwise a 4096^2 u8 image -- 1024 tiles --
+        // fits in one wave and the double buffer never pipelines)
+        if (const char *env = std::getenv("LOP_CONV_CTAS_PER_SM")) {
+            const int cap = std::atoi(env);
+            if (cap > 0 && sms * cap < grid_max) grid_max = sms * cap;
+        }
     }
     const long ntiles = (long)((s.c.roi_w + S::TWE - 1) / S::TWE) * ((s.c.roi_h + TS - 1) / TS) *
                         s.c.batch;
