@@ -250,12 +250,25 @@ lop_status lop_pipeline_bilateral(lop_pipeline *p, const float *host_in, int64_t
                                   float *host_out, int64_t out_stride_bytes, int32_t mode,
                                   double constant, int32_t size_x, int32_t size_y,
                                   const lop_mask *closeness, float sigma_d, float sigma_r);
+/* A sequence of nframes images (an angiography run, L102-L104; BASELINE config
+ * 4): frame f at host_in + f * in_frame_stride_bytes, its result at host_out +
+ * f * out_frame_stride_bytes.  The frames stream through the chunk ring back
+ * to back -- frame f+1 uploads while frame f is filtered and downloaded --
+ * so only the first upload and the last download are not overlapped.  Each
+ * frame is filtered exactly as by lop_pipeline_bilateral. */
+lop_status lop_pipeline_bilateral_frames(lop_pipeline *p, const float *host_in,
+                                         int64_t in_stride_bytes, int64_t in_frame_stride_bytes,
+                                         float *host_out, int64_t out_stride_bytes,
+                                         int64_t out_frame_stride_bytes, int32_t nframes,
+                                         int32_t mode, double constant, int32_t size_x,
+                                         int32_t size_y, const lop_mask *closeness, float sigma_d,
+                                         float sigma_r);
 lop_status lop_pipeline_convolve(lop_pipeline *p, const void *host_in, int32_t in_dtype,
                                  int64_t in_stride_bytes, void *host_out, int32_t out_dtype,
                                  int64_t out_stride_bytes, int32_t mode, double constant,
                                  const lop_mask *mask);
 /* Host->device and device->host bytes moved by the last pipeline call
- * (image rows + window halo rows re-uploaded at chunk seams). */
+ * (image rows + window halo rows re-uploaded at chunk seams; all frames). */
 lop_status lop_pipeline_bytes(const lop_pipeline *p, int64_t *h2d, int64_t *d2h);
 lop_status lop_pipeline_destroy(lop_pipeline *p);
 

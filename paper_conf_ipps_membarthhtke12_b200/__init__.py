@@ -353,6 +353,28 @@ class Pipeline:
                                           float(sigma_r)))
         return host_out
 
+    def bilateral_frames(self, host_in: torch.Tensor, host_out: torch.Tensor, sigma_d: float,
+                         sigma_r: float, mode="clamp", constant=0.0, size=None, mask=None):
+        """A (F, H, W) host sequence streamed through the pipeline back to back
+        (frame f+1 uploads while frame f computes / downloads)."""
+        if host_in.is_cuda or host_in.dim() != 3 or host_in.stride(-1) != 1 or \
+                host_out.shape != host_in.shape or host_out.stride(-1) != 1:
+            raise ValueError("pipeline frames need (F, H, W) host tensors with contiguous rows")
+        es = host_in.element_size()
+        if mask is not None:
+            marr, m = _host_mask(mask, _lib.LOP_F32)
+            sx, sy, mptr = m.size_x, m.size_y, ctypes.byref(m)
+        else:
+            size = int(round(4 * sigma_d)) + 1 if size is None else size
+            sx, sy = (size, size) if isinstance(size, int) else size
+            mptr = None
+        _check(lib.lop_pipeline_bilateral_frames(
+            self._h, host_in.data_ptr(), host_in.stride(1) * es, host_in.stride(0) * es,
+            host_out.data_ptr(), host_out.stride(1) * es, host_out.stride(0) * es,
+            int(host_in.shape[0]), _mode(mode), float(constant), sx, sy, mptr, float(sigma_d),
+            float(sigma_r)))
+        return host_out
+
     def convolve(self, host_in: torch.Tensor, host_out: torch.Tensor, mask, mode="clamp",
                  constant=0.0, shift=0):
         ip, istr = self._host(host_in)

@@ -79,6 +79,9 @@ SIGNATURES = {
     "lop_pipeline_create": (c_i32, [c_i32, c_i32, c_i32, c_i32, ctypes.POINTER(c_vp)]),
     "lop_pipeline_bilateral": (c_i32, [c_vp, c_vp, c_i64, c_vp, c_i64, c_i32, c_dbl, c_i32,
                                        c_i32, ctypes.POINTER(lop_mask), c_flt, c_flt]),
+    "lop_pipeline_bilateral_frames": (c_i32, [c_vp, c_vp, c_i64, c_i64, c_vp, c_i64, c_i64,
+                                              c_i32, c_i32, c_dbl, c_i32, c_i32,
+                                              ctypes.POINTER(lop_mask), c_flt, c_flt]),
     "lop_pipeline_convolve": (c_i32, [c_vp, c_vp, c_i32, c_i64, c_vp, c_i32, c_i64, c_i32,
                                       c_dbl, ctypes.POINTER(lop_mask)]),
     "lop_pipeline_bytes": (c_i32, [c_vp, ctypes.POINTER(c_i64), ctypes.POINTER(c_i64)]),

@@ -145,10 +145,14 @@ std::vector<int> chunk_schedule(int H, int c)
     return cuts;
 }
 
+// nframes images (frame f at host_in + f * in_fstride, host_out + f * out_fstride)
+// stream through the same ring back to back: the chunks of frame f+1 upload
+// while frame f computes and downloads, with no drain between frames.
 template <typename Exec>
 lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t in_stride,
                void *host_out, int32_t out_dtype, int64_t out_stride, int mode, double constant,
-               int size_x, int size_y, Exec exec)
+               int size_x, int size_y, Exec exec, int nframes = 1, int64_t in_fstride = 0,
+               int64_t out_fstride = 0)
 {
     if (!p || !host_in || !host_out) return pfail(LOP_ERR_INVALID, "NULL pipeline or host buffer");
     const int ry = size_y / 2;
@@ -161,10 +165,10 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
     p->h2d_bytes = p->d2h_bytes = 0;
     static const bool trace = std::getenv("LOP_PIPELINE_TRACE") != nullptr;
     const auto t_start = std::chrono::steady_clock::now();
-    const char *hin = static_cast<const char *>(host_in);
-    char *hout = static_cast<char *>(host_out);
+    if (nframes < 1) return pfail(LOP_ERR_INVALID, "nframes must be >= 1");
     const std::vector<int> cuts = chunk_schedule(p->H, p->chunk);
     const int nchunks = (int)cuts.size() - 1;
+    const int ntotal = nchunks * nframes;
     // trace mode: per-chunk timeline (upload start/end, compute end, download end)
     std::vector<cudaEvent_t> tev;
     auto tmark = [&](cudaStream_t s) {
@@ -174,11 +178,14 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
         cudaEventRecord(ev, s);
         tev.push_back(ev);
     };
-    for (int k = 0; k < nchunks; ++k) {
-        const int buf = k % p->nbufs;
+    for (int kk = 0; kk < ntotal; ++kk) {
+        const int f = kk / nchunks, k = kk - f * nchunks;       // frame, chunk within the frame
+        const char *hin = static_cast<const char *>(host_in) + (int64_t)f * in_fstride;
+        char *hout = static_cast<char *>(host_out) + (int64_t)f * out_fstride;
+        const int buf = kk % p->nbufs;
         const int y0 = cuts[k], y1 = cuts[k + 1];
         cudaError_t e;
-        if (k >= p->nbufs) {
+        if (kk >= p->nbufs) {
             e = cudaStreamWaitEvent(p->s_h2d, p->comp_done[buf], 0);
             if (e != cudaSuccess) return perr(e, "wait");
         }
@@ -189,7 +196,7 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
         tmark(p->s_h2d);
         cudaEventRecord(p->up_done[buf], p->s_h2d);
         cudaStreamWaitEvent(p->s_comp, p->up_done[buf], 0);
-        if (k >= p->nbufs) cudaStreamWaitEvent(p->s_comp, p->down_done[buf], 0);
+        if (kk >= p->nbufs) cudaStreamWaitEvent(p->s_comp, p->down_done[buf], 0);
         lop_image out_view;
         std::memset(&out_view, 0, sizeof out_view);
         out_view.data = p->d_out[buf];
@@ -231,14 +238,14 @@ lop_status run(lop_pipeline *p, const void *host_in, int32_t in_dtype, int64_t i
         cudaStreamSynchronize(p->s_d2h);
         const double t_all = std::chrono::duration<double, std::milli>(
                                  std::chrono::steady_clock::now() - t_start).count();
-        std::fprintf(stderr, "lop_pipeline: %d chunks, enqueue %.3f ms, total %.3f ms\n",
-                     nchunks, t_enq, t_all);
+        std::fprintf(stderr, "lop_pipeline: %d chunks x %d frames, enqueue %.3f ms, total %.3f ms\n",
+                     nchunks, nframes, t_enq, t_all);
         // per chunk: rows, upload [start, end], compute [start, end], download end (ms from the first mark)
-        for (int k = 0; k < nchunks && (size_t)(5 * k + 4) < tev.size(); ++k) {
+        for (int k = 0; k < ntotal && (size_t)(5 * k + 4) < tev.size(); ++k) {
             float t[5];
             for (int i = 0; i < 5; ++i) cudaEventElapsedTime(&t[i], tev[0], tev[5 * k + i]);
             std::fprintf(stderr, "  chunk %2d rows %4d  up %.3f-%.3f  comp %.3f-%.3f  down-end %.3f\n", k,
-                         cuts[k + 1] - cuts[k], t[0], t[1], t[2], t[3], t[4]);
+                         cuts[k % nchunks + 1] - cuts[k % nchunks], t[0], t[1], t[2], t[3], t[4]);
         }
         for (cudaEvent_t ev : tev) cudaEventDestroy(ev);
     }
@@ -300,6 +307,22 @@ lop_status lop_pipeline_bilateral(lop_pipeline *p, const float *host_in, int64_t
                [&](const lop_iteration_space *is, const lop_accessor *acc, cudaStream_t s) {
                    return lop_bilateral_execute(is, acc, closeness, sigma_d, sigma_r, s);
                });
+}
+
+lop_status lop_pipeline_bilateral_frames(lop_pipeline *p, const float *host_in,
+                                         int64_t in_stride_bytes, int64_t in_frame_stride_bytes,
+                                         float *host_out, int64_t out_stride_bytes,
+                                         int64_t out_frame_stride_bytes, int32_t nframes,
+                                         int32_t mode, double constant, int32_t size_x,
+                                         int32_t size_y, const lop_mask *closeness, float sigma_d,
+                                         float sigma_r)
+{
+    return run(p, host_in, LOP_F32, in_stride_bytes, host_out, LOP_F32, out_stride_bytes, mode,
+               constant, size_x, size_y,
+               [&](const lop_iteration_space *is, const lop_accessor *acc, cudaStream_t s) {
+                   return lop_bilateral_execute(is, acc, closeness, sigma_d, sigma_r, s);
+               },
+               nframes, in_frame_stride_bytes, out_frame_stride_bytes);
 }
 
 lop_status lop_pipeline_convolve(lop_pipeline *p, const void *host_in, int32_t in_dtype,

@@ -489,6 +489,27 @@ def test_pipeline_host_end_to_end(lop):
     p.close()
 
 
+@pytest.mark.parametrize("bufs", ["auto", "2", "3"])
+def test_pipeline_frames_stream(lop, bufs, monkeypatch):
+    """A frame sequence streamed through the pipeline back to back (ring wraps
+    across frames, small rings included) == each frame filtered on the device."""
+    if bufs != "auto":
+        monkeypatch.setenv("LOP_PIPELINE_BUFS", bufs)
+    F, H, W = 4, 300, 384
+    frames = synthetic.angio_frames(F, H, W, seed=synthetic.config_seed(4), first=0,
+                                    count=F).contiguous().pin_memory()
+    out = torch.empty_like(frames).pin_memory()
+    p = lop.Pipeline(W, H, chunk_rows=64)
+    for mode in ("clamp", "repeat", "constant"):
+        p.bilateral_frames(frames, out, 3.0, 0.1, mode, constant=0.25)
+        for f in range(F):
+            dev = lop.bilateral(frames[f].cuda(), 3.0, 0.1, mode, constant=0.25).cpu()
+            assert torch.equal(out[f], dev), (mode, f)
+    h2d, d2h = p.bytes_moved()
+    assert d2h == F * H * W * 4 and h2d >= F * H * W * 4
+    p.close()
+
+
 def test_launch_count(lop):
     img = torch.rand(64, 64, device="cuda")
     lop.reset_launch_count()
