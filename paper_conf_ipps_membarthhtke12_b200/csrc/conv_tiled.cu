@@ -64,7 +64,12 @@ template <typename T> struct TileShape {
 // lanes (b1, b3) (PRMT with a zero source); the lanes (q, q+2) that straddle
 // two words are one PRMT of two E (or O) words.  All integer arithmetic is
 // exact, so every MODE gives the same bits.
-enum { SW_ON = 1, SW_SYM = 2, SW_SH8 = 4 };
+// SW_I32 -- u8 -> i32 with signed coefficients (Sobel): every lane starts from
+// a bias (sw_bias_h per row sum, sw_bias_v per column sum) chosen on the host
+// so that the final value of each 16-bit lane lies in [0, 65535] -- the 32-bit
+// arithmetic is modular, so borrows between lanes in intermediate steps cancel
+// once the final low lane is in range -- and S = lane - sw_off exactly.
+enum { SW_ON = 1, SW_SYM = 2, SW_SH8 = 4, SW_I32 = 8 };
 
 template <int R, int TS, int MODE>
 __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tcol, int srows,
@@ -73,9 +78,11 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
 {
     constexpr int SWE = TileShape<uint8_t>::SWE;
     constexpr uint32_t M = 0x00FF00FFu;
-    constexpr bool SYM = (MODE & SW_SYM) != 0, SH8 = (MODE & SW_SH8) != 0;
+    constexpr bool SYM = (MODE & SW_SYM) != 0, SH8 = (MODE & SW_SH8) != 0, I32 = (MODE & SW_I32) != 0;
     static_assert(R <= 3, "SWAR sources cover bytes -4..11");
-    const uint32_t rnd = p.shift > 0 ? (1u << (p.shift - 1)) * 0x00010001u : 0u;
+    const uint32_t rnd = I32 ? (uint32_t)p.sw_bias_v * 0x00010001u
+                             : (p.shift > 0 ? (1u << (p.shift - 1)) * 0x00010001u : 0u);
+    const uint32_t hb = I32 ? (uint32_t)p.sw_bias_h * 0x00010001u : 0u;
     uint32_t h[2 * R + 1][4];                     // pairs (0,2) (1,3) (4,6) (5,7)
 #pragma unroll
     for (int k = 0; k < TS + 2 * R; ++k) {
@@ -109,7 +116,7 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
 #pragma unroll
                 for (int t = 0; t < R; ++t) s += (uint32_t)p.ri[t] * (S[J[jj] + t] + S[J[jj] + 2 * R - t]);
             } else {
-                s = (uint32_t)p.ri[0] * S[J[jj]];
+                s = (uint32_t)p.ri[0] * S[J[jj]] + hb;
 #pragma unroll
                 for (int t = 1; t <= 2 * R; ++t) s += (uint32_t)p.ri[t] * S[J[jj] + t];
             }
@@ -131,7 +138,27 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
 #pragma unroll
                 for (int t = 1; t <= 2 * R; ++t) s += (uint32_t)p.ci[t] * h[(o + t) % (2 * R + 1)][jj];
             }
-            q4[jj] = SH8 ? s : (s >> p.shift) & M;
+            q4[jj] = (SH8 || I32) ? s : (s >> p.shift) & M;
+        }
+        if constexpr (I32) {
+            // lanes -> S = lane - sw_off, then (S + 2^(k-1)) >> k (quantize_shift)
+            int v[8];
+#pragma unroll
+            for (int jj = 0; jj < 4; ++jj) {
+                const int px = J[jj];                                // lanes: pixels px, px + 2
+                v[px] = quantize_shift((int)(q4[jj] & 0xFFFFu) - p.sw_off, p.shift);
+                v[px + 2] = quantize_shift((int)(q4[jj] >> 16) - p.sw_off, p.shift);
+            }
+            int32_t *op = reinterpret_cast<int32_t *>(orow0 + (int64_t)o * ostride) + ox0;
+            if (ovec) {
+                *reinterpret_cast<int4 *>(op) = make_int4(v[0], v[1], v[2], v[3]);
+                *reinterpret_cast<int4 *>(op + 4) = make_int4(v[4], v[5], v[6], v[7]);
+            } else {
+#pragma unroll
+                for (int j = 0; j < 8; ++j)
+                    if (ox0 + j < roi_x1) op[j] = v[j];
+            }
+            continue;
         }
         // lo = pixels 0..3 = lanes of q4[0] (0, 2) and q4[1] (1, 3); hi likewise
         const uint32_t lo = SH8 ? __byte_perm(q4[0], q4[1], 0x7351) : __byte_perm(q4[0], q4[1], 0x6240);
@@ -268,6 +295,7 @@ __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &c
                         (sizeof(TO) * PX > 16 ? 16 : sizeof(TO) * PX)) == 0);
     const T *tcol = tile + PADE + threadIdx.x * PX;              // this thread's centre column
     if constexpr (SWAR != 0) {
+        static_assert(SWAR == 0 || sizeof(T) == 1, "SWAR is for u8 inputs");
         conv_u8_swar<R, TS, SWAR>(p, reinterpret_cast<const uint8_t *>(tcol), srows,
                         obase + (int64_t)ty0 * c.out.stride, c.out.stride, ox0, roi_x1, ovec);
         return;
@@ -565,6 +593,32 @@ cudaError_t dispatch_r(const ConvSep &s, cudaStream_t stream)
 
 // SWAR eligibility (u8 -> u8): non-negative factors, sum fits a 16-bit lane,
 // no saturation (sum r * sum c <= 2^shift) and the lane shift stays in-lane.
+// Signed SWAR eligibility (u8 -> i32) and its lane biases: row sums biased by
+// 255 * sum of the negative row factors, column sums by max_h * sum of the
+// negative column factors; both lanes' final values must stay below 2^16.
+bool swar_i32_prepare(ConvSep &s)
+{
+    // opt-in (LOP_CONV_SWAR_I32=1): measured slower than the unpacked kernel for the
+    // Sobel u8 -> i32 on B200 (22.5 vs 19.3 us at 4096^2) -- the i32
+    // stores and the lane extraction dominate, not the multiply-adds
+    const char *on = std::getenv("LOP_CONV_SWAR_I32");
+    if (!on || std::atoi(on) != 1) return false;
+    if (s.kind != CONV_U8_I32 || s.c.rx < 1 || s.c.rx > 3) return false;
+    int64_t rneg = 0, rpos = 0, cneg = 0, cpos = 0, csum = 0;
+    for (int t = 0; t <= 2 * s.c.rx; ++t) {
+        (s.ri[t] < 0 ? rneg : rpos) += s.ri[t] < 0 ? -(int64_t)s.ri[t] : s.ri[t];
+        (s.ci[t] < 0 ? cneg : cpos) += s.ci[t] < 0 ? -(int64_t)s.ci[t] : s.ci[t];
+        csum += s.ci[t];
+    }
+    const int64_t bias_h = 255 * rneg, max_h = bias_h + 255 * rpos;
+    const int64_t bias_v = max_h * cneg, max_v = bias_v + max_h * cpos;
+    if (max_h > 65535 || max_v > 65535) return false;
+    s.sw_bias_h = (int32_t)bias_h;
+    s.sw_bias_v = (int32_t)bias_v;
+    s.sw_off = (int32_t)(bias_v + bias_h * csum);
+    return true;
+}
+
 bool swar_ok(const ConvSep &s)
 {
     if (s.kind != CONV_U8_U8 || s.c.rx < 1 || s.c.rx > 3 || s.shift > 8) return false;
@@ -602,6 +656,16 @@ cudaError_t dispatch_swar_r(const ConvSep &s, cudaStream_t stream)
     return launch_sep<uint8_t, uint8_t, R, SW_ON>(s, stream);
 }
 
+cudaError_t dispatch_swar_i32(const ConvSep &s, cudaStream_t stream)
+{
+    switch (s.c.rx) {
+    case 1: return launch_sep<uint8_t, int32_t, 1, SW_ON | SW_I32>(s, stream);
+    case 2: return launch_sep<uint8_t, int32_t, 2, SW_ON | SW_I32>(s, stream);
+    case 3: return launch_sep<uint8_t, int32_t, 3, SW_ON | SW_I32>(s, stream);
+    default: return cudaErrorNotSupported;
+    }
+}
+
 cudaError_t dispatch_swar(const ConvSep &s, cudaStream_t stream)
 {
     switch (s.c.rx) {
@@ -634,7 +698,8 @@ cudaError_t launch_conv_tiled(const ConvGeneric &p, cudaStream_t stream)
     case CONV_F32: return dispatch_r<float, float>(s, stream);
     case CONV_U8_U8:
         return swar_ok(s) ? dispatch_swar(s, stream) : dispatch_r<uint8_t, uint8_t>(s, stream);
-    case CONV_U8_I32: return dispatch_r<uint8_t, int32_t>(s, stream);
+    case CONV_U8_I32:
+        return swar_i32_prepare(s) ? dispatch_swar_i32(s, stream) : dispatch_r<uint8_t, int32_t>(s, stream);
     default: return cudaErrorNotSupported;
     }
 }

@@ -97,6 +97,9 @@ struct ConvSep {
     int32_t shift;
     float rf[9], cf[9];      // f32 row / column coefficients
     int32_t ri[9], ci[9];    // integer row / column coefficients
+    // signed SWAR (u8 -> i32, conv_tiled.cu): lane biases that keep both 16-bit
+    // lanes of the row sums / column sums in [0, 65535]; S = V - sw_off
+    int32_t sw_bias_h, sw_bias_v, sw_off;
 };
 
 // Fused two-stage local operator (conv_chain.cu): out = M2 (*) (M1 (*) I), both

@@ -823,3 +823,25 @@ def test_sobel_magnitude_4096(lop):
     gx = lop.sobel(img, 0, "clamp").cpu().numpy()
     gy = lop.sobel(img, 1, "clamp").cpu().numpy()
     assert np.array_equal(f, _np_combine(gx, gy, "l2"))
+
+
+@pytest.mark.parametrize("rows,cols,shift", [([-1, 0, 1], [1, 2, 1], 0), ([1, 2, 1], [-1, 0, 1], 0),
+                                             ([1, -4, 6, -4, 1], [-1, 2, -1, 2, -1], 2),
+                                             ([-3, 5, -3], [2, -7, 9, -7, 2], 0),
+                                             ([1, -1, 2, -2, 3, -3, 4], [1, 1, 1, 1, 1, 1, 1], 1)])
+def test_conv_u8_i32_signed_swar(lop, rows, cols, shift, monkeypatch):
+    """u8 -> i32 with signed separable masks on the signed SWAR kernel (lane
+    biases; opt-in LOP_CONV_SWAR_I32=1): bit-exact against the oracle and
+    identical to the default unpacked kernel, every mode, frames, ragged tails."""
+    mi = np.outer(np.array(cols), np.array(rows)).astype(np.int32)
+    u = torch.stack([synthetic.uniform_u8(101, 1037, seed=sum(map(abs, rows)) + s) for s in range(2)])
+    for mode in MODES:
+        monkeypatch.setenv("LOP_CONV_SWAR_I32", "1")
+        q = lop.convolve(u.cuda(), mi, mode, constant=201, shift=shift, out_dtype=torch.int32).cpu()
+        monkeypatch.delenv("LOP_CONV_SWAR_I32")
+        q0 = lop.convolve(u.cuda(), mi, mode, constant=201, shift=shift, out_dtype=torch.int32).cpu()
+        assert torch.equal(q, q0), mode
+        for i in range(2):
+            ref, valid = oracle.convolve_u8(u[i].numpy(), mi, shift, mode, cval=201, out_dtype=np.int32)
+            sel = valid if mode == "undefined" else slice(None)
+            assert (q[i].numpy()[sel] == ref[sel]).all(), (mode, i)
