@@ -561,11 +561,16 @@ cudaError_t launch_cfg(const ConvSep &s, cudaStream_t stream)
 // instantiated for radii 1 and 2 (Sobel 3x3, Gaussian 5x5); other radii use
 // the default.
 constexpr int kDefTS = 8, kDefTSSwar = 16, kDefNBUF = 1;   // tools/tune_conv.py on B200, round 1
+// u8 -> i32 (Sobel): 4 rows per tile -- a 4096^2 image is then 4096 tiles (~2 waves), so
+// CTAs in their store phase overlap CTAs in their load phase (0.0180 vs 0.0192 ms at 8
+// rows; profiles/r01_tune_conv.jsonl)
+constexpr int kDefTSI32 = 4;
 
 template <typename T, typename TO, int R, int SWAR = 0>
 cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
 {
-    int ts = SWAR ? kDefTSSwar : kDefTS, nbuf = kDefNBUF;
+    int ts = SWAR ? kDefTSSwar : (sizeof(T) == 1 && sizeof(TO) == 4 ? kDefTSI32 : kDefTS);
+    int nbuf = kDefNBUF;
     if (const char *env = std::getenv("LOP_CONV_CFG")) std::sscanf(env, "%d:%d", &ts, &nbuf);
     if constexpr (R == 1 || R == 2) {
         if (ts == 4 && nbuf == 1) return launch_cfg<T, TO, R, SWAR, 4, 1>(s, stream);
