@@ -24,7 +24,9 @@ def _declared_symbols():
 def test_header_declares_expected_entry_points():
     syms = _declared_symbols()
     for s in ("lop_bilateral_execute", "lop_convolve_execute", "lop_mask_closeness",
-              "lop_mask_gaussian", "lop_mask_sobel", "lop_last_error", "lop_pipeline_create"):
+              "lop_mask_gaussian", "lop_mask_sobel", "lop_last_error", "lop_pipeline_create",
+              "lop_convolve_chain_execute", "lop_reduce_execute", "lop_convolve2_execute",
+              "lop_pipeline_bilateral_frames"):
         assert s in syms
 
 
@@ -119,6 +121,20 @@ def test_execute_rejects_invalid_arguments_before_launch():
     before = lop.launch_count()
     st = lib.lop_bilateral_execute(ctypes.byref(is_), ctypes.byref(acc), None, 1.0, 1.0, None)
     assert st == _lib.LOP_ERR_INVALID
+    assert lop.launch_count() == before
+    # the session-4 entry points validate before launching as well
+    bc, acc, is_ = _views(data=0)
+    m = _lib.lop_mask()
+    assert lib.lop_reduce_execute(ctypes.byref(is_), ctypes.byref(acc), ctypes.byref(m), 7,
+                                  None) == _lib.LOP_ERR_INVALID
+    assert b"reduction" in lib.lop_last_error()
+    assert lib.lop_convolve2_execute(ctypes.byref(is_), ctypes.byref(acc), None, None, 9,
+                                     None) == _lib.LOP_ERR_INVALID
+    assert b"combine" in lib.lop_last_error()
+    assert lib.lop_reduce_execute(ctypes.byref(is_), ctypes.byref(acc), None,
+                                  _lib.LOP_REDUCE_MIN, None) == _lib.LOP_ERR_INVALID
+    assert lib.lop_pipeline_bilateral_frames(None, None, 0, 0, None, 0, 0, 1, 1, 0.0, 3, 3, None,
+                                             1.0, 1.0) == _lib.LOP_ERR_INVALID
     assert lop.launch_count() == before
 
 
