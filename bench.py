@@ -482,6 +482,14 @@ def conv_extras(lop, synthetic, dev, stream, hbm, img, timed):
                        lop.sobel(f_in[k], 1, "clamp", out=mid_f, stream=s)), 8),
         ("sobel_magnitude_l1_u8_i32_fused",
          lambda k, s: lop.sobel_magnitude(u_in[k], "clamp", out=i_out[k], stream=s), 5)]
+    # global operator (sum of all pixels, deterministic two-level reduction)
+    gres = torch.empty(1, dtype=torch.float64, device=dev)
+    gwork = torch.zeros(1025, dtype=torch.float64, device=dev)     # LOP_GLOBAL_WORK_DOUBLES
+    cases += [
+        ("global_sum_f32", lambda k, s: lop.global_reduce(f_in[k], "sum", out=gres, work=gwork,
+                                                          stream=s), 4),
+        ("global_max_u8", lambda k, s: lop.global_reduce(u_in[k], "max", out=gres, work=gwork,
+                                                         stream=s), 1)]
     res = {}
     H, W = img.shape
     for name, fn, bpp in cases:

@@ -204,6 +204,21 @@ lop_status lop_convolve2_execute(const lop_iteration_space *is, const lop_access
                                  const lop_mask *a, const lop_mask *b, int32_t combine,
                                  void *cuda_stream);
 
+/* Global operator (one output for all pixels, "e.g. the
+ * sum of all pixels"): SUM, MIN or MAX of the pixels of the
+ * region (x0, y0, width, height) of is->image (here the INPUT; width/height 0
+ * = to the image edge), over all frames of a batch.  The result is one double
+ * written to device memory d_result; d_work is a device scratch array of
+ * LOP_GLOBAL_WORK_DOUBLES doubles owned by the caller, ZERO-initialised before
+ * its first use (its last element is an arrival counter that every call leaves
+ * at zero again; calls sharing one d_work must be ordered on one stream).
+ * F32 (sum accumulated in double) or U8 (exact integer sum).  Deterministic:
+ * fixed partition and fixed reduction trees, so the same input gives the same
+ * bits on every run.  Asynchronous on cuda_stream (one kernel launch). */
+#define LOP_GLOBAL_WORK_DOUBLES 1025
+lop_status lop_global_reduce_execute(const lop_iteration_space *is, int32_t op, double *d_result,
+                                     double *d_work, void *cuda_stream);
+
 /* Mask builders (host only).
  * lop_mask_closeness: Eq. (1), float coefficients (Listing 4's mask[]).
  * lop_mask_gaussian:  binomial size x size (size odd; 1..11 for LOP_I32, 1..31

@@ -231,6 +231,29 @@ def convolve2(img, mask_a, mask_b, combine, mode, cval=0.0, rows=None):
     return out, va & vb
 
 
+def global_reduce(img, op, roi=None):
+    """Global operator: one value for all pixels of the
+    region (x0, y0, w, h) of a 2D image or a (B, H, W) stack.  "sum" is the
+    correctly rounded exact sum (math.fsum over the float values; exact integer
+    for u8), "min" / "max" the extreme pixel value."""
+    import math
+    a = np.asarray(img)
+    if a.ndim == 2:
+        a = a[None]
+    if roi is not None:
+        x0, y0, w, h = roi
+        a = a[:, y0:y0 + h, x0:x0 + w]
+    if op == "sum":
+        if a.dtype == np.uint8:
+            return float(int(a.astype(np.int64).sum()))
+        return math.fsum(float(v) for v in a.ravel())
+    if op == "min":
+        return float(min(a.ravel().tolist()))
+    if op == "max":
+        return float(max(a.ravel().tolist()))
+    raise ValueError(op)
+
+
 _REDUCE_OPS = {"min": 1, "max": 2}
 
 

@@ -202,6 +202,26 @@ def reduce(x: torch.Tensor, domain, op="min", mode="clamp", constant=0.0, out=No
                                                                      _REDUCE[op], s))
 
 
+def global_reduce(x: torch.Tensor, op="sum", roi=None, out=None, work=None,
+                  stream=None) -> torch.Tensor:
+    """Global operator: "sum" / "min" / "max" of the pixels
+    of ``roi`` over all frames, as a 1-element float64 CUDA tensor (written
+    asynchronously; deterministic).  ``work``: a reusable zero-initialised
+    float64 scratch tensor of LOP_GLOBAL_WORK_DOUBLES elements."""
+    if out is None:
+        out = torch.empty(1, dtype=torch.float64, device=x.device)
+    if work is None:                         # zero-initialised (its last slot is a counter)
+        work = torch.zeros(_lib.LOP_GLOBAL_WORK_DOUBLES, dtype=torch.float64, device=x.device)
+    is_ = _lib.lop_iteration_space()
+    is_.image = image_view(x)
+    if roi is not None:
+        is_.x0, is_.y0, is_.width, is_.height = (int(v) for v in roi)
+    with torch.cuda.device(x.device):
+        _check(lib.lop_global_reduce_execute(ctypes.byref(is_), _REDUCE[op], out.data_ptr(),
+                                             work.data_ptr(), _stream_handle(x, stream)))
+    return out
+
+
 def erode(x: torch.Tensor, size: int = 3, mode="clamp", constant=0.0, **kw) -> torch.Tensor:
     """Grey-value erosion with a full size x size window (local MIN)."""
     return reduce(x, np.ones((size, size)), "min", mode, constant, **kw)

@@ -18,6 +18,7 @@ LOP_UNDEFINED, LOP_CLAMP, LOP_REPEAT, LOP_MIRROR, LOP_CONSTANT = 0, 1, 2, 3, 4
 LOP_VARIANT_AUTO, LOP_VARIANT_GENERIC, LOP_VARIANT_TILED = 0, 1, 2
 LOP_REDUCE_SUM, LOP_REDUCE_MIN, LOP_REDUCE_MAX = 0, 1, 2
 LOP_COMBINE_L2, LOP_COMBINE_L1, LOP_COMBINE_SUMSQ = 0, 1, 2
+LOP_GLOBAL_WORK_DOUBLES = 1025
 
 c_i32, c_i64, c_dbl, c_flt, c_vp = (ctypes.c_int32, ctypes.c_int64, ctypes.c_double,
                                     ctypes.c_float, ctypes.c_void_p)
@@ -67,6 +68,8 @@ SIGNATURES = {
     "lop_convolve2_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
                                       ctypes.POINTER(lop_accessor), ctypes.POINTER(lop_mask),
                                       ctypes.POINTER(lop_mask), c_i32, c_vp]),
+    "lop_global_reduce_execute": (c_i32, [ctypes.POINTER(lop_iteration_space), c_i32, c_vp,
+                                          c_vp, c_vp]),
     "lop_mask_closeness": (c_i32, [c_flt, c_i32, c_i32, c_vp]),
     "lop_mask_gaussian": (c_i32, [c_i32, c_i32, c_vp, ctypes.POINTER(c_i32)]),
     "lop_mask_sobel": (c_i32, [c_i32, c_i32, c_vp]),

@@ -25,6 +25,8 @@ cudaError_t launch_reduce(const ReduceParams &p, bool allow_tiled, cudaStream_t 
 // launcher returns cudaErrorNotSupported when no instance matches.
 cudaError_t launch_conv_pair(const ConvPair &p, cudaStream_t stream);
 cudaError_t launch_conv_pair_generic(const ConvPairGeneric &p, cudaStream_t stream);
+// Global SUM / MIN / MAX (global_reduce.cu): two launches (parts, final).
+cudaError_t launch_global_reduce(const GlobalReduce &p, cudaStream_t stream);
 // Fused two-stage convolution; cudaErrorNotSupported if no instance matches.
 cudaError_t launch_conv_chain(const ConvChain &p, cudaStream_t stream);
 

@@ -505,6 +505,48 @@ lop_status lop_reduce_execute(const lop_iteration_space *is, const lop_accessor 
                     "reduce launch");
 }
 
+// ------------------------------------------------------- global operators
+lop_status lop_global_reduce_execute(const lop_iteration_space *is, int32_t op, double *d_result,
+                                     double *d_work, void *cuda_stream)
+{
+    static_assert(lop::kGlobalParts + 1 == LOP_GLOBAL_WORK_DOUBLES, "work size");
+    if (!is) return fail(LOP_ERR_INVALID, "iteration space is NULL");
+    if (op != LOP_REDUCE_SUM && op != LOP_REDUCE_MIN && op != LOP_REDUCE_MAX)
+        return fail(LOP_ERR_INVALID, "unknown reduction %d (SUM, MIN, MAX)", op);
+    if (!d_result || !d_work) return fail(LOP_ERR_INVALID, "d_result / d_work is NULL");
+    lop_status st = check_image(is->image, "image");
+    if (st) return st;
+    const lop_image &im = is->image;
+    if (im.dtype != LOP_F32 && im.dtype != LOP_U8)
+        return fail(LOP_ERR_INVALID, "global reductions take F32 or U8 images");
+    for (const void *ptr : {static_cast<const void *>(d_result), static_cast<const void *>(d_work)}) {
+        cudaPointerAttributes attr;
+        if (cudaPointerGetAttributes(&attr, ptr) != cudaSuccess ||
+            (attr.type != cudaMemoryTypeDevice && attr.type != cudaMemoryTypeManaged)) {
+            cudaGetLastError();
+            return fail(LOP_ERR_INVALID, "d_result / d_work must be device memory");
+        }
+    }
+    static thread_local lop::GlobalReduce p;
+    std::memset(&p.c, 0, sizeof p.c);
+    p.c.in = make_geom(im);
+    p.c.roi_x0 = is->x0;
+    p.c.roi_y0 = is->y0;
+    p.c.roi_w = is->width ? is->width : im.width - is->x0;
+    p.c.roi_h = is->height ? is->height : im.height - is->y0;
+    if (p.c.roi_x0 < 0 || p.c.roi_y0 < 0 || p.c.roi_w <= 0 || p.c.roi_h <= 0 ||
+        (int64_t)p.c.roi_x0 + p.c.roi_w > im.width || (int64_t)p.c.roi_y0 + p.c.roi_h > im.height)
+        return fail(LOP_ERR_INVALID, "region [%d,%d)+%dx%d outside the %d x %d image", is->x0,
+                    is->y0, p.c.roi_w, p.c.roi_h, im.width, im.height);
+    p.c.batch = im.batch;
+    p.op = op == LOP_REDUCE_SUM ? lop::RED_SUM : (op == LOP_REDUCE_MIN ? lop::RED_MIN : lop::RED_MAX);
+    p.u8 = im.dtype == LOP_U8;
+    p.work = d_work;
+    p.result = d_result;
+    cudaError_t e = lop::launch_global_reduce(p, static_cast<cudaStream_t>(cuda_stream));
+    return launched(e, "global reduce launch");
+}
+
 // -------------------------------- two local operators + point-operator epilogue
 lop_status lop_convolve2_execute(const lop_iteration_space *is, const lop_accessor *in,
                                  const lop_mask *a, const lop_mask *b, int32_t combine,

@@ -109,13 +109,24 @@ struct ConvSep {
 // Local reduction over a mask domain (Listing 9's convolve(mask, <reduction>, f)
 // with the MIN / MAX reductions; reduce.cu): out = min / max of Read(x+xf, y+yf)
 // over the taps where the mask is non-zero.  dom[yf + ry] bit (xf + rx) = tap.
-enum ReduceOp { RED_MIN = 1, RED_MAX = 2 };
+enum ReduceOp { RED_SUM = 0, RED_MIN = 1, RED_MAX = 2 };
 struct ReduceParams {
     Common c;
     int32_t op;                      // RED_MIN / RED_MAX
     int32_t u8;                      // 1: u8 -> u8, 0: f32 -> f32
     int32_t full;                    // domain is the whole window (separable)
     uint64_t dom[2 * kMaxRadius + 1];
+};
+
+// Global operator (global_reduce.cu): SUM / MIN / MAX over a region of all
+// frames, deterministic (fixed parts, fixed trees), result in double.
+constexpr int kGlobalParts = 1024;                            // + 1 counter = LOP_GLOBAL_WORK_DOUBLES
+struct GlobalReduce {
+    Common c;                    // c.in: the image; c.roi_*: the region; c.batch
+    int32_t op;                  // RED_SUM / RED_MIN / RED_MAX
+    int32_t u8;
+    double *work;                // kGlobalParts doubles + an arrival counter (device)
+    double *result;              // 1 double (device)
 };
 
 // Two local operators on one input, combined by a point operator (conv_pair.cu):

@@ -506,3 +506,35 @@ def test_convolve2_transpose_symmetry():
         m, _ = oracle.convolve2(img, sx, sy, "l2", mode)
         mt, _ = oracle.convolve2(np.ascontiguousarray(img.T), sx, sy, "l2", mode)
         np.testing.assert_allclose(mt, m.T, rtol=0, atol=1e-12)
+
+
+# ------------------------------------------------- global operators (N3) ----
+
+def test_global_reduce_closed_forms():
+    """Sum of a constant image = v N exactly; sum of an integer ramp = the
+    arithmetic-series closed form; min / max of a ramp = its end values;
+    a region and a stack of frames reduce the selected pixels only."""
+    flat = np.full((37, 53), 0.375, np.float32)
+    assert oracle.global_reduce(flat, "sum") == 0.375 * 37 * 53
+    ys, xs = np.mgrid[0:40, 0:50]
+    ramp = (xs + 50 * ys).astype(np.float32)                 # 0 .. 1999, each once
+    assert oracle.global_reduce(ramp, "sum") == 1999 * 2000 / 2
+    assert oracle.global_reduce(ramp, "min") == 0 and oracle.global_reduce(ramp, "max") == 1999
+    # region rows 10..19, columns 5..14: sum of x + 50 y over the block
+    exp = sum(x + 50 * y for y in range(10, 20) for x in range(5, 15))
+    assert oracle.global_reduce(ramp, "sum", roi=(5, 10, 10, 10)) == exp
+    u8 = (np.arange(3 * 16 * 16) % 256).astype(np.uint8).reshape(3, 16, 16)
+    assert oracle.global_reduce(u8, "sum") == 3 * 255 * 256 / 2
+    assert oracle.global_reduce(u8, "max") == 255
+
+
+def test_global_reduce_matches_numpy_and_is_exact():
+    """min / max agree with np.min / np.max; the f32 sum is the exact sum
+    (fractions.Fraction) correctly rounded to double."""
+    from fractions import Fraction
+    rng = _rng(31)
+    img = rng.random((29, 31)).astype(np.float32)
+    assert oracle.global_reduce(img, "min") == float(img.min())
+    assert oracle.global_reduce(img, "max") == float(img.max())
+    exact = sum(Fraction(float(v)) for v in img.ravel())
+    assert oracle.global_reduce(img, "sum") == float(exact)

@@ -845,3 +845,37 @@ def test_conv_u8_i32_signed_swar(lop, rows, cols, shift, monkeypatch):
             ref, valid = oracle.convolve_u8(u[i].numpy(), mi, shift, mode, cval=201, out_dtype=np.int32)
             sel = valid if mode == "undefined" else slice(None)
             assert (q[i].numpy()[sel] == ref[sel]).all(), (mode, i)
+
+
+# ------------------------------------------------- global operators (N3) ----
+
+@pytest.mark.parametrize("shape", [(1, 1), (7, 5), (130, 1031), (1024, 2048)])
+def test_global_reduce(lop, shape):
+    """SUM / MIN / MAX of all pixels: u8 exact, f32 MIN / MAX exact and SUM
+    within 1e-12 relative of the exact sum (double accumulation); the same input
+    gives the same bits twice (fixed partition and trees); regions and frames."""
+    H, W = shape
+    img = synthetic.uniform(H, W, seed=H + W)
+    u8 = synthetic.uniform_u8(H, W, seed=H * W + 1)
+    for op in ("sum", "min", "max"):
+        g = lop.global_reduce(img.cuda(), op).item()
+        ref = oracle.global_reduce(img.numpy(), op)
+        if op == "sum":
+            assert abs(g - ref) <= 1e-12 * max(1.0, abs(ref)), (g, ref)
+            assert lop.global_reduce(img.cuda(), op).item() == g          # deterministic
+        else:
+            assert g == ref
+        assert lop.global_reduce(u8.cuda(), op).item() == oracle.global_reduce(u8.numpy(), op)
+    if H > 10 and W > 10:
+        roi = (3, 5, W - 7, H - 9)
+        frames = torch.stack([img, img * 0.5, img + 0.25]).cuda()
+        for op in ("sum", "min", "max"):
+            g = lop.global_reduce(frames, op, roi=roi).item()
+            ref = oracle.global_reduce(frames.cpu().numpy(), op, roi=roi)
+            assert abs(g - ref) <= 1e-12 * max(1.0, abs(ref)), (op, g, ref)
+    # one scratch buffer reused by many calls: its arrival counter returns to zero
+    work = torch.zeros(1025, dtype=torch.float64, device="cuda")
+    vals = [lop.global_reduce(img.cuda(), op, work=work).item() for op in ("max", "sum", "min") * 3]
+    assert vals[:3] * 3 == vals and work[-1].item() == 0.0
+    with pytest.raises(lop.LopError):
+        lop.global_reduce(img.cuda(), "sum", roi=(0, 0, W + 1, H))
