@@ -336,10 +336,41 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
         for (int xf = -c.rx; xf <= c.rx; ++xf) lx[xf + c.rx] = (float)(-c_d * (double)(xf * xf) * kLog2e);
         for (int yf = -c.ry; yf <= c.ry; ++yf) cy[yf + c.ry] = (float)std::exp(-c_d * (double)(yf * yf));
     }
+    // A user closeness mask (Listing 4 / 5) that factors into x and y factors --
+    // the paper's own mask exp(-c (xf^2 + yf^2)) does -- takes the separable
+    // kernels (and the pair-sharing one): cy[i] = M[i][m], cx[j] = M[n][j] / M[n][m],
+    // accepted when every coefficient is > 0, both factors are exactly
+    // symmetric (pair sharing needs c(d) = c(-d) bit for bit) and cy[i] cx[j]
+    // reproduces M to 2^-20 relative (reading c21).  LOP_BILATERAL_FACTOR=0 keeps
+    // the mask kernels.
+    bool sepform = !closeness;
+    if (closeness) {
+        bool ok = true;
+        if (const char *env = std::getenv("LOP_BILATERAL_FACTOR")) ok = std::atoi(env) != 0;
+        const float *cm = static_cast<const float *>(closeness->coeffs);
+        for (int i = 0; i < sx * sy && ok; ++i) ok = cm[i] > 0;
+        if (ok) {
+            const double centre = cm[c.ry * sx + c.rx];
+            double cxd[2 * lop::kMaxRadius + 1], cyd[2 * lop::kMaxRadius + 1];
+            for (int j = 0; j < sx; ++j) cxd[j] = (double)cm[c.ry * sx + j] / centre;
+            for (int i = 0; i < sy; ++i) cyd[i] = (double)cm[i * sx + c.rx];
+            for (int j = 0; j < sx && ok; ++j) ok = cxd[j] == cxd[sx - 1 - j];
+            for (int i = 0; i < sy && ok; ++i) ok = cyd[i] == cyd[sy - 1 - i];
+            for (int i = 0; i < sy && ok; ++i)
+                for (int j = 0; j < sx && ok; ++j)
+                    ok = std::fabs(cyd[i] * cxd[j] - (double)cm[i * sx + j]) <=
+                         std::ldexp((double)cm[i * sx + j], -20);
+            if (ok) {
+                for (int j = 0; j < sx; ++j) lx[j] = (float)std::log2(cxd[j]);
+                for (int i = 0; i < sy; ++i) cy[i] = (float)cyd[i];
+                sepform = true;
+            }
+        }
+    }
     // window columns whose exp runs on the FMA pipe (ex2_poly) instead of the
     // MUFU: tuned on B200; LOP_BILATERAL_NPOLY overrides
     int npoly = 0;
-    if (!closeness) {
+    if (sepform) {
         npoly = c.rx >= 4 ? kDefaultNpoly : 0;
         if (const char *env = std::getenv("LOP_BILATERAL_NPOLY")) npoly = std::atoi(env);
         npoly = std::max(0, std::min(npoly, lop::bilateral_sep_max_npoly(c.rx)));
@@ -352,10 +383,10 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
     // exponent; LOP_BILATERAL_PAIR overrides
     int pair = kDefaultPair;
     if (const char *env = std::getenv("LOP_BILATERAL_PAIR")) pair = std::atoi(env) != 0;
-    pair = pair && !closeness && scaled && c.rx == c.ry && c.rx >= 1 && c.rx <= lop::kTiledMaxRX;
+    pair = pair && sepform && scaled && c.rx == c.ry && c.rx >= 1 && c.rx <= lop::kTiledMaxRX;
     const double alpha_d = std::sqrt(kLog2e / (2.0 * (double)sigma_r * (double)sigma_r));
     const float alpha = (float)alpha_d, inv_alpha = (float)(1.0 / alpha_d);
-    if (variant != LOP_VARIANT_GENERIC && tiled_ok && !closeness) {
+    if (variant != LOP_VARIANT_GENERIC && tiled_ok && sepform) {
         static thread_local lop::BilateralSep p;
         p.c = c;
         p.nk = nk;
@@ -385,13 +416,13 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
     static thread_local lop::BilateralGeneric p;
     p.c = c;
     p.nk = nk;
-    p.sep = closeness ? 0 : 1;
+    p.sep = sepform ? 1 : 0;
     p.pair = pair;
     p.npoly = npoly;
     p.scaled = scaled;
     p.alpha = alpha;
     p.inv_alpha = inv_alpha;
-    if (closeness) {
+    if (!sepform) {
         std::memcpy(p.lc, lc.get(), sizeof(float) * sx * sy);
     } else {
         std::memcpy(p.lx, lx, sizeof(float) * sx);

@@ -879,3 +879,35 @@ def test_global_reduce(lop, shape):
     assert vals[:3] * 3 == vals and work[-1].item() == 0.0
     with pytest.raises(lop.LopError):
         lop.global_reduce(img.cuda(), "sum", roi=(0, 0, W + 1, H))
+
+
+@pytest.mark.parametrize("size", [3, 9, 13, (13, 7)])
+def test_bilateral_factored_user_mask(lop, size, monkeypatch):
+    """Listing 4's precomputed closeness mask passed explicitly (the paper's own
+    flow) factors into symmetric x / y factors and takes the separable / pair
+    kernels: within tolerance of the oracle on that mask, generic == tiled bit
+    for bit, and within tolerance of the unfactored mask kernel."""
+    sx, sy = (size, size) if isinstance(size, int) else size
+    cm = lop.closeness_mask(3.0, sx, sy)
+    img = synthetic.angio(120, 333, seed=23)
+    for mode in MODES:
+        lop.set_variant("generic")
+        a = lop.bilateral(img.cuda(), 0.0, 0.1, mode, constant=0.5, mask=cm)
+        lop.set_variant("tiled")
+        b = lop.bilateral(img.cuda(), 0.0, 0.1, mode, constant=0.5, mask=cm)
+        lop.set_variant("auto")
+        assert torch.equal(a, b), mode
+        ref, valid = oracle.bilateral_f32(img.numpy(), 0.0, 0.1, mode, cval=0.5,
+                                          cmask=cm.astype(np.float64))
+        sel = valid if mode == "undefined" else None
+        _cmp_float(b.cpu().numpy(), ref, sel)
+        monkeypatch.setenv("LOP_BILATERAL_FACTOR", "0")
+        c = lop.bilateral(img.cuda(), 0.0, 0.1, mode, constant=0.5, mask=cm)
+        monkeypatch.delenv("LOP_BILATERAL_FACTOR")
+        _cmp_float(b.cpu().numpy(), c.cpu().numpy().astype(np.float64), sel)
+    # an asymmetric or non-separable mask keeps the mask kernels (still correct)
+    cm2 = cm.copy()
+    cm2[0, 0] *= 1.5
+    out = lop.bilateral(img.cuda(), 0.0, 0.1, "clamp", mask=cm2)
+    ref, _ = oracle.bilateral_f32(img.numpy(), 0.0, 0.1, "clamp", cmask=cm2.astype(np.float64))
+    _cmp_float(out.cpu().numpy(), ref)
