@@ -679,11 +679,16 @@ __device__ __forceinline__ void pair_put_row(const Common &c, int iy, int ix0, f
         q.x = __fmul_rn(q.x, alpha); q.y = __fmul_rn(q.y, alpha);
         q.z = __fmul_rn(q.z, alpha); q.w = __fmul_rn(q.w, alpha);
         plain[k] = q;
+        // interleaved slot, swizzled: float4 i of a slot lives at i ^ ((i >> 3) & 1),
+        // so the LDS.128 of 8 lanes reading float4 2L + k (2 x 16 B apart) hit 8
+        // distinct 16-B bank groups (no 2-way conflict); columns 4k..4k+3 are
+        // float4 2k, 2k+1, swapped when bit 3 of 2k (= bit 2 of k) is set
+        const int a = ((k >> 2) & 1) ? 4 : 0, a2 = 4 - a;
         float *f = reinterpret_cast<float *>(first + 4 * k);
-        f[0] = q.x; f[2] = q.y; f[4] = q.z; f[6] = q.w;
+        f[a + 0] = q.x; f[a + 2] = q.y; f[a2 + 0] = q.z; f[a2 + 2] = q.w;
         if (second) {
             float *sc = reinterpret_cast<float *>(second + 4 * k) + 1;
-            sc[0] = q.x; sc[2] = q.y; sc[4] = q.z; sc[6] = q.w;
+            sc[a + 0] = q.x; sc[a + 2] = q.y; sc[a2 + 0] = q.z; sc[a2 + 2] = q.w;
         }
     }
 }
@@ -758,10 +763,11 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
             const int sl = slot0 + dy >= NR ? slot0 + dy - NR : slot0 + dy;
             float2 v[4 * NV];
             {
-                const float4 *src = reinterpret_cast<const float4 *>(ring2 + sl * SW) + 2 * lane;
+                const float4 *src = reinterpret_cast<const float4 *>(ring2 + sl * SW);
 #pragma unroll
                 for (int k = 0; k < 2 * NV; ++k) {
-                    const float4 q = src[k];
+                    const int i = 2 * lane + k;                          // swizzled (pair_put_row)
+                    const float4 q = src[i ^ ((i >> 3) & 1)];
                     v[2 * k] = make_float2(q.x, q.y);
                     v[2 * k + 1] = make_float2(q.z, q.w);
                 }
