@@ -19,6 +19,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <cstdlib>
+
 #include "boundary.cuh"
 #include "kernels.h"
 #include "lop_params.h"
@@ -28,12 +30,12 @@ namespace lop {
 
 namespace red {
 constexpr int NT = 128;
-template <typename T> struct Shape {
+template <typename T, int TS_ = (sizeof(T) == 4 ? 8 : 16)> struct Shape {
     static constexpr int PX = sizeof(T) == 4 ? 4 : 8;        // columns per thread
     static constexpr int TWE = NT * PX;                      // tile width (elements)
     static constexpr int PADE = 16 / (int)sizeof(T);         // 16-B pad each side (>= R)
     static constexpr int SWE = TWE + 2 * PADE;               // smem row pitch
-    static constexpr int TS = sizeof(T) == 4 ? 8 : 16;       // output rows per tile
+    static constexpr int TS = TS_;                           // output rows per tile
 };
 }  // namespace red
 
@@ -60,10 +62,10 @@ template <int OP, int N> __device__ __forceinline__ uint32_t red_n(const uint32_
     return m;
 }
 
-template <typename T, int OP, int R>
+template <typename T, int OP, int R, int TS_>
 __global__ void __launch_bounds__(red::NT) reduce_tiled_kernel(const __grid_constant__ ReduceParams p)
 {
-    using S = red::Shape<T>;
+    using S = red::Shape<T, TS_>;
     constexpr int PX = S::PX, SWE = S::SWE, PADE = S::PADE, TS = S::TS, P = 2 * R + 1;
     static_assert(R >= 1 && R <= 4, "halo must fit the 16-B pad");
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -218,21 +220,32 @@ __global__ void __launch_bounds__(256) reduce_generic_kernel(const __grid_consta
 
 namespace {
 
-template <typename T, int OP, int R>
-cudaError_t launch_tiled_r(const ReduceParams &p, cudaStream_t stream)
+template <typename T, int OP, int R, int TS>
+cudaError_t launch_tiled_ts(const ReduceParams &p, cudaStream_t stream)
 {
-    using S = red::Shape<T>;
+    using S = red::Shape<T, TS>;
     const size_t smem = (size_t)(S::TS + 2 * R) * S::SWE * sizeof(T);
     static bool configured = false;
     if (!configured && smem > 48 * 1024) {
-        cudaError_t e = cudaFuncSetAttribute(reduce_tiled_kernel<T, OP, R>,
+        cudaError_t e = cudaFuncSetAttribute(reduce_tiled_kernel<T, OP, R, TS>,
                                              cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         if (e != cudaSuccess) return e;
         configured = true;
     }
     dim3 grid((p.c.roi_w + S::TWE - 1) / S::TWE, (p.c.roi_h + S::TS - 1) / S::TS, p.c.batch);
-    reduce_tiled_kernel<T, OP, R><<<grid, red::NT, smem, stream>>>(p);
+    reduce_tiled_kernel<T, OP, R, TS><<<grid, red::NT, smem, stream>>>(p);
     return cudaGetLastError();
+}
+
+// output rows per tile: default f32 8, u8 16; LOP_REDUCE_TS (4 / 8 / 16) overrides
+template <typename T, int OP, int R>
+cudaError_t launch_tiled_r(const ReduceParams &p, cudaStream_t stream)
+{
+    int ts = sizeof(T) == 4 ? 8 : 16;
+    if (const char *env = std::getenv("LOP_REDUCE_TS")) ts = std::atoi(env);
+    if (ts == 4) return launch_tiled_ts<T, OP, R, 4>(p, stream);
+    if (ts == 16) return launch_tiled_ts<T, OP, R, 16>(p, stream);
+    return launch_tiled_ts<T, OP, R, 8>(p, stream);
 }
 
 template <typename T, int OP>

@@ -699,6 +699,23 @@ def test_reduce_4096_full_bit_exact(lop, mode):
     assert np.array_equal(f.astype(np.float64), ref)
 
 
+@pytest.mark.parametrize("ts", ["4", "8", "16"])
+def test_reduce_tile_rows(lop, ts, monkeypatch):
+    """Every tile height of the MIN / MAX kernel (LOP_REDUCE_TS) gives the
+    oracle's bits: multi-tile frames with ragged tails, both types."""
+    monkeypatch.setenv("LOP_REDUCE_TS", ts)
+    u = torch.stack([synthetic.uniform_u8(203, 1037, seed=s + 60) for s in range(2)]).cuda()
+    f = torch.stack([synthetic.uniform(203, 1037, seed=s + 61) for s in range(2)]).cuda()
+    for mode in ("clamp", "repeat", "constant"):
+        q = lop.erode(u, 5, mode, constant=3).cpu().numpy()
+        d = lop.dilate(f, 3, mode, constant=0.5).cpu().numpy()
+        for i in range(2):
+            refq, _ = oracle.reduce(u[i].cpu().numpy(), np.ones((5, 5)), "min", mode, 3)
+            assert np.array_equal(q[i].astype(np.int64), refq), (mode, i)
+            ref, _ = oracle.reduce(f[i].cpu().numpy(), np.ones((3, 3)), "max", mode, 0.5)
+            assert np.array_equal(d[i].astype(np.float64), ref), (mode, i)
+
+
 def test_reduce_roi_offset_frames_and_validation(lop):
     frames = torch.stack([synthetic.uniform_u8(70, 1100, seed=s) for s in range(3)]).cuda()
     full = lop.erode(frames, 5, "mirror")
