@@ -69,7 +69,11 @@ template <typename T> struct TileShape {
 // so that the final value of each 16-bit lane lies in [0, 65535] -- the 32-bit
 // arithmetic is modular, so borrows between lanes in intermediate steps cancel
 // once the final low lane is in range -- and S = lane - sw_off exactly.
-enum { SW_ON = 1, SW_SYM = 2, SW_SH8 = 4, SW_I32 = 8 };
+// SW_BIN5 -- both factors are the binomial [1 4 6 4 1] (the 5x5 Gaussian):
+// the coefficients are compile-time constants (the paper's outlook, L946-L950:
+// "propagate the constants of the filter masks"), so a sum is
+// (a + e) + 4 (b + d) + 6 c -- two adds, a shift-add and one IMAD.
+enum { SW_ON = 1, SW_SYM = 2, SW_SH8 = 4, SW_I32 = 8, SW_BIN5 = 16 };
 
 template <int R, int TS, int MODE>
 __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tcol, int srows,
@@ -79,6 +83,8 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
     constexpr int SWE = TileShape<uint8_t>::SWE;
     constexpr uint32_t M = 0x00FF00FFu;
     constexpr bool SYM = (MODE & SW_SYM) != 0, SH8 = (MODE & SW_SH8) != 0, I32 = (MODE & SW_I32) != 0;
+    constexpr bool BIN5 = (MODE & SW_BIN5) != 0;
+    static_assert(!BIN5 || (R == 2 && SYM && SH8), "binomial 5x5 constants");
     static_assert(R <= 3, "SWAR sources cover bytes -4..11");
     const uint32_t rnd = I32 ? (uint32_t)p.sw_bias_v * 0x00010001u
                              : (p.shift > 0 ? (1u << (p.shift - 1)) * 0x00010001u : 0u);
@@ -111,7 +117,10 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
 #pragma unroll
         for (int jj = 0; jj < 4; ++jj) {
             uint32_t s;
-            if constexpr (SYM) {
+            if constexpr (BIN5) {
+                const uint32_t *x = S + J[jj];
+                s = (x[0] + x[4]) + ((x[1] + x[3]) << 2) + 6u * x[2];
+            } else if constexpr (SYM) {
                 s = (uint32_t)p.ri[R] * S[J[jj] + R];
 #pragma unroll
                 for (int t = 0; t < R; ++t) s += (uint32_t)p.ri[t] * (S[J[jj] + t] + S[J[jj] + 2 * R - t]);
@@ -128,7 +137,11 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
 #pragma unroll
         for (int jj = 0; jj < 4; ++jj) {
             uint32_t s;
-            if constexpr (SYM) {
+            if constexpr (BIN5) {
+                const uint32_t h0 = h[o % 5][jj], h1 = h[(o + 1) % 5][jj], h2 = h[(o + 2) % 5][jj],
+                               h3 = h[(o + 3) % 5][jj], h4 = h[(o + 4) % 5][jj];
+                s = (h0 + h4 + rnd) + ((h1 + h3) << 2) + 6u * h2;
+            } else if constexpr (SYM) {
                 s = (uint32_t)p.ci[R] * h[(o + R) % (2 * R + 1)][jj] + rnd;    // rounding folded in
 #pragma unroll
                 for (int t = 0; t < R; ++t)
@@ -650,13 +663,24 @@ int swar_mode(const ConvSep &s)
     const int n = 2 * s.c.rx;
     bool sym = true;
     for (int t = 0; t <= n; ++t) sym = sym && s.ri[t] == s.ri[n - t] && s.ci[t] == s.ci[n - t];
-    return sym && s.shift == 8 ? (SW_ON | SW_SYM | SW_SH8) : SW_ON;
+    if (!(sym && s.shift == 8)) return SW_ON;
+    bool bin5 = s.c.rx == 2;
+    const int b5[5] = {1, 4, 6, 4, 1};
+    for (int t = 0; t < 5 && bin5; ++t) bin5 = s.ri[t] == b5[t] && s.ci[t] == b5[t];
+    if (const char *env = std::getenv("LOP_CONV_SWAR"))
+        if (std::atoi(env) == 7) bin5 = false;                      // runtime-coefficient variant
+    return bin5 ? (SW_ON | SW_SYM | SW_SH8 | SW_BIN5) : (SW_ON | SW_SYM | SW_SH8);
 }
 
 template <int R>
 cudaError_t dispatch_swar_r(const ConvSep &s, cudaStream_t stream)
 {
-    if (swar_mode(s) == (SW_ON | SW_SYM | SW_SH8))
+    const int mode = swar_mode(s);
+    if constexpr (R == 2) {
+        if (mode == (SW_ON | SW_SYM | SW_SH8 | SW_BIN5))
+            return launch_sep<uint8_t, uint8_t, R, SW_ON | SW_SYM | SW_SH8 | SW_BIN5>(s, stream);
+    }
+    if (mode & SW_SH8)
         return launch_sep<uint8_t, uint8_t, R, SW_ON | SW_SYM | SW_SH8>(s, stream);
     return launch_sep<uint8_t, uint8_t, R, SW_ON>(s, stream);
 }

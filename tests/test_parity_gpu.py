@@ -317,10 +317,11 @@ def test_conv_u8_swar_masks(lop, conv_variant, rows, cols, shift):
         assert (q[sel] == refq[sel]).all(), mode
 
 
-@pytest.mark.parametrize("swar", ["1", "auto"])
+@pytest.mark.parametrize("swar", ["1", "7", "auto"])
 @pytest.mark.parametrize("size", [3, 5])
 def test_conv_u8_swar_variants_bit_identical(lop, swar, size, monkeypatch):
-    """The SWAR variants (plain: LOP_CONV_SWAR=1; palindromic / shift-8: auto)
+    """The SWAR variants (plain: LOP_CONV_SWAR=1; palindromic / shift-8 with
+    runtime coefficients: 7; auto = compile-time binomial constants for the 5x5)
     give the oracle's bits on multi-tile images with ragged tails and frames."""
     if swar != "auto":
         monkeypatch.setenv("LOP_CONV_SWAR", swar)
