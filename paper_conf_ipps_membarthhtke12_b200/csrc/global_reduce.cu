@@ -7,7 +7,7 @@
 // Deterministic: a fixed number of CTAs (kGlobalParts, independent of the GPU)
 // each reduce a fixed contiguous block of rows -- every thread a fixed set of
 // columns, in a fixed order, accumulating in double (f32) or int64 (u8 SUM) --
-// then a fixed tree in shared memory; the last CTA to finish combines the
+// then a fixed tree (warp butterflies, then the warp sums); the last CTA to finish combines the
 // parts in a fixed tree.  The same input always gives the same bits.
 // Bound: HBM (the image is read once).
 #include <cuda_runtime.h>
@@ -27,8 +27,25 @@ template <int OP> __device__ __forceinline__ double comb(double a, double b)
     return OP == RED_MIN ? fmin(a, b) : (OP == RED_MAX ? fmax(a, b) : a + b);
 }
 
+// A ragged or unaligned column group: its n < V (or misaligned) elements
+// loaded one by one into the identity-padded group `q` (kept out of line).
+template <typename T>
+__device__ __noinline__ uint4 glob_partial_group(const T *src, int n, uint4 q)
+{
+    uint32_t w[4] = {q.x, q.y, q.z, q.w};
+    for (int j = 0; j < n; ++j) {
+        if constexpr (sizeof(T) == 4) {
+            w[j] = __float_as_uint(__ldg(src + j));
+        } else {
+            const int k = j >> 2, s = 8 * (j & 3);
+            w[k] = (w[k] & ~(0xFFu << s)) | ((uint32_t)__ldg(src + j) << s);
+        }
+    }
+    return make_uint4(w[0], w[1], w[2], w[3]);
+}
+
 // CTA c reduces rows [c * R / P, (c + 1) * R / P) of the R = batch * roi_h
-// region rows; thread t the 16-byte column groups t, t + NT, ... of each row.
+// region rows; thread t the items t, t + NT, ... of its (row, 16-byte column group) list.
 template <typename T, int OP>
 __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_constant__ GlobalReduce p)
 {
@@ -56,28 +73,60 @@ __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_c
         else facc = OP == RED_MIN ? fminf(facc, v) : fmaxf(facc, v);
     };
     constexpr int V = 16 / (int)sizeof(T);                       // elements per 16-B load
-#pragma unroll 2
-    for (int64_t r = r0; r < r1; ++r) {
-        const int b = (int)(r / c.roi_h), y = c.roi_y0 + (int)(r - (int64_t)b * c.roi_h);
-        const T *row = reinterpret_cast<const T *>(c.in.data + (int64_t)b * c.in.bstride +
-                                                   (int64_t)y * c.in.stride) + c.roi_x0;
-        const bool vec = (reinterpret_cast<uintptr_t>(row) % 16) == 0;               // row-uniform
-#pragma unroll 4
-        for (int x = V * threadIdx.x; x < c.roi_w; x += V * glob::NT) {
-            const int n = min(V, c.roi_w - x);
-            if (vec && n == V) {                                 // one 16-B load, in column order
-                const uint4 q = __ldg(reinterpret_cast<const uint4 *>(row + x));
-                if constexpr (F) {
-                    add_f(__uint_as_float(q.x)); add_f(__uint_as_float(q.y));
-                    add_f(__uint_as_float(q.z)); add_f(__uint_as_float(q.w));
+    // The CTA's rows form (row, column group) items in row-major order; thread t
+    // takes items t, t + NT, ... in that order.  U items are fetched before any
+    // is accumulated (U independent 16-B loads in flight per thread: the first
+    // version read one row at a time and stalled on memory latency).  The item
+    // -> (frame, row, group) walk is incremental: one division per thread.
+    const int G = max((c.roi_w + V - 1) / V, 1);                 // column groups per row
+    const int dr = glob::NT / G, dg = glob::NT % G;
+    int64_t r = c.roi_w > 0 ? r0 + threadIdx.x / G : r1;         // empty region: no items
+    int g = (int)(threadIdx.x % G);
+    const int64_t rr = r < r1 ? r : 0;
+    int b = c.roi_h > 0 ? (int)(rr / c.roi_h) : 0, y = (int)(rr - (int64_t)b * c.roi_h);
+    auto row_at = [&](int bb, int yy) {
+        return c.in.data + (int64_t)bb * c.in.bstride + (int64_t)(c.roi_y0 + yy) * c.in.stride +
+               (int64_t)c.roi_x0 * (int64_t)sizeof(T);
+    };
+    const char *rowp = row_at(b, y);
+    // Identity element of the operator (partial groups are padded with it).
+    const float fid = OP == RED_SUM ? 0.0f : (OP == RED_MIN ? __int_as_float(0x7f800000)
+                                                           : -__int_as_float(0x7f800000));
+    const uint32_t bid = OP == RED_MIN ? 0xFFFFFFFFu : 0u;
+    const uint32_t idw = F ? __float_as_uint(fid) : bid;
+    constexpr int U = 8;
+    while (r < r1) {
+        uint4 q[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            q[u] = make_uint4(idw, idw, idw, idw);
+            if (r < r1) {
+                const int x = g * V;
+                const char *src = rowp + (int64_t)x * (int64_t)sizeof(T);
+                if (x + V <= c.roi_w && (reinterpret_cast<uintptr_t>(src) % 16) == 0)
+                    q[u] = __ldg(reinterpret_cast<const uint4 *>(src));
+                else                                              // ragged / unaligned
+                    q[u] = glob_partial_group<T>(reinterpret_cast<const T *>(src),
+                                                 min(V, c.roi_w - x), q[u]);
+                g += dg;
+                int adv = dr;
+                if (g >= G) { g -= G; ++adv; }
+                r += adv; y += adv;
+                if (y < c.roi_h) {
+                    rowp += (int64_t)adv * c.in.stride;
                 } else {
-                    add_word(q.x, 4); add_word(q.y, 4); add_word(q.z, 4); add_word(q.w, 4);
+                    while (y >= c.roi_h) { y -= c.roi_h; ++b; }
+                    rowp = row_at(b, y);
                 }
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {                             // in item and column order
+            if constexpr (F) {
+                add_f(__uint_as_float(q[u].x)); add_f(__uint_as_float(q[u].y));
+                add_f(__uint_as_float(q[u].z)); add_f(__uint_as_float(q[u].w));
             } else {
-                for (int j = 0; j < n; ++j) {
-                    if constexpr (F) add_f(__ldg(row + x + j));
-                    else add_word((uint32_t)__ldg(row + x + j), 1);
-                }
+                add_word(q[u].x, 4); add_word(q[u].y, 4); add_word(q[u].z, 4); add_word(q[u].w, 4);
             }
         }
     }
@@ -93,22 +142,28 @@ __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_c
         }
         acc = (double)m;
     }
-    __shared__ double sh[glob::NT];
-    sh[threadIdx.x] = acc;
-    __syncthreads();
+    // Fixed trees: a shuffle butterfly within each warp, then warp 0 over the
+    // NT / 32 warp sums (fewer barriers than a shared-memory tree).
+    __shared__ double sh[glob::NT / 32];
+    auto cta_reduce = [&](double v) {
 #pragma unroll
-    for (int s = glob::NT / 2; s > 0; s >>= 1) {                 // fixed tree
-        if ((int)threadIdx.x < s) sh[threadIdx.x] = comb<OP>(sh[threadIdx.x], sh[threadIdx.x + s]);
+        for (int s = 16; s > 0; s >>= 1) v = comb<OP>(v, __shfl_xor_sync(0xFFFFFFFFu, v, s));
+        if ((threadIdx.x & 31) == 0) sh[threadIdx.x >> 5] = v;
         __syncthreads();
-    }
+        double t = sh[0];
+#pragma unroll
+        for (int w = 1; w < glob::NT / 32; ++w) t = comb<OP>(t, sh[w]);
+        return t;                                                 // same bits in every thread
+    };
+    const double part = cta_reduce(acc);
     // The last CTA to finish combines the parts (fixed tree over the part index,
     // so the result does not depend on which CTA is last); the arrival counter
-    // lives in work[kGlobalParts] and is reset for the next call.
+    // lives in work[kGlobalCounter] and is reset for the next call.
     __shared__ bool last;
     if (threadIdx.x == 0) {
-        p.work[blockIdx.x] = sh[0];
+        p.work[blockIdx.x] = part;
         __threadfence();
-        unsigned int *count = reinterpret_cast<unsigned int *>(p.work + kGlobalParts);
+        unsigned int *count = reinterpret_cast<unsigned int *>(p.work + kGlobalCounter);
         last = atomicAdd(count, 1u) == kGlobalParts - 1;
     }
     __syncthreads();
@@ -118,16 +173,11 @@ __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_c
     double a = __ldcg(p.work + threadIdx.x * PER);
 #pragma unroll
     for (int i = 1; i < PER; ++i) a = comb<OP>(a, __ldcg(p.work + threadIdx.x * PER + i));
-    sh[threadIdx.x] = a;
-    __syncthreads();
-#pragma unroll
-    for (int s = glob::NT / 2; s > 0; s >>= 1) {
-        if ((int)threadIdx.x < s) sh[threadIdx.x] = comb<OP>(sh[threadIdx.x], sh[threadIdx.x + s]);
-        __syncthreads();
-    }
+    __syncthreads();                                              // sh reused
+    const double total = cta_reduce(a);
     if (threadIdx.x == 0) {
-        *p.result = sh[0];
-        *reinterpret_cast<unsigned int *>(p.work + kGlobalParts) = 0u;
+        *p.result = total;
+        *reinterpret_cast<unsigned int *>(p.work + kGlobalCounter) = 0u;
     }
 }
 

@@ -540,7 +540,7 @@ lop_status lop_reduce_execute(const lop_iteration_space *is, const lop_accessor 
 lop_status lop_global_reduce_execute(const lop_iteration_space *is, int32_t op, double *d_result,
                                      double *d_work, void *cuda_stream)
 {
-    static_assert(lop::kGlobalParts + 1 == LOP_GLOBAL_WORK_DOUBLES, "work size");
+    static_assert(lop::kGlobalCounter + 1 == LOP_GLOBAL_WORK_DOUBLES, "work size");
     if (!is) return fail(LOP_ERR_INVALID, "iteration space is NULL");
     if (op != LOP_REDUCE_SUM && op != LOP_REDUCE_MIN && op != LOP_REDUCE_MAX)
         return fail(LOP_ERR_INVALID, "unknown reduction %d (SUM, MIN, MAX)", op);

@@ -120,12 +120,17 @@ struct ReduceParams {
 
 // Global operator (global_reduce.cu): SUM / MIN / MAX over a region of all
 // frames, deterministic (fixed parts, fixed trees), result in double.
-constexpr int kGlobalParts = 1024;                            // + 1 counter = LOP_GLOBAL_WORK_DOUBLES
+#ifndef LOP_GLOBAL_PARTS
+#define LOP_GLOBAL_PARTS 512
+#endif
+constexpr int kGlobalParts = LOP_GLOBAL_PARTS;               // fixed partition (not per GPU)
+constexpr int kGlobalCounter = 1024;                         // + 1 = LOP_GLOBAL_WORK_DOUBLES
+static_assert(kGlobalParts <= kGlobalCounter && kGlobalParts % 256 == 0, "global parts");
 struct GlobalReduce {
     Common c;                    // c.in: the image; c.roi_*: the region; c.batch
     int32_t op;                  // RED_SUM / RED_MIN / RED_MAX
     int32_t u8;
-    double *work;                // kGlobalParts doubles + an arrival counter (device)
+    double *work;                // kGlobalParts doubles, arrival counter at [kGlobalCounter]
     double *result;              // 1 double (device)
 };
 

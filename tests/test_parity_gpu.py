@@ -891,6 +891,11 @@ def test_global_reduce(lop, shape):
             g = lop.global_reduce(frames, op, roi=roi).item()
             ref = oracle.global_reduce(frames.cpu().numpy(), op, roi=roi)
             assert abs(g - ref) <= 1e-12 * max(1.0, abs(ref)), (op, g, ref)
+        # u8 frames over an unaligned region: ragged and misaligned column groups
+        uframes = torch.stack([u8, 255 - u8, u8 // 2]).cuda()
+        for op in ("sum", "min", "max"):
+            g = lop.global_reduce(uframes, op, roi=roi).item()
+            assert g == oracle.global_reduce(uframes.cpu().numpy(), op, roi=roi), op
     # one scratch buffer reused by many calls: its arrival counter returns to zero
     work = torch.zeros(1025, dtype=torch.float64, device="cuda")
     vals = [lop.global_reduce(img.cuda(), op, work=work).item() for op in ("max", "sum", "min") * 3]
