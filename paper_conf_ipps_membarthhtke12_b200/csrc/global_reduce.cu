@@ -55,18 +55,24 @@ __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_c
     constexpr bool F = sizeof(T) == 4;
     // per-thread accumulators in the cheapest exact form: f32 SUM in double;
     // f32 MIN / MAX in float (exact); u8 SUM in int32 by byte dot products
-    // (IDP4A); u8 MIN / MAX on packed bytes (__vminu4 / __vmaxu4)
+    // (IDP4A); u8 MIN / MAX on bytes in 16-bit lanes
     double dacc = 0.0;
     float facc = OP == RED_MIN ? __int_as_float(0x7f800000) : -__int_as_float(0x7f800000);
     unsigned int iacc = 0;
-    uint32_t bacc = OP == RED_MIN ? 0xFFFFFFFFu : 0u;
+    // u8 MIN / MAX: even and odd bytes in the 16-bit lanes of two accumulators
+    // (native VIMNMX.U16x2; __vminu4 / __vmaxu4 are emulated on sm_100)
+    uint32_t eacc = OP == RED_MIN ? 0x00FF00FFu : 0u, oacc = eacc;
     auto add_word = [&](uint32_t w, int nbytes) {                // u8: 4 packed pixels
         if (nbytes < 4) {                                         // pad with the identity
             const uint32_t keep = nbytes == 0 ? 0u : (0xFFFFFFFFu >> (8 * (4 - nbytes)));
             w = OP == RED_MIN ? (w | ~keep) : (w & keep);
         }
         if (OP == RED_SUM) iacc = __dp4a(w, 0x01010101u, iacc);   // unsigned bytes, exact
-        else bacc = OP == RED_MIN ? __vminu4(bacc, w) : __vmaxu4(bacc, w);
+        else {
+            const uint32_t e = w & 0x00FF00FFu, o = (w >> 8) & 0x00FF00FFu;
+            eacc = OP == RED_MIN ? __vminu2(eacc, e) : __vmaxu2(eacc, e);
+            oacc = OP == RED_MIN ? __vminu2(oacc, o) : __vmaxu2(oacc, o);
+        }
     };
     auto add_f = [&](float v) {
         if (OP == RED_SUM) dacc += (double)v;
@@ -134,12 +140,8 @@ __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_c
     if constexpr (F) acc = OP == RED_SUM ? dacc : (double)facc;
     else if (OP == RED_SUM) acc = (double)iacc;                   // exact (partials < 2^31)
     else {
-        uint32_t m = bacc & 0xFF;
-#pragma unroll
-        for (int j = 1; j < 4; ++j) {
-            const uint32_t v = (bacc >> (8 * j)) & 0xFF;
-            m = OP == RED_MIN ? min(m, v) : max(m, v);
-        }
+        const uint32_t l = OP == RED_MIN ? __vminu2(eacc, oacc) : __vmaxu2(eacc, oacc);
+        const uint32_t m = OP == RED_MIN ? min(l & 0xFFFFu, l >> 16) : max(l & 0xFFFFu, l >> 16);
         acc = (double)m;
     }
     // Fixed trees: a shuffle butterfly within each warp, then warp 0 over the
