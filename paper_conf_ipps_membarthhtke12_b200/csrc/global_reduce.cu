@@ -18,6 +18,10 @@
 
 namespace lop {
 
+#ifndef LOP_GLOBAL_U
+#define LOP_GLOBAL_U 8
+#endif
+
 namespace glob {
 constexpr int NT = 256;
 }
@@ -100,7 +104,7 @@ __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_c
                                                            : -__int_as_float(0x7f800000));
     const uint32_t bid = OP == RED_MIN ? 0xFFFFFFFFu : 0u;
     const uint32_t idw = F ? __float_as_uint(fid) : bid;
-    constexpr int U = 8;
+    constexpr int U = LOP_GLOBAL_U;                              // 16-B groups in flight per thread
     while (r < r1) {
         uint4 q[U];
 #pragma unroll
