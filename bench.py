@@ -2,30 +2,43 @@
 """bench.py -- throughput of the local-operator hot path on B200.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl lop|reference]
-                    [--workload bilateral4096|frames|bands] [--mode clamp]
+                    [--mode clamp] [--no-partitioned] [--no-extras]
 
 One JSON line on rank 0 (driver contract):
   metric / unit   BASELINE.json's metric, in Mpixel/s
-  value           whole-job Mpixel/s, inputs resident in HBM, CUDA events on
-                  the launching stream, K steps between barrier+synchronize,
-                  max over ranks
-  e2e             the same metric through the host pipeline API
+  value           whole-job Mpixel/s of the headline workload, inputs resident
+                  in HBM, CUDA events on the launching stream, K steps between
+                  barrier+synchronize, max over ranks
+  partitioned     BASELINE configs 4 and 5 -- the paths that shard -- at this
+                  N, each with the SAME total work at every N (strong
+                  scaling): c4 = 1024 frames of 1024^2 split over the ranks
+                  (no data-path collective), c5 = one 32768^2 image in row
+                  bands with the NCCL halo exchange; per-rank ms, halo ms,
+                  SFU fraction, NCCL communicator size
+  e2e             the headline metric through the host pipeline API
                   (lop.Pipeline: pinned host in -> device -> pinned host out,
-                  copies inside the timed region)
+                  copies inside the timed region), with the pinned copy
+                  ceiling measured in the same run and the fraction of it
   roofline        the dominant kernel against its bound (SFU for the
                   bilateral filter: 84 distinct ex2 per pixel = (13*13 - 1) / 2 with
                   symmetric pair-sharing; frac_vs_168_ex2_per_px against the
                   unshared count, which the pair kernel exceeds)
   cpu_baseline    the C oracle (double, OpenMP) on a bounded sample, rank 0, N=1
   clocks          nvidia-smi samples taken during the timed region
-  gpu_launches    lop kernel launches inside the timed region (liblop counter)
+  gpu_launches    lop kernel launches inside the headline's timed region
+                  (liblop counter, reset right before it)
 
-A step is one pass of the whole hot path over one batch:
-workload bilateral4096 (default, BASELINE config 2 with clamp): every rank
-filters its own 4096x4096 f32 image (13x13, sigma_d=3, sigma_r=5), i.e.
-frame-parallel weak scaling with no data-path collective.
-workload frames (config 4): 1024 frames of 1024^2 split over the ranks.
-workload bands (config 5): one 32768^2 image in row bands, NCCL halo exchange.
+Headline workload (identical at every N, so the scaling run's N=1 line is
+this bench line): BASELINE config 2 with clamp -- every rank filters its own
+4096x4096 f32 image per step (13x13, sigma_d=3, sigma_r=5), i.e. weak scaling
+with no data-path collective.  The partitioned configs carry the strong
+scaling of the frame and band splits.
+
+Launch: under torchrun (WORLD_SIZE set) every rank runs; `--gpus N` with
+N > 1 and no WORLD_SIZE re-executes itself under torch.distributed.run with
+N ranks (127.0.0.1); --gpus disagreeing with WORLD_SIZE is an error.
+--dry-run: plumbing only (gloo, CPU): every rank reports its partition of
+configs 4 and 5; rank 0 prints them (tests/test_bench_launch.py).
 """
 from __future__ import annotations
 
@@ -33,6 +46,7 @@ import argparse
 import json
 import math
 import os
+import socket
 import statistics
 import subprocess
 import sys
@@ -45,21 +59,28 @@ sys.path.insert(0, ROOT)
 BASELINE_METRIC = "Mpixel/s per filter at 1/2/4/8 B200; % of HBM GB/s or FP32/SFU roofline"
 SM_COUNT = 148
 MUFU_PER_CLK_PER_SM = 16          # MUFU.EX2 lanes per clock per SM on sm_100
+C4_FRAMES, C4_SIZE = 1024, 1024   # BASELINE config 4
+C5_SIZE = 32768                   # BASELINE config 5
+SIGMA_D, SIGMA_R, WINDOW = 3.0, 5.0, 13
 
 
 def parse(argv=None):
     ap = argparse.ArgumentParser()
-    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--gpus", type=int, default=None,
+                    help="ranks (default: WORLD_SIZE, else 1); N > 1 without torchrun self-launches")
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--impl", choices=["lop", "reference"], default="lop")
     ap.add_argument("--workload", choices=["bilateral4096", "frames", "bands"],
-                    default="bilateral4096")
+                    default="bilateral4096", help="headline workload (default: config 2)")
     ap.add_argument("--mode", default="clamp")
     ap.add_argument("--no-extras", action="store_true", help="skip per-filter side measurements")
+    ap.add_argument("--no-partitioned", action="store_true", help="skip the c4 / c5 records")
+    ap.add_argument("--part-steps", type=int, default=5, help="timed steps of c4 / c5")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--dry-run", action="store_true", help="launch plumbing only (gloo, no GPU)")
     return ap.parse_args(argv)
 
 
@@ -74,6 +95,41 @@ def load_peaks():
             "_source": "fallback (B200_PROFILING.md)"}
 
 
+def sfu_peak_tex2(peaks) -> float:
+    """148 SM x 16 MUFU.EX2 / clk x max SM clock, in T ex2 / s."""
+    return SM_COUNT * MUFU_PER_CLK_PER_SM * float(peaks.get("sm_max_mhz", 1965.0)) * 1e6 / 1e12
+
+
+# ------------------------------------------------------------- launching ----
+
+def _free_port() -> int:
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def relaunch_if_needed(args, argv):
+    """Returns an exit code if this process only launched the ranks, else None."""
+    env_world = os.environ.get("WORLD_SIZE")
+    if env_world is None:
+        n = args.gpus or 1
+        if n <= 1:
+            return None
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+               "--nproc-per-node=%d" % n, "--master-addr=127.0.0.1",
+               "--master-port=%d" % _free_port(), os.path.abspath(__file__)] + list(argv)
+        print("[bench] --gpus %d without torchrun: launching %d ranks: %s" % (n, n, " ".join(cmd)),
+              file=sys.stderr, flush=True)
+        return subprocess.call(cmd)
+    if args.gpus is not None and args.gpus != int(env_world):
+        print(json.dumps({"error": "--gpus %d disagrees with WORLD_SIZE=%s" % (args.gpus, env_world)}),
+              flush=True)
+        return 2
+    return None
+
+
 # ------------------------------------------------------------ distributed ----
 
 class Dist:
@@ -81,7 +137,7 @@ class Dist:
         self.world = int(os.environ.get("WORLD_SIZE", "1"))
         self.rank = int(os.environ.get("RANK", "0"))
         self.local = int(os.environ.get("LOCAL_RANK", "0"))
-        self.pg = None
+        self.backend = None
 
     def init(self, backend="nccl"):
         import torch
@@ -91,22 +147,63 @@ class Dist:
                 torch.cuda.set_device(self.local)
             dist.init_process_group(backend, device_id=(torch.device("cuda", self.local)
                                                         if backend == "nccl" else None))
-            self.pg = dist.group.WORLD
+            self.backend = backend
+            # communicator evidence: the process group's size as NCCL sees it
+            print("[bench] rank %d/%d: %s process group initialised, group size %d" %
+                  (self.rank, self.world, backend, dist.get_world_size()), file=sys.stderr,
+                  flush=True)
+
+    def comm_info(self):
+        if self.world == 1:
+            return {"backend": None, "world_size": 1}
+        import torch
+        import torch.distributed as dist
+        info = {"backend": dist.get_backend(), "world_size": dist.get_world_size()}
+        if info["backend"] == "nccl":
+            v = torch.cuda.nccl.version()
+            info["nccl_version"] = ".".join(str(x) for x in v) if isinstance(v, tuple) else str(v)
+        return info
 
     def barrier(self):
         if self.world > 1:
             import torch.distributed as dist
             dist.barrier()
 
-    def max(self, v: float) -> float:
+    def _reduce(self, v, op):
         if self.world == 1:
             return v
         import torch
         import torch.distributed as dist
-        t = torch.tensor([v], dtype=torch.float64,
-                         device="cuda" if torch.cuda.is_available() else "cpu")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dev = "cuda" if self.backend == "nccl" else "cpu"
+        t = torch.tensor([v], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=op)
         return float(t.item())
+
+    def max(self, v: float) -> float:
+        if self.world == 1:
+            return v
+        import torch.distributed as dist
+        return self._reduce(v, dist.ReduceOp.MAX)
+
+    def gather(self, v: float) -> list:
+        """v of every rank, in rank order."""
+        if self.world == 1:
+            return [v]
+        import torch
+        import torch.distributed as dist
+        dev = "cuda" if self.backend == "nccl" else "cpu"
+        t = torch.tensor([v], dtype=torch.float64, device=dev)
+        out = [torch.zeros_like(t) for _ in range(self.world)]
+        dist.all_gather(out, t)
+        return [float(x.item()) for x in out]
+
+    def gather_obj(self, obj):
+        if self.world == 1:
+            return [obj]
+        import torch.distributed as dist
+        out = [None] * self.world
+        dist.all_gather_object(out, obj)
+        return out
 
     def close(self):
         if self.world > 1:
@@ -173,9 +270,10 @@ class ClockSampler:
 
 # ------------------------------------------------------------------ timing ----
 
-def time_steps(step, K, W, dist, stream):
+def time_steps(step, K, W, dist, stream, lop=None):
     """W warm-up steps, then K timed steps bracketed by barrier + synchronize;
-    returns (total_ms max over ranks, per-launch ms list on this rank)."""
+    returns (total_ms max over ranks, per-step ms list on this rank, lop
+    launches inside the timed region or None)."""
     import torch
     for i in range(W):
         step(i)
@@ -186,18 +284,21 @@ def time_steps(step, K, W, dist, stream):
           for _ in range(K)]
     t0 = torch.cuda.Event(enable_timing=True)
     t1 = torch.cuda.Event(enable_timing=True)
+    if lop is not None:
+        lop.reset_launch_count()
     t0.record(stream)
     for i in range(K):
         ev[i][0].record(stream)
         step(i)
         ev[i][1].record(stream)
     t1.record(stream)
+    launches = lop.launch_count() if lop is not None else None
     torch.cuda.synchronize()
     dist.barrier()
     torch.cuda.synchronize()
     total = t0.elapsed_time(t1)
     per = [a.elapsed_time(b) for a, b in ev]
-    return dist.max(total), per
+    return dist.max(total), per, launches
 
 
 def flush_l2(buf):
@@ -206,9 +307,176 @@ def flush_l2(buf):
 
 # --------------------------------------------------------------- workloads ----
 
+# --------------------------------------------------------------- workloads ----
+
+def workload_c2(args, dist, lop, synthetic, dev, stream):
+    """BASELINE config 2: one 4096^2 image per rank per step (weak scaling)."""
+    import torch
+    H = Wd = 4096
+    n_sets = 3                             # rotating sets: 3 x 128 MiB > 126 MB L2
+    seed = synthetic.config_seed(2) + 7919 * dist.rank
+    base = synthetic.angio(H, Wd, seed=seed, device=dev)
+    ins = [base.clone() for _ in range(n_sets)]
+    outs = [torch.empty_like(base) for _ in range(n_sets)]
+
+    def step(i):
+        lop.bilateral(ins[i % n_sets], SIGMA_D, SIGMA_R, args.mode, size=WINDOW,
+                      out=outs[i % n_sets], stream=stream)
+    config = {"workload": "bilateral 4096x4096 f32, 13x13 (sigma_d=3), sigma_r=5, %s; "
+                          "one image per rank per step (BASELINE config 2)" % args.mode,
+              "height": H, "width": Wd, "window": WINDOW, "sigma_d": SIGMA_D,
+              "sigma_r": SIGMA_R, "boundary": args.mode,
+              "l2": "rotating %d input/output sets (%d MiB) > 126 MB L2" % (n_sets, n_sets * 128),
+              "parallelism": "frame-parallel x%d (independent images)" % dist.world}
+    return dict(step=step, px_rank=H * Wd, px_total=H * Wd * dist.world, config=config,
+                scaling="weak", launches_per_step=1, base=base)
+
+
+def workload_c4(args, dist, lop, synthetic, dev, stream):
+    """BASELINE config 4: 1024 frames of 1024^2, contiguous frame ranges per
+    rank (dist.frame_range), one batched launch per rank, no collective."""
+    import torch
+    from paper_conf_ipps_membarthhtke12_b200 import dist as ldist
+    F, S = C4_FRAMES, C4_SIZE
+    lo, hi = ldist.frame_range(F, dist.world, dist.rank)
+    frames = synthetic.angio_frames(F, S, S, seed=synthetic.config_seed(4), first=lo,
+                                    count=hi - lo, device=dev)
+    out = torch.empty_like(frames)
+
+    def step(i):
+        lop.bilateral(frames, SIGMA_D, SIGMA_R, args.mode, size=WINDOW, out=out, stream=stream)
+    config = {"workload": "%d frames x %d^2 f32 bilateral 13x13 %s, frame-parallel "
+                          "(BASELINE config 4)" % (F, S, args.mode),
+              "frames": F, "frame_size": S, "window": WINDOW, "boundary": args.mode,
+              "frames_this_rank": [lo, hi],
+              "l2": "inputs (4 GiB / N) larger than L2",
+              "parallelism": "frame-parallel x%d, contiguous frame ranges" % dist.world}
+    return dict(step=step, px_rank=(hi - lo) * S * S, px_total=F * S * S, config=config,
+                scaling="strong", launches_per_step=1)
+
+
+def workload_c5(args, dist, lop, synthetic, dev, stream):
+    """BASELINE config 5: one 32768^2 image in row bands, NCCL halo exchange
+    (dist.bilateral_bands: interior rows overlap the exchange)."""
+    import torch
+    from paper_conf_ipps_membarthhtke12_b200 import dist as ldist
+    GH = GW = C5_SIZE
+    band = ldist.Bands(GH, GW, dist.world, dist.rank, halo=WINDOW // 2, device=dev,
+                       mode=args.mode)
+    band.fill(lambda y0, y1: synthetic.angio(GH, GW, seed=synthetic.config_seed(5),
+                                             device=dev, row_range=(y0, y1)))
+    out = torch.empty_like(band.owned)
+
+    def step(i):
+        ldist.bilateral_bands(lop, band, SIGMA_D, SIGMA_R, args.mode, size=WINDOW, out=out,
+                              stream=stream)
+
+    def exchange_only(i):
+        band.exchange(stream)
+    config = {"workload": "%d^2 f32 bilateral 13x13 %s, row bands + NCCL halo exchange "
+                          "(BASELINE config 5)" % (GH, args.mode),
+              "height": GH, "width": GW, "window": WINDOW, "boundary": args.mode,
+              "rows_this_rank": [band.y0, band.y1], "halo_rows": band.halo,
+              "l2": "inputs (4 GiB / N) larger than L2",
+              "parallelism": "row-bands x%d" % dist.world}
+    return dict(step=step, px_rank=band.rows * GW, px_total=GH * GW, config=config,
+                scaling="strong", launches_per_step=ldist.launches_per_band_step(band, WINDOW),
+                exchange=exchange_only, halo_bytes=band.halo_bytes)
+
+
+WORKLOADS = {"bilateral4096": workload_c2, "frames": workload_c4, "bands": workload_c5}
+
+
+def sfu_roofline(peaks, px_per_launch, launch_ms):
+    """SFU roofline of the bilateral pair kernel for `px_per_launch` pixels
+    per launch of mean duration `launch_ms` (one GPU)."""
+    taps = WINDOW * WINDOW - 1                 # algorithmic ex2 per pixel (SURVEY §8(d))
+    pair = os.environ.get("LOP_BILATERAL_PAIR", "1") != "0"
+    ex2_px = taps // 2 if pair else taps
+    ex2_per_launch = ex2_px * px_per_launch
+    achieved = ex2_per_launch / (launch_ms / 1000.0) / 1e12
+    achieved_168 = taps * px_per_launch / (launch_ms / 1000.0) / 1e12
+    peak = sfu_peak_tex2(peaks)
+    return {"bound": "alu",
+            "kernel": "lop::bilateral_pair_kernel<6>" if pair else "lop::bilateral_sep_kernel<6>",
+            "achieved": round(achieved, 4), "peak": round(peak, 4), "unit": "Tex2/s",
+            "frac": round(achieved / peak, 4),
+            "work_per_launch": "%d ex2 (= %d distinct per px x %d px)" % (ex2_per_launch, ex2_px,
+                                                                         px_per_launch),
+            "frac_vs_168_ex2_per_px": round(achieved_168 / peak, 4),
+            "peak_basis": "148 SM x 16 MUFU.EX2/clk x %.0f MHz (sm_max_mhz, %s)" %
+                          (float(peaks.get("sm_max_mhz", 1965.0)), peaks["_source"]),
+            "avg_launch_ms": round(launch_ms, 5)}
+
+
+def run_partitioned(args, dist, lop, synthetic, dev, stream, peaks):
+    """Configs 4 and 5 at this N (same total work at every N): one record each."""
+    import torch
+    out = {}
+    K, W = max(1, args.part_steps), 3
+    peak = sfu_peak_tex2(peaks)
+    ex2_px = (WINDOW * WINDOW - 1) // 2
+    for name, make in (("c4", workload_c4), ("c5", workload_c5)):
+        t_setup = time.perf_counter()
+        wl = make(args, dist, lop, synthetic, dev, stream)
+        torch.cuda.synchronize()
+        setup_s = time.perf_counter() - t_setup
+        total_ms, per, launches = time_steps(wl["step"], K, W, dist, stream, lop)
+        rank_ms = statistics.mean(per)
+        per_rank = dist.gather(rank_ms)
+        value = wl["px_total"] * K / (total_ms / 1000.0) / 1e6
+        rec = {"value": round(value, 2), "unit": "Mpixel/s", "scaling": "strong",
+               "n_gpus": dist.world, "steps": K, "warmup": W,
+               "ms_per_step": round(total_ms / K, 4),
+               "per_rank_ms": [round(v, 4) for v in per_rank],
+               "px_per_step": wl["px_total"],
+               # SFU fraction of all N GPUs at the 84 distinct ex2 / px of the pair kernel
+               "sfu_frac": round(ex2_px * wl["px_total"] / (total_ms / K / 1000.0) / 1e12 /
+                                 (peak * dist.world), 4),
+               "gpu_launches": launches,
+               "launches_per_step_per_rank": wl["launches_per_step"],
+               "setup_s": round(setup_s, 1),
+               "config": wl["config"], "comm": dist.comm_info()}
+        if "exchange" in wl:
+            ex_ms, ex_per, _ = time_steps(wl["exchange"], K, W, dist, stream)
+            rec["halo_exchange_ms"] = round(ex_ms / K, 4)
+            rec["halo_exchange_per_rank_ms"] = [round(v, 4) for v in dist.gather(statistics.mean(ex_per))]
+            rec["halo_bytes_per_rank"] = wl["halo_bytes"]
+            rec["halo_note"] = ("exchange alone, timed like the steps; inside a step it overlaps "
+                                "the interior rows (dist.bilateral_bands)")
+        out[name] = rec
+        del wl
+        torch.cuda.empty_cache()
+    return out
+
+
+def measure_copy_ceiling(dev, nbytes, reps=5):
+    """Pinned host<->device copy rate with both directions busy at once (the
+    pipeline's situation), GB/s per direction."""
+    import torch
+    n = nbytes // 4
+    h_src = torch.empty(n, dtype=torch.float32).pin_memory()
+    h_dst = torch.empty(n, dtype=torch.float32).pin_memory()
+    d_a = torch.empty(n, dtype=torch.float32, device=dev)
+    d_b = torch.empty(n, dtype=torch.float32, device=dev)
+    s1, s2 = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
+
+    def both():
+        with torch.cuda.stream(s1):
+            d_a.copy_(h_src, non_blocking=True)
+        with torch.cuda.stream(s2):
+            h_dst.copy_(d_b, non_blocking=True)
+    both()
+    torch.cuda.synchronize()
+    t = time.perf_counter()
+    for _ in range(reps):
+        both()
+    torch.cuda.synchronize()
+    return reps * n * 4 / (time.perf_counter() - t) / 1e9
+
+
 def run_lop(args, dist, peaks):
     import torch
-    import numpy as np
     import synthetic
     import paper_conf_ipps_membarthhtke12_b200 as lop
 
@@ -216,157 +484,92 @@ def run_lop(args, dist, peaks):
     torch.cuda.set_device(dev)
     stream = torch.cuda.current_stream(dev)
     K, W = args.steps, max(3, args.warmup)
-    sigma_d, sigma_r, size = 3.0, 5.0, 13
-    taps = size * size - 1                     # algorithmic ex2 per pixel
-    result = {}
-
-    if args.workload == "bilateral4096":
-        H = Wd = 4096
-        n_sets = 3                             # rotating sets: 3 x 128 MiB > 126 MB L2
-        seed = synthetic.config_seed(2) + 7919 * dist.rank
-        base = synthetic.angio(H, Wd, seed=seed, device=dev)
-        ins = [base.clone() for _ in range(n_sets)]
-        outs = [torch.empty_like(base) for _ in range(n_sets)]
-        px_per_step_rank = H * Wd
-
-        def step(i):
-            lop.bilateral(ins[i % n_sets], sigma_d, sigma_r, args.mode, size=size,
-                          out=outs[i % n_sets], stream=stream)
-        config = {"workload": "bilateral 4096x4096 f32, 13x13 (sigma_d=3), sigma_r=5, %s; "
-                              "one image per rank per step (BASELINE config 2)" % args.mode,
-                  "height": H, "width": Wd, "window": size, "sigma_d": sigma_d,
-                  "sigma_r": sigma_r, "boundary": args.mode,
-                  "l2": "rotating %d input/output sets (%d MiB) > 126 MB L2" %
-                        (n_sets, n_sets * 128),
-                  "parallelism": "frame-parallel x%d (independent images)" % dist.world}
-        scaling = "weak"
-    elif args.workload == "frames":
-        F, S = 1024, 1024
-        lo, hi = F * dist.rank // dist.world, F * (dist.rank + 1) // dist.world
-        frames = synthetic.angio_frames(F, S, S, seed=synthetic.config_seed(4), first=lo,
-                                        count=hi - lo, device=dev)
-        out = torch.empty_like(frames)
-        px_per_step_rank = (hi - lo) * S * S
-
-        def step(i):
-            lop.bilateral(frames, sigma_d, sigma_r, args.mode, size=size, out=out, stream=stream)
-        config = {"workload": "1024 frames x 1024^2 f32 bilateral 13x13 %s, frame-parallel "
-                              "(BASELINE config 4)" % args.mode,
-                  "frames": F, "frame_size": S, "window": size, "boundary": args.mode,
-                  "l2": "inputs (4 GiB / N) larger than L2",
-                  "parallelism": "frame-parallel x%d" % dist.world}
-        scaling = "strong"
-    else:
-        from paper_conf_ipps_membarthhtke12_b200 import dist as ldist
-        GHt = GW = 32768
-        band = ldist.Bands(GHt, GW, dist.world, dist.rank, halo=size // 2, device=dev,
-                           mode=args.mode)
-        band.fill(lambda y0, y1: synthetic.angio(GHt, GW, seed=synthetic.config_seed(5),
-                                                 device=dev, row_range=(y0, y1)))
-        out = torch.empty_like(band.owned)
-        px_per_step_rank = band.rows * GW
-
-        def step(i):
-            ldist.bilateral_bands(lop, band, sigma_d, sigma_r, args.mode, size=size, out=out,
-                                  stream=stream)
-        config = {"workload": "32768^2 f32 bilateral 13x13 %s, row bands + NCCL halo exchange "
-                              "(BASELINE config 5)" % args.mode,
-                  "height": GHt, "width": GW, "window": size, "boundary": args.mode,
-                  "l2": "inputs (4 GiB / N) larger than L2",
-                  "parallelism": "row-bands x%d" % dist.world}
-        scaling = "strong"
-
+    wl = WORKLOADS[args.workload](args, dist, lop, synthetic, dev, stream)
     clocks = ClockSampler(dist.local)
     clocks.start()
-    lop.reset_launch_count()
-    total_ms, per = time_steps(step, K, W, dist, stream)
-    launches = lop.launch_count() - W * (1 if args.workload != "bands" else 1)
+    total_ms, per, launches = time_steps(wl["step"], K, W, dist, stream, lop)
     # keep the GPU busy a little longer so the sampler sees the clocks under load
     t_end = time.time() + max(0.0, 1.0 - total_ms / 1000.0)
     i = 0
     while time.time() < t_end:
-        step(i)
+        wl["step"](i)
         i += 1
         if i % 20 == 0:
             torch.cuda.synchronize()
     torch.cuda.synchronize()
     clk = clocks.stop()
 
-    px_total = px_per_step_rank * dist.world * K
-    value = px_total / (total_ms / 1000.0) / 1e6
+    value = wl["px_total"] * K / (total_ms / 1000.0) / 1e6
     avg_launch_ms = sum(per) / len(per)
     # The symmetric pair-sharing kernel (default) needs (W^2-1)/2 = 84 distinct
     # ex2 per pixel (SURVEY §8(d)'s tighter bound): that is `achieved`/`frac`.
     # Against the W^2-1 = 168 of the unshared method (Listing 5) the ratio can
     # exceed 1 -- reported beside it as frac_vs_168_ex2_per_px.
-    pair = os.environ.get("LOP_BILATERAL_PAIR", "1") != "0"
-    ex2_px = taps // 2 if pair else taps
-    ex2_per_launch = ex2_px * px_per_step_rank
-    achieved = ex2_per_launch / (avg_launch_ms / 1000.0) / 1e12
-    achieved_168 = taps * px_per_step_rank / (avg_launch_ms / 1000.0) / 1e12
-    sm_mhz_peak = float(peaks.get("sm_max_mhz", 1965.0))
-    peak = SM_COUNT * MUFU_PER_CLK_PER_SM * sm_mhz_peak * 1e6 / 1e12
-    traffic = None
-    tp = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tp):
-        with open(tp) as f:
-            tj = json.load(f)
-            traffic = tj.get("bilateral_13x13_4096" if pair else "bilateral_sep_13x13_4096")
-    roofline = {"bound": "alu",
-                "kernel": "lop::bilateral_pair_kernel<6>" if pair else "lop::bilateral_sep_kernel<6>",
-                "achieved": round(achieved, 4), "peak": round(peak, 4), "unit": "Tex2/s",
-                "frac": round(achieved / peak, 4), "traffic": traffic,
-                "work_per_launch": "%d ex2 (= %d distinct per px x %d px)" % (ex2_per_launch, ex2_px,
-                                                                             px_per_step_rank),
-                "frac_vs_168_ex2_per_px": round(achieved_168 / peak, 4),
-                "peak_basis": "148 SM x 16 MUFU.EX2/clk x %.0f MHz (sm_max_mhz, %s)" %
-                              (sm_mhz_peak, peaks["_source"]),
-                "avg_launch_ms": round(avg_launch_ms, 5)}
-    result.update(dict(metric=BASELINE_METRIC, value=round(value, 2), unit="Mpixel/s",
-                       n_gpus=dist.world, steps=K, warmup=W,
-                       ms_per_step=round(total_ms / K, 5), higher_is_better=True,
-                       scaling=scaling, vs_baseline=None, dtype="f32", data="synthetic",
-                       config=config, roofline=roofline, clocks=clk, gpu_launches=int(launches)))
+    roofline = sfu_roofline(peaks, wl["px_rank"], avg_launch_ms)
+    # DRAM traffic is not measurable inside this process (no profiler); the ncu
+    # capture of the same kernel is committed under profiles/ 
+    roofline["traffic"] = None
+    roofline["traffic_note"] = "dram bytes per launch: see profiles/r02_*ncu_full_bilateral_pair*.md"
+    result = dict(metric=BASELINE_METRIC, value=round(value, 2), unit="Mpixel/s",
+                  n_gpus=dist.world, steps=K, warmup=W, ms_per_step=round(total_ms / K, 5),
+                  higher_is_better=True, scaling=wl["scaling"], vs_baseline=None, dtype="f32",
+                  data="synthetic", config=wl["config"], roofline=roofline, clocks=clk,
+                  gpu_launches=int(launches), comm=dist.comm_info())
 
     # ---- e2e through the host pipeline API (rank-local, max over ranks)
     if args.workload == "bilateral4096" and args.e2e_steps > 0:
-        H = Wd = 4096
-        K = args.e2e_steps
-        # one host frame per step (distinct pinned buffers), streamed back to back
-        host_in = base.cpu().unsqueeze(0).repeat(K, 1, 1).pin_memory()
-        host_out = torch.empty_like(host_in).pin_memory()
-        # single synchronous image: 1024-row chunks (ramped); a frame stream: 2048-row
-        # chunks (the fill / drain is paid once per stream; tools/pipe_frames_sweep.py)
-        one = host_in[0]
-        pipe1 = lop.Pipeline(Wd, H, device=dist.local, chunk_rows=1024)
-        pipe1.bilateral(one, host_out[0], sigma_d, sigma_r, args.mode, size=size)
-        dist.barrier()
-        t0 = time.perf_counter()
-        pipe1.bilateral(one, host_out[0], sigma_d, sigma_r, args.mode, size=size)
-        t_single = dist.max(time.perf_counter() - t0)
-        pipe1.close()
-        pipe = lop.Pipeline(Wd, H, device=dist.local, chunk_rows=2048)
-        # warm-up over every frame: the first DMA touching each pinned page is slower
-        pipe.bilateral_frames(host_in, host_out, sigma_d, sigma_r, args.mode, size=size)
-        dist.barrier()
-        t0 = time.perf_counter()
-        pipe.bilateral_frames(host_in, host_out, sigma_d, sigma_r, args.mode, size=size)
-        t = dist.max(time.perf_counter() - t0)
-        h2d, d2h = pipe.bytes_moved()
-        pipe.close()
-        result["e2e"] = {"value": round(H * Wd * dist.world * K / t / 1e6, 2),
-                         "unit": "Mpixel/s", "h2d_bytes_per_step": int(h2d // K),
-                         "d2h_bytes_per_step": int(d2h // K),
-                         "single_image_call_Mpx_s": round(H * Wd * dist.world / t_single / 1e6, 2),
-                         "api": "lop.Pipeline.bilateral_frames (lop_pipeline_bilateral_frames): "
-                                "%d steps = %d pinned host frames (the config-2 image) streamed "
-                                "back to back in 2048-row chunks on 3 streams (H2D / kernel / "
-                                "D2H), every frame's upload and download inside the timed "
-                                "region; wall clock; single_image_call = one synchronous "
-                                "lop_pipeline_bilateral call" % (K, K)}
+        result["e2e"] = run_e2e(args, dist, lop, wl["base"], dev)
     if not args.no_extras and dist.world == 1 and args.workload == "bilateral4096":
         result["filters"] = extras(lop, synthetic, dev, stream, peaks)
+    del wl
+    torch.cuda.empty_cache()
+    if not args.no_partitioned:
+        result["partitioned"] = run_partitioned(args, dist, lop, synthetic, dev, stream, peaks)
     return result
+
+
+def run_e2e(args, dist, lop, base, dev):
+    H = Wd = 4096
+    K = args.e2e_steps
+    # one host frame per step (distinct pinned buffers), streamed back to back
+    host_in = base.cpu().unsqueeze(0).repeat(K, 1, 1).pin_memory()
+    host_out = host_in.clone().pin_memory()
+    # single synchronous image: 1024-row chunks (ramped); a frame stream: 2048-row
+    # chunks (the fill / drain is paid once per stream; tools/pipe_frames_sweep.py)
+    one = host_in[0]
+    pipe1 = lop.Pipeline(Wd, H, device=dist.local, chunk_rows=1024)
+    pipe1.bilateral(one, host_out[0], SIGMA_D, SIGMA_R, args.mode, size=WINDOW)
+    dist.barrier()
+    t0 = time.perf_counter()
+    pipe1.bilateral(one, host_out[0], SIGMA_D, SIGMA_R, args.mode, size=WINDOW)
+    t_single = dist.max(time.perf_counter() - t0)
+    pipe1.close()
+    pipe = lop.Pipeline(Wd, H, device=dist.local, chunk_rows=2048)
+    # warm-up over every frame: the first DMA touching each pinned page is slower
+    pipe.bilateral_frames(host_in, host_out, SIGMA_D, SIGMA_R, args.mode, size=WINDOW)
+    dist.barrier()
+    t0 = time.perf_counter()
+    pipe.bilateral_frames(host_in, host_out, SIGMA_D, SIGMA_R, args.mode, size=WINDOW)
+    t = dist.max(time.perf_counter() - t0)
+    h2d, d2h = pipe.bytes_moved()
+    pipe.close()
+    # the copy ceiling in the same run: both directions busy at once, 64 MiB each
+    ceil_gbs = measure_copy_ceiling(dev, H * Wd * 4)
+    t_floor = max(h2d, d2h) / (ceil_gbs * 1e9)
+    return {"value": round(H * Wd * dist.world * K / t / 1e6, 2),
+            "unit": "Mpixel/s", "h2d_bytes_per_step": int(h2d // K),
+            "d2h_bytes_per_step": int(d2h // K),
+            "pcie_ceiling_gbs": round(ceil_gbs, 2),
+            "frac": round(t_floor / t, 4),
+            "single_image_call_Mpx_s": round(H * Wd * dist.world / t_single / 1e6, 2),
+            "api": "lop.Pipeline.bilateral_frames (lop_pipeline_bilateral_frames): "
+                   "%d steps = %d pinned host frames (the config-2 image) streamed "
+                   "back to back in 2048-row chunks on 3 streams (H2D / kernel / "
+                   "D2H), every frame's upload and download inside the timed "
+                   "region; wall clock; single_image_call = one synchronous "
+                   "lop_pipeline_bilateral call" % (K, K),
+            "ceiling_method": "pinned H2D and D2H of 64 MiB at once on two streams, 5 reps, "
+                              "GB/s per direction; frac = max(h2d, d2h bytes) / ceiling / time"}
 
 
 def extras(lop, synthetic, dev, stream, peaks):
@@ -536,6 +739,10 @@ def run_reference(args, dist):
     """--impl reference: the oracle timed on the host cores (rank 0 only)."""
     if dist.rank != 0:
         return None
+    if dist.world > 1 and os.environ.get("OMP_NUM_THREADS") == "1":
+        # torchrun sets OMP_NUM_THREADS=1 per rank; the one rank that runs the
+        # oracle uses all host cores, as at N = 1 (libgomp reads it at load)
+        os.environ["OMP_NUM_THREADS"] = str(os.cpu_count() or 1)
     import oracle
     oracle.build()
     H = Wd = 4096
@@ -564,7 +771,7 @@ def run_reference(args, dist):
     value = rows * Wd * K / t / 1e6
     sample = ("%d rows x 4096 px of the config-2 image per step (of 4096 rows), "
               "13x13, sigma_d=3, sigma_r=5, %s" % (rows, args.mode))
-    return dict(metric=BASELINE_METRIC, value=round(value, 4), unit="Mpixel/s", n_gpus=args.gpus,
+    return dict(metric=BASELINE_METRIC, value=round(value, 4), unit="Mpixel/s", n_gpus=dist.world,
                 steps=K, warmup=W, ms_per_step=round(t / K * 1000, 3), higher_is_better=True,
                 scaling="weak", vs_baseline=None, dtype="f64", data="synthetic", impl="reference",
                 config={"workload": "bilateral 4096x4096 f32 input, 13x13 (sigma_d=3), "
@@ -576,9 +783,32 @@ def run_reference(args, dist):
                      "d2h_bytes_per_step": 0})
 
 
+def run_dry(args, dist):
+    """--dry-run: the launch and partition plumbing without a GPU (gloo)."""
+    from paper_conf_ipps_membarthhtke12_b200 import dist as ldist
+    dist.init("gloo")
+    lo, hi = ldist.frame_range(C4_FRAMES, dist.world, dist.rank)
+    y0, y1 = ldist.band_range(C5_SIZE, dist.world, dist.rank)
+    mine = {"rank": dist.rank, "c4_frames": [lo, hi], "c5_rows": [y0, y1],
+            "pid": os.getpid()}
+    plans = dist.gather_obj(mine)
+    total = dist.gather(float(hi - lo))
+    if dist.rank == 0:
+        print(json.dumps({"dry_run": True, "n_gpus": dist.world, "comm": dist.comm_info(),
+                          "ranks": plans, "c4_frames_total": int(sum(total))}), flush=True)
+    dist.close()
+    return 0
+
+
 def main(argv=None):
+    argv = sys.argv[1:] if argv is None else argv
     args = parse(argv)
+    rc = relaunch_if_needed(args, argv)
+    if rc is not None:
+        return rc
     dist = Dist()
+    if args.dry_run:
+        return run_dry(args, dist)
     if args.impl == "reference":
         if dist.rank == 0:
             line = run_reference(args, dist)

@@ -32,6 +32,11 @@
  *     addressable for y in [-halo_top, height + halo_bottom).
  *   - Index types: coordinates are int32, byte offsets int64 (a 32768^2 f32
  *     image is 4 GiB).
+ *   - No in-place operation: a local operator reads input pixels that other
+ *     threads may already have written, so the byte range of the input view
+ *     (all frames, halo rows included) must not intersect that of the output
+ *     view; overlapping views return LOP_ERR_INVALID before any launch (the
+ *     check is on address ranges, so interleaved layouts are rejected too).
  */
 #ifndef LOP_H
 #define LOP_H

@@ -293,7 +293,8 @@ def bilateral_f32(img, sigma_d, sigma_r, mode, cval=0.0, size=None, cmask=None, 
     """Bilateral filter (Alg. 1) of a float32 image; returns (out f64, valid).
 
     ``cmask`` None -> closeness from Eq. (1) per tap with window ``size``
-    (default 4*sigma_d+1, PAPER.md L325 / Listing 3); else the given mask
+    (default 2*round(2*sigma_d)+1 = 4*sigma_d+1 for integer sigma_d,
+    PAPER.md L325 / Listing 3; odd for every sigma_d, reading c1); else the given mask
     (Listing 5: c = CMask(xf, yf)).
     """
     img, stride = _img(img, np.float32)
@@ -304,7 +305,7 @@ def bilateral_f32(img, sigma_d, sigma_r, mode, cval=0.0, size=None, cmask=None, 
         cptr = _ptr(cmask)
     else:
         if size is None:
-            size = int(round(4 * sigma_d)) + 1
+            size = 2 * int(round(2 * sigma_d)) + 1     # 4*sigma_d+1, always odd (reading c1)
         mw, mh = (size, size) if isinstance(size, int) else size
         cptr = None
     y0, y1 = (0, H) if rows is None else rows
@@ -324,7 +325,7 @@ def bilateral_f32_points(img, sigma_d, sigma_r, mode, xs, ys, cval=0.0, size=Non
         cptr = _ptr(cmask)
     else:
         if size is None:
-            size = int(round(4 * sigma_d)) + 1
+            size = 2 * int(round(2 * sigma_d)) + 1     # 4*sigma_d+1, always odd (reading c1)
         mw, mh = (size, size) if isinstance(size, int) else size
         cptr = None
     xs = np.ascontiguousarray(xs, np.int64)

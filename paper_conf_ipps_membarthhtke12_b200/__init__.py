@@ -39,6 +39,12 @@ __all__ = ["bilateral", "convolve", "convolve_chain", "gaussian", "sobel", "clos
            "Pipeline", "LopError", "image_view", "MODES", "library_path"]
 
 
+def _default_window(sigma_d: float) -> int:
+    """2*round(2 sigma_d) + 1: the paper's 4 sigma_d + 1 for
+    integer sigma_d, and odd for every sigma_d (reading c1)."""
+    return 2 * int(round(2.0 * float(sigma_d))) + 1
+
+
 def library_path() -> str:
     return _lib.LIB_PATH
 
@@ -141,7 +147,7 @@ def bilateral(x: torch.Tensor, sigma_d: float, sigma_r: float, mode="clamp", con
     else:
         marr, mptr = None, None
         if size is None:
-            size = int(round(4 * sigma_d)) + 1
+            size = _default_window(sigma_d)
         size_xy = (size, size) if isinstance(size, int) else tuple(size)
     if out is None:
         out = torch.empty_like(x)
@@ -282,7 +288,7 @@ def sobel(x: torch.Tensor, direction: int = 0, mode="clamp", constant=0.0, **kw)
 
 def closeness_mask(sigma_d: float, size_x: int | None = None, size_y: int | None = None):
     """Eq. (1) closeness coefficients as Listing 4's float mask[] (yf outer)."""
-    size_x = int(round(4 * sigma_d)) + 1 if size_x is None else size_x
+    size_x = _default_window(sigma_d) if size_x is None else size_x
     size_y = size_x if size_y is None else size_y
     out = np.empty((size_y, size_x), np.float32)
     _check(lib.lop_mask_closeness(float(sigma_d), size_x, size_y, out.ctypes.data))
@@ -365,7 +371,7 @@ class Pipeline:
             marr, m = _host_mask(mask, _lib.LOP_F32)
             sx, sy, mptr = m.size_x, m.size_y, ctypes.byref(m)
         else:
-            size = int(round(4 * sigma_d)) + 1 if size is None else size
+            size = _default_window(sigma_d) if size is None else size
             sx, sy = (size, size) if isinstance(size, int) else size
             mptr = None
         _check(lib.lop_pipeline_bilateral(self._h, ip, istr, op, ostr, _mode(mode),
@@ -385,7 +391,7 @@ class Pipeline:
             marr, m = _host_mask(mask, _lib.LOP_F32)
             sx, sy, mptr = m.size_x, m.size_y, ctypes.byref(m)
         else:
-            size = int(round(4 * sigma_d)) + 1 if size is None else size
+            size = _default_window(sigma_d) if size is None else size
             sx, sy = (size, size) if isinstance(size, int) else size
             mptr = None
         _check(lib.lop_pipeline_bilateral_frames(

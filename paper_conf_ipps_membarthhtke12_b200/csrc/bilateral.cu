@@ -28,6 +28,7 @@
 #include <cstdlib>
 
 #include "boundary.cuh"
+#include "launch_cache.h"
 #include "lop_params.h"
 
 namespace lop {
@@ -840,14 +841,10 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
 // ------------------------------------------------------------- launchers
 template <typename P, typename K>
 static cudaError_t launch_tiled(K kernel, const P &p, size_t smem, cudaStream_t stream,
-                                size_t &configured)
+                                PerDevice &configured)
 {
-    if (smem > 48 * 1024 && smem > configured) {
-        cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)smem);
-        if (e != cudaSuccess) return e;
-        configured = smem;
-    }
+    cudaError_t e = ensure_smem(kernel, smem, configured);
+    if (e != cudaSuccess) return e;
     dim3 grid((p.c.roi_w + tiled::TW - 1) / tiled::TW, (p.c.roi_h + tiled::TH - 1) / tiled::TH,
               p.c.batch);
     kernel<<<grid, tiled::NT, smem, stream>>>(p);
@@ -858,7 +855,7 @@ template <int RX, bool SC>
 static cudaError_t launch_tiled_rx_sc(const BilateralTiled &p, cudaStream_t stream)
 {
     using S = tiled::Shape<RX>;
-    static size_t configured = 0;
+    static PerDevice configured;
     const size_t smem = (size_t)((tiled::TH + 2 * p.c.ry) * S::SW + (2 * p.c.ry + 1) * 4 * S::MV) *
                         sizeof(float);
     return launch_tiled(bilateral_tiled_kernel<RX, SC>, p, smem, stream, configured);
@@ -874,7 +871,7 @@ template <int RX, int NP, bool SC>
 static cudaError_t launch_sep_rx_np(const BilateralSep &p, cudaStream_t stream)
 {
     using S = tiled::Shape<RX>;
-    static size_t configured = 0;
+    static PerDevice configured;
     const size_t smem = (size_t)((tiled::TH + 2 * p.c.ry) * S::SW + ((2 * p.c.ry + 1 + 3) & ~3)) *
                         sizeof(float);
     return launch_tiled(bilateral_sep_kernel<RX, NP, SC>, p, smem, stream, configured);
@@ -904,27 +901,22 @@ template <int R>
 static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
 {
     using S = pair::Shape<R>;
-    static int resident = 0;
+    static PerDevice smem_set, resident_cache;
     const size_t smem = (size_t)pair::NW * S::WARP_FLOATS * sizeof(float);
-    if (!resident) {
-        int dev = 0, sms = 0, per_sm = 0;
-        cudaError_t e = cudaFuncSetAttribute(bilateral_pair_kernel<R>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e == cudaSuccess) e = cudaGetDevice(&dev);
-        if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (e == cudaSuccess)
-            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, bilateral_pair_kernel<R>,
-                                                              pair::NW * 32, smem);
-        if (e != cudaSuccess) return e;
-        resident = std::max(1, sms * per_sm);
-    }
+    cudaError_t e;
+    const int64_t resident = resident_ctas(bilateral_pair_kernel<R>, pair::NW * 32, smem, smem_set,
+                                           resident_cache, e);
+    if (e != cudaSuccess) return e;
+    e = ensure_smem(bilateral_pair_kernel<R>, smem, smem_set);
+    if (e != cudaSuccess) return e;
     BilateralSep p = p0;
     const int64_t strips = ((p.c.roi_x0 & 3) + p.c.roi_w + S::OW - 1) / S::OW;
     int T = 0;
     if (const char *env = std::getenv("LOP_PAIR_ROWS")) T = std::atoi(env);
-    static thread_local int64_t memo_key[3] = {-1, -1, -1};
+    static thread_local int64_t memo_key[4] = {-1, -1, -1, -1};
     static thread_local int memo_T = 0;
-    if (T <= 0 && memo_key[0] == p.c.roi_h && memo_key[1] == strips && memo_key[2] == p.c.batch)
+    if (T <= 0 && memo_key[0] == p.c.roi_h && memo_key[1] == strips && memo_key[2] == p.c.batch &&
+        memo_key[3] == resident)
         T = memo_T;
     if (T <= 0) {
         // every T from 1 to the ROI height: waves of resident CTAs x rows per warp
@@ -941,7 +933,7 @@ static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
             if (T == 0 || cost < best) { best = cost; T = t; }
             if (segs == 1) break;
         }
-        memo_key[0] = p.c.roi_h; memo_key[1] = strips; memo_key[2] = p.c.batch;
+        memo_key[0] = p.c.roi_h; memo_key[1] = strips; memo_key[2] = p.c.batch; memo_key[3] = resident;
         memo_T = T;
     }
     p.pair_rows = T;

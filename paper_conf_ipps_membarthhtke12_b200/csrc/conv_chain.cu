@@ -23,6 +23,7 @@
 
 #include "boundary.cuh"
 #include "kernels.h"
+#include "launch_cache.h"
 #include "lop_params.h"
 #include "stage.cuh"
 
@@ -692,13 +693,9 @@ cudaError_t launch_chain_cfg(const ConvChain &p, cudaStream_t stream)
     using S = chain::Shape<T>;
     const size_t smem = (size_t)(TS + 2 * R1 + 2 * R2) * S::ISW * sizeof(T) +
                         (size_t)(TS + 2 * R2) * S::GW * sizeof(T);
-    static bool configured = false;
-    if (!configured) {
-        cudaError_t e = cudaFuncSetAttribute(conv_chain_kernel<T, TO, R1, R2, TS>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        configured = true;
-    }
+    static PerDevice configured;
+    const cudaError_t e = ensure_smem(conv_chain_kernel<T, TO, R1, R2, TS>, smem, configured);
+    if (e != cudaSuccess) return e;
     const Common &c = p.s1.c;
     dim3 grid((c.roi_w + S::OW - 1) / S::OW, (c.roi_h + TS - 1) / TS, c.batch);
     conv_chain_kernel<T, TO, R1, R2, TS><<<grid, chain::NT, smem, stream>>>(p);
@@ -743,22 +740,17 @@ bool launch_chain_stream(const ConvChain &p0, cudaStream_t stream, cudaError_t &
     const int sy0 = std::max(c.roi_y0, R2 - c.off_y);
     const int sy1 = std::min(c.roi_y0 + c.roi_h, g.GH - R2 - c.off_y);
     if (sy1 - sy0 < 16) return false;
-    static int resident = 0;
+    static PerDevice smem_set, resident_cache;
     constexpr size_t smem_stream = (size_t)chain::NW * S::WARP_BYTES;
     using TS = chain::Shape<T>;
     constexpr size_t smem_tile = (size_t)(chain::TSB + 2 * R1 + 2 * R2) * TS::ISW * sizeof(T) +
                                  (size_t)(chain::TSB + 2 * R2) * TS::GW * sizeof(T);
     constexpr size_t smem = smem_stream > smem_tile ? smem_stream : smem_tile;
     auto kern = conv_chain_stream_kernel<T, TO, R1, R2>;
-    if (!resident) {
-        int dev = 0, sms = 0, per_sm = 0;
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e == cudaSuccess) e = cudaGetDevice(&dev);
-        if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, chain::NT, smem);
-        if (e != cudaSuccess) { err = e; return true; }
-        resident = std::max(1, sms * per_sm);
-    }
+    cudaError_t e;
+    const int64_t resident = resident_ctas(kern, chain::NT, smem, smem_set, resident_cache, e);
+    if (e == cudaSuccess) e = ensure_smem(kern, smem, smem_set);
+    if (e != cudaSuccess) { err = e; return true; }
     ConvChain p = p0;
     ChainPlan &pl = p.plan;
     pl.sy0 = sy0;

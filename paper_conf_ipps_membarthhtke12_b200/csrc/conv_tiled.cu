@@ -31,6 +31,7 @@
 #include "boundary.cuh"
 #include "stage.cuh"
 #include "kernels.h"
+#include "launch_cache.h"
 #include "lop_params.h"
 
 namespace lop {
@@ -540,27 +541,21 @@ cudaError_t launch_cfg(const ConvSep &s, cudaStream_t stream)
 {
     using S = TileShape<T>;
     const size_t smem = (size_t)NBUF * (TS + 2 * R) * S::ROW_BYTES;
-    static int grid_max = 0;
-    if (!grid_max) {
-        if (smem > 48 * 1024) {
-            cudaError_t e = cudaFuncSetAttribute(conv_sep_kernel<T, TO, R, SWAR, TS, NBUF>,
-                                                 cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                                 (int)smem);
-            if (e != cudaSuccess) return e;
-        }
-        int dev = 0, sms = 0, per_sm = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-            &per_sm, conv_sep_kernel<T, TO, R, SWAR, TS, NBUF>, convt::NT, smem);
-        grid_max = sms * (per_sm > 0 ? per_sm : 1);
-        // persistent (NBUF = 2) grid: LOP_CONV_CTAS_PER_SM caps the resident CTAs so
-        // that each walks several tiles (otherwise a 4096^2 u8 image -- 1024 tiles --
-        // fits in one wave and the double buffer never pipelines)
-        if (const char *env = std::getenv("LOP_CONV_CTAS_PER_SM")) {
-            const int cap = std::atoi(env);
-            if (cap > 0 && sms * cap < grid_max) grid_max = sms * cap;
-        }
+    static PerDevice smem_set, resident;
+    cudaError_t e;
+    int64_t grid_max = resident_ctas(conv_sep_kernel<T, TO, R, SWAR, TS, NBUF>, convt::NT, smem,
+                                     smem_set, resident, e);
+    if (e != cudaSuccess) return e;
+    e = ensure_smem(conv_sep_kernel<T, TO, R, SWAR, TS, NBUF>, smem, smem_set);
+    if (e != cudaSuccess) return e;
+    // persistent (NBUF = 2) grid: LOP_CONV_CTAS_PER_SM caps the resident CTAs so
+    // that each walks several tiles (otherwise a 4096^2 u8 image -- 1024 tiles --
+    // fits in one wave and the double buffer never pipelines)
+    if (const char *env = std::getenv("LOP_CONV_CTAS_PER_SM")) {
+        int sms = 0;
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, current_device());
+        const int cap = std::atoi(env);
+        if (cap > 0 && (int64_t)sms * cap < grid_max) grid_max = (int64_t)sms * cap;
     }
     const long ntiles = (long)((s.c.roi_w + S::TWE - 1) / S::TWE) * ((s.c.roi_h + TS - 1) / TS) *
                         s.c.batch;

@@ -143,6 +143,34 @@ lop_status check_rows(const lop::Geom &g, int mode, int64_t iy_lo, int64_t iy_hi
     return LOP_OK;
 }
 
+// Byte range [lo, hi) of device memory a view spans: rows -halo_top ..
+// height + halo_bottom - 1 of every frame.
+void view_span(const lop_image &im, int64_t halo_top, int64_t halo_bottom, uintptr_t &lo,
+               uintptr_t &hi)
+{
+    const int64_t es = elem_size(im.dtype);
+    const int64_t last_frame = im.batch > 1 ? (int64_t)(im.batch - 1) * im.batch_stride_bytes : 0;
+    const uintptr_t base = reinterpret_cast<uintptr_t>(im.data);
+    lo = base - (uintptr_t)(halo_top * im.stride_bytes);
+    hi = base + (uintptr_t)(last_frame + (im.height + halo_bottom - 1) * im.stride_bytes +
+                            (int64_t)im.width * es);
+}
+
+// The stencil kernels read input rows other CTAs (warps) may already have
+// written: input and output storage must not overlap (include/lop.h).
+lop_status check_disjoint(const lop_image &in, const lop_image &out)
+{
+    uintptr_t a0, a1, b0, b1;
+    view_span(in, in.halo_top, in.halo_bottom, a0, a1);
+    view_span(out, 0, 0, b0, b1);
+    if (a0 < b1 && b0 < a1)
+        return fail(LOP_ERR_INVALID,
+                    "input and output storage overlap (input bytes [%p, %p), output [%p, %p)): "
+                    "local operators cannot run in place", (void *)a0, (void *)a1, (void *)b0,
+                    (void *)b1);
+    return LOP_OK;
+}
+
 struct Prepared {
     lop::Common c;
 };
@@ -169,6 +197,8 @@ lop_status prepare(const lop_iteration_space *is, const lop_accessor *in, Prepar
     if (ii.width != oi.width || ii.height != oi.height)
         return fail(LOP_ERR_INVALID, "input %d x %d and output %d x %d differ (Listing 2 l.8-9)",
                     ii.width, ii.height, oi.width, oi.height);
+    st = check_disjoint(ii, oi);
+    if (st) return st;
     if (!std::isfinite(bc.constant)) return fail(LOP_ERR_INVALID, "constant is not finite");
     if (ii.dtype == LOP_U8 && bc.mode == LOP_CONSTANT &&
         (bc.constant < 0 || bc.constant > 255 || bc.constant != std::floor(bc.constant)))

@@ -23,6 +23,7 @@
 
 #include "boundary.cuh"
 #include "kernels.h"
+#include "launch_cache.h"
 #include "lop_params.h"
 #include "stage.cuh"
 
@@ -225,13 +226,9 @@ cudaError_t launch_tiled_ts(const ReduceParams &p, cudaStream_t stream)
 {
     using S = red::Shape<T, TS>;
     const size_t smem = (size_t)(S::TS + 2 * R) * S::SWE * sizeof(T);
-    static bool configured = false;
-    if (!configured && smem > 48 * 1024) {
-        cudaError_t e = cudaFuncSetAttribute(reduce_tiled_kernel<T, OP, R, TS>,
-                                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        configured = true;
-    }
+    static PerDevice configured;
+    const cudaError_t e = ensure_smem(reduce_tiled_kernel<T, OP, R, TS>, smem, configured);
+    if (e != cudaSuccess) return e;
     dim3 grid((p.c.roi_w + S::TWE - 1) / S::TWE, (p.c.roi_h + S::TS - 1) / S::TS, p.c.batch);
     reduce_tiled_kernel<T, OP, R, TS><<<grid, red::NT, smem, stream>>>(p);
     return cudaGetLastError();

@@ -23,13 +23,7 @@ for w in $WHAT; do
     bench)
       timeout 900 python bench.py > "$OUT/bench.json" 2> "$OUT/bench.err"
       echo "bench exit $?" >> "$OUT/status.txt" ;;
-    benchalt)
-      timeout 900 python bench.py --workload frames --steps 5 --warmup 3 --no-cpu-baseline \
-        > "$OUT/bench_frames.json" 2> "$OUT/bench_frames.err"
-      echo "bench_frames exit $?" >> "$OUT/status.txt"
-      timeout 900 python bench.py --workload bands --steps 5 --warmup 3 --no-cpu-baseline \
-        > "$OUT/bench_bands.json" 2> "$OUT/bench_bands.err"
-      echo "bench_bands exit $?" >> "$OUT/status.txt"
+    reference)
       timeout 600 python bench.py --impl reference --steps 3 --warmup 1 \
         > "$OUT/bench_reference.json" 2> "$OUT/bench_reference.err"
       echo "bench_reference exit $?" >> "$OUT/status.txt" ;;
@@ -39,12 +33,12 @@ for w in $WHAT; do
     ncu)
       timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"bilateral|conv" -c 40 --csv \
         --log-file "$OUT/launches.csv" python bench.py --steps 20 --warmup 3 --no-extras \
-        --no-cpu-baseline --e2e-steps 0 > "$OUT/ncu_launch_bench.log" 2>&1
+        --no-cpu-baseline --e2e-steps 0 --no-partitioned > "$OUT/ncu_launch_bench.log" 2>&1
       echo "ncu exit $?" >> "$OUT/status.txt" ;;
     full)
       timeout 900 ncu --set full --clock-control none --import-source on \
         -k regex:bilateral_ -s 3 -c 1 -o "$OUT/prof_bilateral" -f \
-        python bench.py --steps 5 --warmup 3 --no-extras --no-cpu-baseline --e2e-steps 0 \
+        python bench.py --steps 5 --warmup 3 --no-extras --no-cpu-baseline --e2e-steps 0 --no-partitioned \
         > "$OUT/ncu_full.log" 2>&1
       echo "full exit $?" >> "$OUT/status.txt" ;;
     fullconv)
