@@ -224,6 +224,70 @@ lop_status lop_convolve2_execute(const lop_iteration_space *is, const lop_access
 lop_status lop_global_reduce_execute(const lop_iteration_space *is, int32_t op, double *d_result,
                                      double *d_work, void *cuda_stream);
 
+/* Local operator over several Accessors with a per-tap function
+ * (SURVEY §8(f) N2): PAPER.md L556-L558 ("In case multiple Accessors are used
+ * within one kernel, the largest window size specified is taken") and
+ * Listing 9 (L961-L964) `convolve(cMask, SUM, [&] () { return cMask() *
+ * Input(cMask); })`, with the per-tap function chosen from a fixed set
+ * (reading c22):
+ *   out(x, y) = op over k = 0..n_inputs-1, yf, xf of
+ *               f(M_k(xf, yf), Read_k(x + ox_k + xf, y + oy_k + yf), c_k)
+ *   c_k = Read_k(x + ox_k, y + oy_k)           (accessor k's window centre)
+ *   f:  LOP_TAP_PRODUCT  M * v            (Listing 9's cMask() * Input(cMask))
+ *       LOP_TAP_ABSDIFF  M * |v - c_k|
+ *       LOP_TAP_SQDIFF   M * (v - c_k)^2
+ *       LOP_TAP_SQUARE   M * v^2
+ *   op: LOP_REDUCE_SUM over all taps; LOP_REDUCE_MIN / _MAX over the taps
+ *       with M_k != 0 (reading c18).
+ * inputs[k]: an Accessor (its own image, BoundaryCondition -- mode, window,
+ * constant -- and offset); masks[k]: its mask, of its BoundaryCondition's
+ * window size (odd, up to 31 x 31 each, 3844 taps in total).  The launch's
+ * halo is the largest window (L556-L558).  All images share the output's
+ * width / height / batch.
+ * dtypes: every input F32 with F32 masks -> F32 output (SUM accumulated in
+ * f32 in a fixed order: per accessor, per window row a left-to-right partial
+ * sum, rows top to bottom, accessors in order); or every input U8 with I32
+ * masks -> I32 output (exact integers; the worst-case magnitude must fit
+ * int32, else LOP_ERR_UNSUPPORTED).
+ * Kernel configuration: Algorithm 2 on B200 terms --
+ * see lop_alg2_select. */
+typedef enum {
+    LOP_TAP_PRODUCT = 0,
+    LOP_TAP_ABSDIFF = 1,
+    LOP_TAP_SQDIFF = 2,
+    LOP_TAP_SQUARE = 3
+} lop_tap_fn;
+#define LOP_MAX_ACCESSORS 4
+lop_status lop_local_execute(const lop_iteration_space *is, const lop_accessor *const *inputs,
+                             const lop_mask *const *masks, int32_t n_inputs, int32_t op,
+                             int32_t tap_fn, void *cuda_stream);
+
+/* Algorithm 2, the kernel-configuration heuristic, as a
+ * pure host function (no CUDA call; the library feeds it cudaOccupancy*
+ * figures).  cand[i] describes configuration i: threads per CTA, its tiling
+ * (block_x x block_y threads, each thread computing out_x x out_y outputs),
+ * whether it fits the device's resource limits (valid) and its occupancy
+ * (resident threads per SM / max threads per SM).  Lines 1-3: drop
+ * configurations whose thread count is not a multiple of simd_width or that
+ * are not valid; sort by descending occupancy, then ascending threads.
+ * Lines 4-17 (border handling, rx | ry > 0): among the configurations with
+ * the highest occupancy, take the one with the fewest threads in CTAs whose
+ * footprint (tile + window radii rx, ry) leaves the width x height image
+ * (ties keep the earlier one); the caller lists each thread count's tiling
+ * with y preferred (block_x = simd_width).  Lines 18-20 (no border
+ * handling): the first configuration (the caller lists x-preferred tilings).
+ * Returns the index chosen, -1 if none is valid; *border_threads (optional)
+ * receives its border-handling thread count. */
+typedef struct {
+    int32_t block_x, block_y;   /* threads */
+    int32_t out_x, out_y;       /* outputs per thread */
+    int32_t valid;              /* within the device's resource limits */
+    double occupancy;           /* 0..1 */
+} lop_config_candidate;
+int32_t lop_alg2_select(const lop_config_candidate *cand, int32_t n, int32_t simd_width,
+                        int32_t width, int32_t height, int32_t rx, int32_t ry,
+                        int64_t *border_threads);
+
 /* Mask builders (host only).
  * lop_mask_closeness: Eq. (1), float coefficients (Listing 4's mask[]).
  * lop_mask_gaussian:  binomial size x size (size odd; 1..11 for LOP_I32, 1..31

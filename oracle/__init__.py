@@ -88,6 +88,11 @@ def _load():
                                                  i32, dbl, i64, i64, vp, vp]
             lib.oracle_bilateral_f32_points.argtypes = [vp, i64, i64, i64, vp, i32, i32, dbl,
                                                         dbl, i32, dbl, vp, vp, i64, vp, vp]
+            pa = ctypes.POINTER(ctypes.c_void_p)
+            lib.oracle_local_f32.argtypes = [i32, pa, vp, i64, i64, pa, vp, vp, vp, vp, vp, vp,
+                                             i32, i32, i64, i64, vp, vp]
+            lib.oracle_local_u8.argtypes = [i32, pa, vp, i64, i64, pa, vp, vp, vp, vp, vp, vp,
+                                            i32, i32, i64, i64, vp, vp]
             _lib = lib
     return _lib
 
@@ -336,4 +341,52 @@ def bilateral_f32_points(img, sigma_d, sigma_r, mode, xs, ys, cval=0.0, size=Non
                                         mw, mh, float(sigma_d), float(sigma_r), _mode(mode),
                                         float(cval), _ptr(xs), _ptr(ys), len(xs), _ptr(out),
                                         _ptr(valid))
+    return out, valid.astype(bool)
+
+
+LOCAL_OPS = {"sum": 0, "min": 1, "max": 2}
+TAP_FNS = {"product": 0, "absdiff": 1, "sqdiff": 2, "square": 3}
+
+
+def local(imgs, masks, op="sum", fn="product", modes="clamp", cvals=0.0, offsets=None,
+          rows=None):
+    """Local operator over K accessors (N2; Listing 9):
+    out = op over k, taps of fn(M_k, Read_k(x+ox_k+xf, y+oy_k+yf), centre_k).
+    imgs: K images of one shape and dtype (float32 -> double result, uint8 ->
+    exact int64); masks: K 2D masks (odd sizes, float for f32, int for u8);
+    modes / cvals / offsets: one per accessor (or a single value for all)."""
+    K = len(imgs)
+    assert K == len(masks) and K >= 1
+    u8 = np.asarray(imgs[0]).dtype == np.uint8
+    dt = np.uint8 if u8 else np.float32
+    ims = [_img(im, dt) for im in imgs]
+    H, W = ims[0][0].shape
+    assert all(im.shape == (H, W) for im, _ in ims)
+    mdt = np.int32 if u8 else np.float64
+    ms = [np.ascontiguousarray(m, mdt) for m in masks]
+    modes = [modes] * K if isinstance(modes, (str, int)) else list(modes)
+    cvals = [cvals] * K if np.isscalar(cvals) else list(cvals)
+    offsets = [(0, 0)] * K if offsets is None else list(offsets)
+    img_ptrs = (ctypes.c_void_p * K)(*[im.ctypes.data for im, _ in ims])
+    m_ptrs = (ctypes.c_void_p * K)(*[m.ctypes.data for m in ms])
+    strides = np.array([s for _, s in ims], np.int64)
+    mws = np.array([m.shape[1] for m in ms], np.int32)
+    mhs = np.array([m.shape[0] for m in ms], np.int32)
+    oxs = np.array([o[0] for o in offsets], np.int32)
+    oys = np.array([o[1] for o in offsets], np.int32)
+    mds = np.array([_mode(md) for md in modes], np.int32)
+    y0, y1 = (0, H) if rows is None else rows
+    valid = np.empty((y1 - y0, W), np.uint8)
+    if u8:
+        cv = np.array([int(c) for c in cvals], np.int64)
+        out = np.empty((y1 - y0, W), np.int64)
+        fnc = _load().oracle_local_u8
+    else:
+        cv = np.array([float(c) for c in cvals], np.float64)
+        out = np.empty((y1 - y0, W), np.float64)
+        fnc = _load().oracle_local_f32
+    fnc(K, ctypes.cast(img_ptrs, ctypes.POINTER(ctypes.c_void_p)), _ptr(strides), W, H,
+        ctypes.cast(m_ptrs, ctypes.POINTER(ctypes.c_void_p)), _ptr(mws), _ptr(mhs), _ptr(oxs),
+        _ptr(oys), _ptr(mds), _ptr(cv), LOCAL_OPS[op], TAP_FNS[fn], y0, y1, _ptr(out),
+        _ptr(valid))
     return out, valid.astype(bool)

@@ -396,3 +396,133 @@ void oracle_bilateral_f32_points(const float *img, int64_t W, int64_t H, int64_t
         out[i] = bilateral_px(img, W, H, stride, cmask, mw, mh, sigma_d, sigma_r, mode, cval,
                               xs[i], ys[i], &valid[i]);
 }
+
+/* ------------------------------------------------------------------ */
+/* Local operator over several Accessors.            */
+/* "In case multiple Accessors are used within one */
+/* kernel, the largest window size specified is taken"; L160-L162 and */
+/* L315-L318: an Accessor reads its input through its own               */
+/* BoundaryCondition (mode, window) at an offset; Listing 9 (L961-L964):*/
+/*   output() = convolve(cMask, SUM, [&] () {                           */
+/*                  return cMask() * Input(cMask); });                  */
+/* -- a reduction over the mask's taps of a per-tap function.  Here K   */
+/* accessors k, each with its own mask M_k (size mw_k x mh_k, odd),     */
+/* offset (ox_k, oy_k), mode and constant; f from a fixed set           */
+/* (reading c22):                                                       */
+/*   fn 0 PRODUCT  f = M * v             (Listing 9's cMask()*Input())  */
+/*   fn 1 ABSDIFF  f = M * |v - c|       c = Read_k(x + ox_k, y + oy_k) */
+/*   fn 2 SQDIFF   f = M * (v - c)^2         (the accessor's own centre) */
+/*   fn 3 SQUARE   f = M * v^2                                          */
+/* and the reduction op 0 SUM (over all taps), 1 MIN, 2 MAX (over the    */
+/* taps with M != 0, reading c18):                                       */
+/*   out(x, y) = op_{k, yf, xf} f(M_k(xf, yf),                          */
+/*                  Read_k(x + ox_k + xf, y + oy_k + yf), c_k)           */
+/* Undefined mode: the output is valid iff no read of any accessor      */
+/* (its whole window, centre included) leaves its image (reading c9).   */
+/* f32 images: double arithmetic; u8 images: exact int64.               */
+/* ------------------------------------------------------------------ */
+static double tap_fn_f64(int fn, double M, double v, double c)
+{
+    switch (fn) {
+    case 1: return M * fabs(v - c);
+    case 2: return M * (v - c) * (v - c);
+    case 3: return M * v * v;
+    default: return M * v;
+    }
+}
+
+static int64_t tap_fn_i64(int fn, int64_t M, int64_t v, int64_t c)
+{
+    switch (fn) {
+    case 1: return M * (v > c ? v - c : c - v);
+    case 2: return M * (v - c) * (v - c);
+    case 3: return M * v * v;
+    default: return M * v;
+    }
+}
+
+static double local_px_f32(int K, const float *const *imgs, const int64_t *strides, int64_t W,
+                           int64_t H, const double *const *masks, const int *mws, const int *mhs,
+                           const int *oxs, const int *oys, const int *modes, const double *cvals,
+                           int op, int fn, int64_t x, int64_t y, uint8_t *valid)
+{
+    int undef = 0, first = 1;
+    double acc = 0.0;
+    for (int k = 0; k < K; ++k) {
+        const int m = mws[k] / 2, n = mhs[k] / 2;
+        const int64_t cx = x + oxs[k], cy = y + oys[k];
+        const double c = read_f32(imgs[k], W, H, strides[k], cx, cy, modes[k], cvals[k], &undef);
+        for (int yf = -n; yf <= n; ++yf)
+            for (int xf = -m; xf <= m; ++xf) {
+                const double M = masks[k][(yf + n) * mws[k] + (xf + m)];
+                const double v = read_f32(imgs[k], W, H, strides[k], cx + xf, cy + yf, modes[k],
+                                          cvals[k], &undef);
+                if (op == 0) {
+                    acc += tap_fn_f64(fn, M, v, c);
+                } else if (M != 0.0) {
+                    const double f = tap_fn_f64(fn, M, v, c);
+                    if (first || (op == 1 ? f < acc : f > acc)) acc = f;
+                    first = 0;
+                }
+            }
+    }
+    *valid = (uint8_t)!undef;
+    return acc;
+}
+
+static int64_t local_px_u8(int K, const uint8_t *const *imgs, const int64_t *strides, int64_t W,
+                           int64_t H, const int32_t *const *masks, const int *mws, const int *mhs,
+                           const int *oxs, const int *oys, const int *modes, const int64_t *cvals,
+                           int op, int fn, int64_t x, int64_t y, uint8_t *valid)
+{
+    int undef = 0, first = 1;
+    int64_t acc = 0;
+    for (int k = 0; k < K; ++k) {
+        const int m = mws[k] / 2, n = mhs[k] / 2;
+        const int64_t cx = x + oxs[k], cy = y + oys[k];
+        const int64_t c = read_u8(imgs[k], W, H, strides[k], cx, cy, modes[k], cvals[k], &undef);
+        for (int yf = -n; yf <= n; ++yf)
+            for (int xf = -m; xf <= m; ++xf) {
+                const int64_t M = masks[k][(yf + n) * mws[k] + (xf + m)];
+                const int64_t v = read_u8(imgs[k], W, H, strides[k], cx + xf, cy + yf, modes[k],
+                                          cvals[k], &undef);
+                if (op == 0) {
+                    acc += tap_fn_i64(fn, M, v, c);
+                } else if (M != 0) {
+                    const int64_t f = tap_fn_i64(fn, M, v, c);
+                    if (first || (op == 1 ? f < acc : f > acc)) acc = f;
+                    first = 0;
+                }
+            }
+    }
+    *valid = (uint8_t)!undef;
+    return acc;
+}
+
+void oracle_local_f32(int K, const float *const *imgs, const int64_t *strides, int64_t W,
+                      int64_t H, const double *const *masks, const int *mws, const int *mhs,
+                      const int *oxs, const int *oys, const int *modes, const double *cvals,
+                      int op, int fn, int64_t y0, int64_t y1, double *out, uint8_t *valid)
+{
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t y = y0; y < y1; ++y)
+        for (int64_t x = 0; x < W; ++x) {
+            int64_t o = (y - y0) * W + x;
+            out[o] = local_px_f32(K, imgs, strides, W, H, masks, mws, mhs, oxs, oys, modes, cvals,
+                                  op, fn, x, y, &valid[o]);
+        }
+}
+
+void oracle_local_u8(int K, const uint8_t *const *imgs, const int64_t *strides, int64_t W,
+                     int64_t H, const int32_t *const *masks, const int *mws, const int *mhs,
+                     const int *oxs, const int *oys, const int *modes, const int64_t *cvals,
+                     int op, int fn, int64_t y0, int64_t y1, int64_t *out, uint8_t *valid)
+{
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t y = y0; y < y1; ++y)
+        for (int64_t x = 0; x < W; ++x) {
+            int64_t o = (y - y0) * W + x;
+            out[o] = local_px_u8(K, imgs, strides, W, H, masks, mws, mhs, oxs, oys, modes, cvals,
+                                 op, fn, x, y, &valid[o]);
+        }
+}

@@ -34,7 +34,8 @@ _DT = {torch.uint8: _lib.LOP_U8, torch.int32: _lib.LOP_I32, torch.float32: _lib.
 VARIANTS = {"auto": _lib.LOP_VARIANT_AUTO, "generic": _lib.LOP_VARIANT_GENERIC,
             "tiled": _lib.LOP_VARIANT_TILED}
 
-__all__ = ["bilateral", "convolve", "convolve_chain", "gaussian", "sobel", "closeness_mask", "gaussian_mask",
+__all__ = ["bilateral", "convolve", "convolve_chain", "gaussian", "sobel", "local", "alg2_select",
+           "closeness_mask", "gaussian_mask",
            "sobel_mask", "set_variant", "get_variant", "launch_count", "reset_launch_count",
            "Pipeline", "LopError", "image_view", "MODES", "library_path"]
 
@@ -226,6 +227,71 @@ def global_reduce(x: torch.Tensor, op="sum", roi=None, out=None, work=None,
         _check(lib.lop_global_reduce_execute(ctypes.byref(is_), _REDUCE[op], out.data_ptr(),
                                              work.data_ptr(), _stream_handle(x, stream)))
     return out
+
+
+_TAP = {"product": _lib.LOP_TAP_PRODUCT, "absdiff": _lib.LOP_TAP_ABSDIFF,
+        "sqdiff": _lib.LOP_TAP_SQDIFF, "square": _lib.LOP_TAP_SQUARE}
+
+
+def local(inputs, masks, op="sum", fn="product", modes="clamp", constants=0.0, offsets=None,
+          out=None, roi=None, stream=None) -> torch.Tensor:
+    """Local operator over several Accessors with a per-tap function
+    (lop_local_execute; Listing 9):
+    out = op over k, taps of fn(M_k, Read_k(x+ox_k+xf, y+oy_k+yf), centre_k).
+    inputs: up to 4 CUDA images of one shape and dtype (float32 -> float32,
+    uint8 -> int32); masks: one 2D host mask per input (its window);
+    modes / constants / offsets: per input (or one value for all)."""
+    K = len(inputs)
+    if K != len(masks):
+        raise ValueError("one mask per input")
+    modes = [modes] * K if isinstance(modes, (str, int)) else list(modes)
+    constants = [constants] * K if np.isscalar(constants) else list(constants)
+    offsets = [(0, 0)] * K if offsets is None else list(offsets)
+    x0 = inputs[0]
+    mdt = _lib.LOP_F32 if x0.dtype == torch.float32 else _lib.LOP_I32
+    if out is None:
+        out = torch.empty(x0.shape, dtype=torch.float32 if x0.dtype == torch.float32 else torch.int32,
+                          device=x0.device)
+    keep, bcs, accs, ms = [], [], [], []
+    for k in range(K):
+        arr, m = _host_mask(masks[k], mdt)
+        bc = _lib.lop_boundary_condition()
+        bc.image = image_view(inputs[k])
+        bc.mode = _mode(modes[k])
+        bc.size_x, bc.size_y = m.size_x, m.size_y
+        bc.constant = float(constants[k])
+        keep += [arr, bc]
+        bcs.append(bc)
+        accs.append(_lib.lop_accessor(ctypes.pointer(bc), int(offsets[k][0]), int(offsets[k][1])))
+        ms.append(m)
+    acc_arr = (ctypes.POINTER(_lib.lop_accessor) * K)(*[ctypes.pointer(a) for a in accs])
+    m_arr = (ctypes.POINTER(_lib.lop_mask) * K)(*[ctypes.pointer(m) for m in ms])
+    is_ = _lib.lop_iteration_space()
+    is_.image = image_view(out)
+    if roi is not None:
+        is_.x0, is_.y0, is_.width, is_.height = (int(v) for v in roi)
+    with torch.cuda.device(x0.device):
+        _check(lib.lop_local_execute(ctypes.byref(is_), acc_arr, m_arr, K, _REDUCE[op], _TAP[fn],
+                                     _stream_handle(x0, stream)))
+    del keep
+    return out
+
+
+def alg2_select(candidates, width, height, rx, ry, simd_width=32):
+    """Algorithm 2 over candidate configurations, each a
+    dict(block_x, block_y, out_x=1, out_y=1, valid=True, occupancy);
+    returns (index, border_threads) -- the library's own selector."""
+    n = len(candidates)
+    arr = (_lib.lop_config_candidate * n)()
+    for a, c in zip(arr, candidates):
+        a.block_x, a.block_y = int(c["block_x"]), int(c["block_y"])
+        a.out_x, a.out_y = int(c.get("out_x", 1)), int(c.get("out_y", 1))
+        a.valid = int(bool(c.get("valid", True)))
+        a.occupancy = float(c["occupancy"])
+    bh = ctypes.c_int64(0)
+    i = lib.lop_alg2_select(ctypes.cast(arr, ctypes.c_void_p), n, int(simd_width), int(width),
+                            int(height), int(rx), int(ry), ctypes.byref(bh))
+    return i, bh.value
 
 
 def erode(x: torch.Tensor, size: int = 3, mode="clamp", constant=0.0, **kw) -> torch.Tensor:

@@ -19,6 +19,8 @@ LOP_VARIANT_AUTO, LOP_VARIANT_GENERIC, LOP_VARIANT_TILED = 0, 1, 2
 LOP_REDUCE_SUM, LOP_REDUCE_MIN, LOP_REDUCE_MAX = 0, 1, 2
 LOP_COMBINE_L2, LOP_COMBINE_L1, LOP_COMBINE_SUMSQ = 0, 1, 2
 LOP_GLOBAL_WORK_DOUBLES = 1025
+LOP_TAP_PRODUCT, LOP_TAP_ABSDIFF, LOP_TAP_SQDIFF, LOP_TAP_SQUARE = 0, 1, 2, 3
+LOP_MAX_ACCESSORS = 4
 
 c_i32, c_i64, c_dbl, c_flt, c_vp = (ctypes.c_int32, ctypes.c_int64, ctypes.c_double,
                                     ctypes.c_float, ctypes.c_void_p)
@@ -46,6 +48,11 @@ class lop_mask(ctypes.Structure):
                 ("shift", c_i32)]
 
 
+class lop_config_candidate(ctypes.Structure):
+    _fields_ = [("block_x", c_i32), ("block_y", c_i32), ("out_x", c_i32), ("out_y", c_i32),
+                ("valid", c_i32), ("occupancy", c_dbl)]
+
+
 class lop_iteration_space(ctypes.Structure):
     _fields_ = [("image", lop_image), ("x0", c_i32), ("y0", c_i32), ("width", c_i32),
                 ("height", c_i32)]
@@ -70,6 +77,12 @@ SIGNATURES = {
                                       ctypes.POINTER(lop_mask), c_i32, c_vp]),
     "lop_global_reduce_execute": (c_i32, [ctypes.POINTER(lop_iteration_space), c_i32, c_vp,
                                           c_vp, c_vp]),
+    "lop_local_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
+                                  ctypes.POINTER(ctypes.POINTER(lop_accessor)),
+                                  ctypes.POINTER(ctypes.POINTER(lop_mask)), c_i32, c_i32, c_i32,
+                                  c_vp]),
+    "lop_alg2_select": (c_i32, [c_vp, c_i32, c_i32, c_i32, c_i32, c_i32, c_i32,
+                                ctypes.POINTER(c_i64)]),
     "lop_mask_closeness": (c_i32, [c_flt, c_i32, c_i32, c_vp]),
     "lop_mask_gaussian": (c_i32, [c_i32, c_i32, c_vp, ctypes.POINTER(c_i32)]),
     "lop_mask_sobel": (c_i32, [c_i32, c_i32, c_vp]),

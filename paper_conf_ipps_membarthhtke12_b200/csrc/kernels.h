@@ -30,4 +30,8 @@ cudaError_t launch_global_reduce(const GlobalReduce &p, cudaStream_t stream);
 // Fused two-stage convolution; cudaErrorNotSupported if no instance matches.
 cudaError_t launch_conv_chain(const ConvChain &p, cudaStream_t stream);
 
+// Local operator over several accessors (local.cu): tiled (shared-memory
+// staging) or generic; the CTA shape from Algorithm 2 (select.cpp).
+cudaError_t launch_local(const LocalParams &p, bool tiled, cudaStream_t stream);
+
 }  // namespace lop

@@ -1,0 +1,379 @@
+// local.cu -- local operator over several Accessors with a per-tap function
+// (include/lop.h lop_local_execute):
+//   PAPER.md L556-L558  "In case multiple Accessors are used within one
+//                        kernel, the largest window size specified is taken"
+//   Listing 9 L961-L964 convolve(cMask, SUM, [&] () { return cMask() *
+//                        Input(cMask); }) -- a reduction over the mask's taps
+//                        of a per-tap function (reading c22: a fixed set).
+//   out(x, y) = op_{k, yf, xf} f(M_k(xf, yf), Read_k(x + ox_k + xf,
+//                                 y + oy_k + yf), Read_k(x + ox_k, y + oy_k))
+//
+// Two kernels with the same per-output arithmetic in the same order (so the
+// outputs are bit-identical, tested):
+//  * local_tiled_kernel: every accessor's footprint (tile + its own window +
+//    offset) is staged once into shared memory with the boundary resolved at
+//    staging time (interior CTAs: unchecked loads; border CTAs: per element,
+//    Table I) -- the B200 form of the paper's nine-region kernels (Fig. 3);
+//    a thread computes one column x 4 rows, so consecutive lanes read
+//    consecutive shared-memory words (no bank conflicts) and every staged row
+//    a thread loads serves up to 4 outputs.
+//  * local_generic_kernel: one thread per output, per-tap boundary resolution
+//    (interior CTAs skip it).
+// The CTA shape of both comes from Algorithm 2 (select.cpp): occupancy from
+// cudaOccupancyMaxActiveBlocksPerMultiprocessor, then the fewest threads in
+// border CTAs with y-preferred tilings.
+// Summation order (SUM, f32): per accessor, per window row a left-to-right
+// partial sum (first tap M*g, then FMA), rows folded top to bottom (FADD),
+// accessors folded in order (FADD).  MIN / MAX: exact, taps with M != 0.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <climits>
+#include <cmath>
+#include <cstring>
+#include <type_traits>
+
+#include "boundary.cuh"
+#include "kernels.h"
+#include "launch_cache.h"
+#include "lop_params.h"
+#include "select.h"
+
+namespace lop {
+
+namespace local {
+constexpr int OUT_Y = 4;                     // output rows per thread (tiled kernel)
+enum { FN_PRODUCT = 0, FN_ABSDIFF = 1, FN_SQDIFF = 2, FN_SQUARE = 3 };
+}  // namespace local
+
+// g(v, c) of the per-tap function f = M * g
+template <int FN>
+__device__ __forceinline__ float tap_g(float v, float c)
+{
+    if (FN == local::FN_ABSDIFF) return fabsf(__fsub_rn(v, c));
+    if (FN == local::FN_SQDIFF) { const float d = __fsub_rn(v, c); return __fmul_rn(d, d); }
+    if (FN == local::FN_SQUARE) return __fmul_rn(v, v);
+    return v;
+}
+template <int FN>
+__device__ __forceinline__ int tap_g(int v, int c)
+{
+    if (FN == local::FN_ABSDIFF) return abs(v - c);
+    if (FN == local::FN_SQDIFF) return (v - c) * (v - c);
+    if (FN == local::FN_SQUARE) return v * v;
+    return v;
+}
+
+// Per-output accumulator: SUM keeps (total, accessor sum, row partial);
+// MIN / MAX a running extreme initialised to the identity.
+template <typename V, int OP>
+struct LocalAccum {
+    V total, acck, rs;
+    __device__ __forceinline__ void init()
+    {
+        if constexpr (std::is_same<V, float>::value)
+            total = OP == RED_MIN ? INFINITY : (OP == RED_MAX ? -INFINITY : 0.0f);
+        else
+            total = OP == RED_MIN ? INT_MAX : (OP == RED_MAX ? INT_MIN : 0);
+        acck = rs = (V)0;
+    }
+    // tap xf of a window row (first: the row's first tap)
+    template <int FN>
+    __device__ __forceinline__ void tap(V M, V v, V c, bool first)
+    {
+        const V g = tap_g<FN>(v, c);
+        if (OP == RED_SUM) {
+            if (std::is_same<V, float>::value) rs = first ? __fmul_rn(M, g) : __fmaf_rn(M, g, rs);
+            else rs = first ? M * g : rs + M * g;
+        } else if (M != (V)0) {
+            const V f = std::is_same<V, float>::value ? (V)__fmul_rn(M, g) : M * g;
+            total = OP == RED_MIN ? min(total, f) : max(total, f);
+        }
+    }
+    __device__ __forceinline__ void end_row(bool first_row)
+    {
+        if (OP == RED_SUM) acck = first_row ? rs : (std::is_same<V, float>::value ? (V)__fadd_rn(acck, rs) : acck + rs);
+    }
+    __device__ __forceinline__ void end_accessor(bool first_acc)
+    {
+        if (OP == RED_SUM) total = first_acc ? acck : (std::is_same<V, float>::value ? (V)__fadd_rn(total, acck) : total + acck);
+    }
+};
+
+template <bool U8>
+__device__ __forceinline__ void local_store(const Common &c, int b, int x, int y, float vf, int vi)
+{
+    char *orow = c.out.data + (int64_t)b * c.out.bstride + (int64_t)y * c.out.stride;
+    if (U8) reinterpret_cast<int32_t *>(orow)[x] = vi;
+    else reinterpret_cast<float *>(orow)[x] = vf;
+}
+
+template <bool U8>
+__device__ __forceinline__ auto local_read(const LocalAcc &a, int b, int ix, int iy)
+{
+    if constexpr (U8) return read_u8(a.in, b, ix, iy, a.mode, a.cval_i);
+    else return read_f32(a.in, b, ix, iy, a.mode, a.cval_f);
+}
+
+// Is accessor a's footprint of output rectangle [x0, x0+w) x [y0, y0+h)
+// inside the image (global rows, columns)?  Then no boundary handling.
+__device__ __forceinline__ bool local_interior(const LocalAcc &a, int x0, int y0, int w, int h)
+{
+    const int ix0 = x0 + a.off_x - a.rx, iy0 = y0 + a.off_y - a.ry;
+    const int gy = iy0 + a.in.gy0;
+    return ix0 >= 0 && ix0 + w + 2 * a.rx <= a.in.W && gy >= 0 && gy + h + 2 * a.ry <= a.in.GH;
+}
+
+// ------------------------------------------------------------------ tiled
+template <bool U8, int OP, int FN>
+__global__ void __launch_bounds__(1024) local_tiled_kernel(const __grid_constant__ LocalParams p)
+{
+    using V = typename std::conditional<U8, int, float>::type;
+    constexpr int OY = local::OUT_Y;
+    extern __shared__ float4 smem4[];
+    V *sm = reinterpret_cast<V *>(smem4);
+    const Common &c = p.c;
+    const int tw = blockDim.x, th = OY * blockDim.y;
+    const int b = blockIdx.z;
+    const int tx0 = c.roi_x0 + blockIdx.x * tw, ty0 = c.roi_y0 + blockIdx.y * th;
+    const int roi_x1 = c.roi_x0 + c.roi_w, roi_y1 = c.roi_y0 + c.roi_h;
+    const int rows = min(th, roi_y1 - ty0);               // output rows of this tile
+    const int tid = threadIdx.y * blockDim.x + threadIdx.x, nthr = blockDim.x * blockDim.y;
+    // stage every accessor's footprint (only the rows the tile's outputs need)
+    int base = 0;
+    for (int k = 0; k < p.n; ++k) {
+        const LocalAcc &a = p.acc[k];
+        const int sw = tw + 2 * a.rx, sh = rows + 2 * a.ry;
+        const int ix0 = tx0 + a.off_x - a.rx, iy0 = ty0 + a.off_y - a.ry;
+        const bool interior = local_interior(a, tx0, ty0, tw, rows);
+        const char *fb = a.in.data + (int64_t)b * a.in.bstride;
+        for (int i = tid; i < sw * sh; i += nthr) {
+            const int r = i / sw, x = i - r * sw;
+            V v;
+            if (interior) {
+                const char *rp = fb + (int64_t)(iy0 + r) * a.in.stride;
+                if constexpr (U8) v = (int)__ldg(reinterpret_cast<const uint8_t *>(rp) + ix0 + x);
+                else v = __ldg(reinterpret_cast<const float *>(rp) + ix0 + x);
+            } else {
+                v = local_read<U8>(a, b, ix0 + x, iy0 + r);
+            }
+            sm[base + i] = v;
+        }
+        base += sw * sh;
+    }
+    __syncthreads();
+
+    const int x = tx0 + threadIdx.x;
+    const int y0 = OY * threadIdx.y;                       // first output row (tile-relative)
+    const int nj = min(OY, rows - y0);
+    if (x >= roi_x1 || nj <= 0) return;
+    LocalAccum<V, OP> acc[OY];
+#pragma unroll
+    for (int j = 0; j < OY; ++j) acc[j].init();
+    base = 0;
+    for (int k = 0; k < p.n; ++k) {
+        const LocalAcc &a = p.acc[k];
+        const int sw = tw + 2 * a.rx, sh = rows + 2 * a.ry;
+        const int sx = 2 * a.rx + 1;
+        const V *t = sm + base + threadIdx.x + a.rx;      // column of this thread's outputs
+        V cen[OY];
+#pragma unroll
+        for (int j = 0; j < OY; ++j) cen[j] = j < nj ? t[(y0 + j + a.ry) * sw] : (V)0;
+        const V *mk = (const V *)(U8 ? (const void *)(p.m.i + a.moff) : (const void *)(p.m.f + a.moff));
+        // staged row r feeds output j with window row yf = r - j - ry
+        for (int r = 0; r < nj + 2 * a.ry; ++r) {
+            const V *row = t + (y0 + r) * sw;
+            for (int xf = -a.rx; xf <= a.rx; ++xf) {
+                const V v = row[xf];
+#pragma unroll
+                for (int j = 0; j < OY; ++j) {
+                    const int yf = r - j - a.ry;
+                    if (j < nj && yf >= -a.ry && yf <= a.ry)
+                        acc[j].template tap<FN>(mk[(yf + a.ry) * sx + xf + a.rx], v, cen[j], xf == -a.rx);
+                }
+            }
+#pragma unroll
+            for (int j = 0; j < OY; ++j) {
+                const int yf = r - j - a.ry;
+                if (j < nj && yf >= -a.ry && yf <= a.ry) acc[j].end_row(yf == -a.ry);
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < OY; ++j) acc[j].end_accessor(k == 0);
+        base += sw * sh;
+    }
+#pragma unroll
+    for (int j = 0; j < OY; ++j)
+        if (j < nj) local_store<U8>(c, b, x, ty0 + y0 + j, (float)acc[j].total, (int)acc[j].total);
+}
+
+// ---------------------------------------------------------------- generic
+template <bool U8, int OP, int FN>
+__global__ void __launch_bounds__(1024) local_generic_kernel(const __grid_constant__ LocalParams p)
+{
+    using V = typename std::conditional<U8, int, float>::type;
+    const Common &c = p.c;
+    const int bx0 = c.roi_x0 + blockIdx.x * blockDim.x, by0 = c.roi_y0 + blockIdx.y * blockDim.y;
+    const int x = bx0 + threadIdx.x, y = by0 + threadIdx.y;
+    const int b = blockIdx.z;
+    if (x >= c.roi_x0 + c.roi_w || y >= c.roi_y0 + c.roi_h) return;
+    LocalAccum<V, OP> acc;
+    acc.init();
+    for (int k = 0; k < p.n; ++k) {
+        const LocalAcc &a = p.acc[k];
+        const int sx = 2 * a.rx + 1;
+        const int ix = x + a.off_x, iy = y + a.off_y;
+        // CTAs whose footprint stays inside the image skip the per-tap
+        // boundary resolution (Algorithm 2 counts the others' threads)
+        const bool interior = local_interior(a, bx0, by0, blockDim.x, blockDim.y);
+        const char *fb = a.in.data + (int64_t)b * a.in.bstride;
+        auto rd = [&](int xx, int yy) -> V {
+            if (interior) {
+                const char *rp = fb + (int64_t)yy * a.in.stride;
+                if constexpr (U8) return (int)__ldg(reinterpret_cast<const uint8_t *>(rp) + xx);
+                else return __ldg(reinterpret_cast<const float *>(rp) + xx);
+            }
+            return local_read<U8>(a, b, xx, yy);
+        };
+        const V cen = rd(ix, iy);
+        const V *mk = (const V *)(U8 ? (const void *)(p.m.i + a.moff) : (const void *)(p.m.f + a.moff));
+        for (int yf = -a.ry; yf <= a.ry; ++yf) {
+            for (int xf = -a.rx; xf <= a.rx; ++xf)
+                acc.template tap<FN>(mk[(yf + a.ry) * sx + xf + a.rx], rd(ix + xf, iy + yf), cen, xf == -a.rx);
+            acc.end_row(yf == -a.ry);
+        }
+        acc.end_accessor(k == 0);
+    }
+    local_store<U8>(c, b, x, y, (float)acc.total, (int)acc.total);
+}
+
+// --------------------------------------------------------------- launcher
+namespace {
+
+size_t tiled_smem(const LocalParams &p, int bx, int by)
+{
+    size_t n = 0;
+    for (int k = 0; k < p.n; ++k)
+        n += (size_t)(bx + 2 * p.acc[k].rx) * (local::OUT_Y * by + 2 * p.acc[k].ry);
+    return n * 4;
+}
+
+// Algorithm 2 over the thread counts 32, 64, ..., 1024 (multiples of the
+// SIMD width): tiling y-preferred (32 x T/32) with border handling, x-preferred
+// (T x 1) without; resource limits from the kernel's attributes and the
+// device's opt-in shared memory; occupancy from the CUDA occupancy API.
+template <typename K>
+cudaError_t choose_config(K kernel, const LocalParams &p, bool tiled, int &bx, int &by)
+{
+    const int dev = current_device();
+    cudaFuncAttributes fa;
+    cudaError_t e = cudaFuncGetAttributes(&fa, kernel);
+    int smem_max = 0, max_thr_sm = 0;
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&smem_max, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&max_thr_sm, cudaDevAttrMaxThreadsPerMultiProcessor, dev);
+    if (e != cudaSuccess) return e;
+    int fx = 0, fy = 0;                                   // footprint radii (window + offset)
+    for (int k = 0; k < p.n; ++k) {
+        fx = max(fx, p.acc[k].rx + abs(p.acc[k].off_x));
+        fy = max(fy, p.acc[k].ry + abs(p.acc[k].off_y));
+    }
+    const bool border = fx > 0 || fy > 0;
+    lop_config_candidate cand[32];
+    int n = 0;
+    for (int t = 32; t <= 1024; t += 32) {
+        lop_config_candidate &cd = cand[n++];
+        cd.block_x = border ? 32 : t;
+        cd.block_y = border ? t / 32 : 1;
+        cd.out_x = 1;
+        cd.out_y = tiled ? local::OUT_Y : 1;
+        const size_t smem = tiled ? tiled_smem(p, cd.block_x, cd.block_y) : 0;
+        cd.valid = t <= fa.maxThreadsPerBlock && smem <= (size_t)smem_max;
+        cd.occupancy = 0.0;
+        if (cd.valid) {
+            if (smem > 48 * 1024) {
+                e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+                if (e != cudaSuccess) return e;
+            }
+            int blocks = 0;
+            e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks, kernel, t, smem);
+            if (e != cudaSuccess) return e;
+            cd.occupancy = (double)blocks * t / max_thr_sm;
+            cd.valid = blocks > 0;
+        }
+    }
+    const int i = alg2_select(cand, n, 32, p.c.roi_w, p.c.roi_h, fx, fy, nullptr);
+    if (i < 0) return cudaErrorInvalidConfiguration;
+    bx = cand[i].block_x;
+    by = cand[i].block_y;
+    return cudaSuccess;
+}
+
+template <bool U8, int OP, int FN>
+cudaError_t launch_local_t(const LocalParams &p, bool tiled, cudaStream_t stream)
+{
+    // configuration cache: the last geometry per (thread, instance)
+    struct Key { int dev, w, h, batch, n, tiled; int r[4 * kLocalMaxAcc]; };
+    static thread_local Key last{};
+    static thread_local int last_bx = 0, last_by = 0;
+    Key key{};
+    key.dev = current_device(); key.w = p.c.roi_w; key.h = p.c.roi_h; key.batch = p.c.batch;
+    key.n = p.n; key.tiled = tiled;
+    for (int k = 0; k < p.n; ++k) {
+        key.r[4 * k] = p.acc[k].rx; key.r[4 * k + 1] = p.acc[k].ry;
+        key.r[4 * k + 2] = p.acc[k].off_x; key.r[4 * k + 3] = p.acc[k].off_y;
+    }
+    int bx = 0, by = 0;
+    if (last_bx && !memcmp(&key, &last, sizeof key)) {
+        bx = last_bx; by = last_by;
+    } else {
+        cudaError_t e = tiled ? choose_config(local_tiled_kernel<U8, OP, FN>, p, true, bx, by)
+                              : choose_config(local_generic_kernel<U8, OP, FN>, p, false, bx, by);
+        if (e != cudaSuccess) return e;
+        last = key; last_bx = bx; last_by = by;
+    }
+    if (tiled) {
+        const size_t smem = tiled_smem(p, bx, by);
+        static PerDevice configured;
+        cudaError_t e = ensure_smem(local_tiled_kernel<U8, OP, FN>, smem, configured);
+        if (e != cudaSuccess) return e;
+        dim3 grid((p.c.roi_w + bx - 1) / bx, (p.c.roi_h + local::OUT_Y * by - 1) / (local::OUT_Y * by),
+                  p.c.batch);
+        local_tiled_kernel<U8, OP, FN><<<grid, dim3(bx, by), smem, stream>>>(p);
+    } else {
+        dim3 grid((p.c.roi_w + bx - 1) / bx, (p.c.roi_h + by - 1) / by, p.c.batch);
+        local_generic_kernel<U8, OP, FN><<<grid, dim3(bx, by), 0, stream>>>(p);
+    }
+    return cudaGetLastError();
+}
+
+template <bool U8, int OP>
+cudaError_t launch_local_op(const LocalParams &p, bool tiled, cudaStream_t s)
+{
+    switch (p.fn) {
+    case local::FN_PRODUCT: return launch_local_t<U8, OP, local::FN_PRODUCT>(p, tiled, s);
+    case local::FN_ABSDIFF: return launch_local_t<U8, OP, local::FN_ABSDIFF>(p, tiled, s);
+    case local::FN_SQDIFF: return launch_local_t<U8, OP, local::FN_SQDIFF>(p, tiled, s);
+    case local::FN_SQUARE: return launch_local_t<U8, OP, local::FN_SQUARE>(p, tiled, s);
+    default: return cudaErrorInvalidValue;
+    }
+}
+
+template <bool U8>
+cudaError_t launch_local_u8(const LocalParams &p, bool tiled, cudaStream_t s)
+{
+    switch (p.op) {
+    case RED_SUM: return launch_local_op<U8, RED_SUM>(p, tiled, s);
+    case RED_MIN: return launch_local_op<U8, RED_MIN>(p, tiled, s);
+    case RED_MAX: return launch_local_op<U8, RED_MAX>(p, tiled, s);
+    default: return cudaErrorInvalidValue;
+    }
+}
+
+}  // namespace
+
+cudaError_t launch_local(const LocalParams &p, bool tiled, cudaStream_t stream)
+{
+    return p.u8 ? launch_local_u8<true>(p, tiled, stream) : launch_local_u8<false>(p, tiled, stream);
+}
+
+}  // namespace lop

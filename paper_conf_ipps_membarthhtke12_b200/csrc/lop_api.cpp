@@ -767,4 +767,95 @@ lop_status lop_convolve_chain_execute(const lop_iteration_space *is, const lop_a
     return launched(e, "conv_chain launch");
 }
 
+// ------------------------------------- local operator over several accessors
+lop_status lop_local_execute(const lop_iteration_space *is, const lop_accessor *const *inputs,
+                             const lop_mask *const *masks, int32_t n_inputs, int32_t op,
+                             int32_t tap_fn, void *cuda_stream)
+{
+    if (!inputs || !masks) return fail(LOP_ERR_INVALID, "inputs / masks is NULL");
+    if (n_inputs < 1 || n_inputs > LOP_MAX_ACCESSORS)
+        return fail(LOP_ERR_INVALID, "n_inputs %d outside 1..%d", n_inputs, LOP_MAX_ACCESSORS);
+    if (op != LOP_REDUCE_SUM && op != LOP_REDUCE_MIN && op != LOP_REDUCE_MAX)
+        return fail(LOP_ERR_INVALID, "unknown reduction %d (SUM, MIN, MAX)", op);
+    if (tap_fn < LOP_TAP_PRODUCT || tap_fn > LOP_TAP_SQUARE)
+        return fail(LOP_ERR_INVALID, "unknown tap function %d", tap_fn);
+    static thread_local lop::LocalParams p;
+    p.n = n_inputs;
+    p.op = op == LOP_REDUCE_SUM ? lop::RED_SUM : (op == LOP_REDUCE_MIN ? lop::RED_MIN : lop::RED_MAX);
+    p.fn = tap_fn;
+    int taps = 0, rx = 0, ry = 0;
+    bool any_tap = false;
+    double bound = 0.0;                               // worst-case |out| (integer path)
+    const double gmax = tap_fn == LOP_TAP_SQDIFF || tap_fn == LOP_TAP_SQUARE ? 255.0 * 255.0 : 255.0;
+    for (int k = 0; k < n_inputs; ++k) {
+        Prepared pp;
+        lop_status st = prepare(is, inputs[k], pp);
+        if (st) return fail(st, "accessor %d: %s", k, lop_last_error());
+        const lop::Common &c = pp.c;
+        const int32_t idt = inputs[k]->bc->image.dtype;
+        if (k == 0) {
+            p.c = c;
+            const int32_t odt = is->image.dtype;
+            if (idt == LOP_F32 && odt == LOP_F32) p.u8 = 0;
+            else if (idt == LOP_U8 && odt == LOP_I32) p.u8 = 1;
+            else return fail(LOP_ERR_INVALID, "unsupported dtype combination %d -> %d (F32 -> F32, U8 -> I32)",
+                             idt, odt);
+        } else if ((idt == LOP_U8) != (p.u8 == 1)) {
+            return fail(LOP_ERR_INVALID, "accessor %d: every input must have the same dtype", k);
+        }
+        if (c.rx > lop::kLocalMaxR || c.ry > lop::kLocalMaxR)
+            return fail(LOP_ERR_UNSUPPORTED, "accessor %d: window larger than 31 x 31", k);
+        const lop_mask *m = masks[k];
+        const int sx = 2 * c.rx + 1, sy = 2 * c.ry + 1;
+        if (!m || !m->coeffs) return fail(LOP_ERR_INVALID, "mask %d is NULL", k);
+        if (m->size_x != sx || m->size_y != sy)
+            return fail(LOP_ERR_INVALID, "mask %d is %d x %d, its accessor's window %d x %d", k,
+                        m->size_x, m->size_y, sx, sy);
+        if (m->dtype != (p.u8 ? LOP_I32 : LOP_F32) || m->shift != 0)
+            return fail(LOP_ERR_INVALID, "mask %d: %s images need %s masks with shift 0", k,
+                        p.u8 ? "U8" : "F32", p.u8 ? "I32" : "F32");
+        if (taps + sx * sy > lop::kLocalMaxTaps)
+            return fail(LOP_ERR_UNSUPPORTED, "masks have more than %d taps in total", lop::kLocalMaxTaps);
+        lop::LocalAcc &a = p.acc[k];
+        a.in = c.in;
+        a.off_x = c.off_x;
+        a.off_y = c.off_y;
+        a.mode = c.mode;
+        a.rx = c.rx;
+        a.ry = c.ry;
+        a.cval_f = c.cval_f;
+        a.cval_i = c.cval_i;
+        a.moff = taps;
+        double l1 = 0.0, mx = 0.0;
+        for (int i = 0; i < sx * sy; ++i) {
+            if (p.u8) {
+                const int32_t v = static_cast<const int32_t *>(m->coeffs)[i];
+                p.m.i[taps + i] = v;
+                any_tap |= v != 0;
+                l1 += std::fabs((double)v);
+                mx = std::max(mx, std::fabs((double)v));
+            } else {
+                const float v = static_cast<const float *>(m->coeffs)[i];
+                if (!std::isfinite(v)) return fail(LOP_ERR_INVALID, "mask %d coefficient %d not finite", k, i);
+                p.m.f[taps + i] = v;
+                any_tap |= v != 0.0f;
+            }
+        }
+        bound += op == LOP_REDUCE_SUM ? l1 * gmax : 0.0;
+        if (op != LOP_REDUCE_SUM) bound = std::max(bound, mx * gmax);
+        taps += sx * sy;
+        rx = std::max(rx, c.rx);
+        ry = std::max(ry, c.ry);
+    }
+    if (op != LOP_REDUCE_SUM && !any_tap)
+        return fail(LOP_ERR_INVALID, "MIN / MAX need at least one non-zero mask coefficient");
+    if (p.u8 && bound >= 2147483647.0)
+        return fail(LOP_ERR_UNSUPPORTED, "integer masks too large: the result may overflow int32");
+    p.c.rx = rx;                                     // the largest window (L556-L558)
+    p.c.ry = ry;
+    const bool tiled = g_variant != LOP_VARIANT_GENERIC;
+    return launched(lop::launch_local(p, tiled, static_cast<cudaStream_t>(cuda_stream)),
+                    "local launch");
+}
+
 }  // extern "C"

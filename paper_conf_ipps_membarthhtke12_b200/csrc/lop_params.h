@@ -171,4 +171,29 @@ struct ConvChain {
     ChainPlan plan;
 };
 
+// Local operator over several Accessors with a per-tap function (local.cu;
+// SURVEY §8(f) N2, Listing 9).  Accessor k reads its own
+// image through its own boundary condition at its own offset; its mask
+// occupies m[moff .. moff + (2ry+1)(2rx+1)).  c.rx / c.ry: the largest radii
+// (the launch's halo).  op: RED_SUM / RED_MIN / RED_MAX; fn: LOP_TAP_*.
+constexpr int kLocalMaxAcc = 4;
+constexpr int kLocalMaxR = 15;                                // each mask up to 31 x 31
+constexpr int kLocalMaxTaps = 3844;                           // all masks together
+struct LocalAcc {
+    Geom in;
+    int32_t off_x, off_y, mode, rx, ry;
+    float cval_f;
+    int32_t cval_i;
+    int32_t moff;
+};
+struct LocalParams {
+    Common c;                    // output, ROI, batch, largest radii
+    int32_t n, op, fn, u8;
+    LocalAcc acc[kLocalMaxAcc];
+    union {
+        float f[kLocalMaxTaps];
+        int32_t i[kLocalMaxTaps];
+    } m;
+};
+
 }  // namespace lop

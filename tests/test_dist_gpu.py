@@ -48,8 +48,9 @@ def _worker(rank, world, port, q):
             for sigma_r in (5.0, 0.1):
                 band = ldist.Bands(H, W, world, rank, 6, device="cuda", mode=mode)
                 assert band.staged()
-                band.fill(lambda a, b: synthetic.angio(H, W, seed=SEED, device="cuda",
-                                                       row_range=(a, b)))
+                # rows drawn on the host (the CPU and CUDA noise generators differ),
+                # so the oracle below sees the same image
+                band.fill(lambda a, b: synthetic.angio(H, W, seed=SEED, row_range=(a, b)).cuda())
                 band.top.fill_(float("nan"))           # must be overwritten by the exchange
                 band.bottom.fill_(float("nan"))
                 s = torch.cuda.Stream()                # a side stream
@@ -57,7 +58,7 @@ def _worker(rank, world, port, q):
                 out = ldist.bilateral_bands(lop, band, 3.0, sigma_r, mode, constant=0.5,
                                             size=13, stream=s)
                 s.synchronize()
-                res[(mode, sigma_r)] = (band.y0, out.cpu())
+                res[(mode, sigma_r)] = (band.y0, out.cpu().numpy())   # by value
         q.put((rank, res, lop.launch_count()))
     finally:
         dist.destroy_process_group()
@@ -85,7 +86,7 @@ def test_bands_cuda_kernels_on_several_ranks_match_oracle(world):
         for sigma_r in (5.0, 0.1):
             bands = [got[r][(mode, sigma_r)] for r in range(world)]
             assert [b[0] for b in bands] == [H * r // world for r in range(world)]
-            full = torch.cat([b[1] for b in bands]).numpy()
+            full = np.concatenate([b[1] for b in bands])
             ref, valid = oracle.bilateral_f32(img.numpy(), 3.0, sigma_r, mode, cval=0.5, size=13)
             sel = valid if mode == "undefined" else np.ones_like(valid)
             err = float(np.abs(full[sel] - ref[sel]).max())
