@@ -659,14 +659,20 @@ def conv_extras(lop, synthetic, dev, stream, hbm, img, timed):
     mid_f = torch.empty_like(img)
     mid_u = torch.empty_like(u8)
     cases += [
-        ("chain_gauss5_sobel3_f32_fused",
+        ("chain_gauss5_sobel3_f32",
          lambda k, s: lop.convolve_chain(f_in[k], gf, sxf, "clamp", out=f_out[k], stream=s), 8),
+        ("chain_gauss5_sobel3_f32_fused_kernel",
+         lambda k, s: lop.convolve_chain(f_in[k], gf, sxf, "clamp", out=f_out[k], stream=s,
+                                         fused=True), 8),
         ("chain_gauss5_sobel3_f32_two_pass",
          lambda k, s: lop.convolve(lop.convolve(f_in[k], gf, "clamp", out=mid_f, stream=s), sxf,
                                    "clamp", out=f_out[k], stream=s), 8),
-        ("chain_gauss5_sobel3_u8_i32_fused",
+        ("chain_gauss5_sobel3_u8_i32",
          lambda k, s: lop.convolve_chain(u_in[k], gi, sxi, "clamp", shift1=gk, out=i_out[k],
                                          stream=s), 5),
+        ("chain_gauss5_sobel3_u8_i32_fused_kernel",
+         lambda k, s: lop.convolve_chain(u_in[k], gi, sxi, "clamp", shift1=gk, out=i_out[k],
+                                         stream=s, fused=True), 5),
         ("chain_gauss5_sobel3_u8_i32_two_pass",
          lambda k, s: lop.convolve(lop.convolve(u_in[k], gi, "clamp", shift=gk, out=mid_u,
                                                 stream=s), sxi, "clamp", out=i_out[k], stream=s),
@@ -685,6 +691,20 @@ def conv_extras(lop, synthetic, dev, stream, hbm, img, timed):
                        lop.sobel(f_in[k], 1, "clamp", out=mid_f, stream=s)), 8),
         ("sobel_magnitude_l1_u8_i32_fused",
          lambda k, s: lop.sobel_magnitude(u_in[k], "clamp", out=i_out[k], stream=s), 5)]
+    # local operator over two accessors (N2; Listing 9): two
+    # consecutive frames, SUM of PRODUCT with a 5x5 and a 3x3 mask (a spatio-temporal
+    # average), and MAX of ABSDIFF on u8 -> i32 (local contrast of two frames)
+    f_in_b = [img.clone() for _ in range(sets)]
+    u_in_b = [u8.clone() for _ in range(sets)]
+    m5 = np.full((5, 5), 0.5 / 25, np.float32)
+    m3 = np.full((3, 3), 0.5 / 9, np.float32)
+    cases += [
+        ("local_2acc_sum_product_f32",
+         lambda k, s: lop.local([f_in[k], f_in_b[k]], [m5, m3], "sum", "product", "clamp",
+                                out=f_out[k], stream=s), 12),
+        ("local_2acc_max_absdiff_u8_i32",
+         lambda k, s: lop.local([u_in[k], u_in_b[k]], [np.ones((3, 3), np.int32)] * 2, "max",
+                                "absdiff", "clamp", out=i_out[k], stream=s), 6)]
     # global operator (sum of all pixels, deterministic two-level reduction)
     gres = torch.empty(1, dtype=torch.float64, device=dev)
     gwork = torch.zeros(1025, dtype=torch.float64, device=dev)     # LOP_GLOBAL_WORK_DOUBLES

@@ -175,6 +175,20 @@ lop_status lop_convolve_execute(const lop_iteration_space *is, const lop_accesso
 lop_status lop_convolve_chain_execute(const lop_iteration_space *is, const lop_accessor *in,
                                       const lop_mask *first, const lop_mask *second,
                                       void *cuda_stream);
+/* The same chain with a caller-owned device workspace of at least
+ * lop_convolve_chain_workspace_bytes() bytes (the intermediate image, whole
+ * input extent, input dtype, 16-B aligned rows): the library then runs the
+ * route measured faster on B200 -- two lop_convolve_execute passes through the
+ * workspace, whose intermediate stays in L2 (DESIGN.md §6 "Fused chain") --
+ * with a result bit-identical to lop_convolve_chain_execute.  A NULL or too
+ * small workspace runs the fused kernel.  Two kernel launches. */
+lop_status lop_convolve_chain_workspace_bytes(const lop_iteration_space *is, const lop_accessor *in,
+                                              const lop_mask *first, const lop_mask *second,
+                                              int64_t *bytes);
+lop_status lop_convolve_chain_execute_ws(const lop_iteration_space *is, const lop_accessor *in,
+                                         const lop_mask *first, const lop_mask *second,
+                                         void *d_workspace, int64_t workspace_bytes,
+                                         void *cuda_stream);
 
 /* Local reduction over a mask domain -- Listing 9's
  * convolve(mask, <reduction>, f) (L956-L967) with the MIN / MAX reductions

@@ -175,11 +175,30 @@ def convolve(x: torch.Tensor, mask, mode="clamp", constant=0.0, shift=0, out=Non
                     lambda is_, acc, s: lib.lop_convolve_execute(is_, acc, ctypes.byref(m), s))
 
 
+_WORKSPACE = {}
+
+
+def _workspace(device, stream_handle: int, nbytes: int) -> torch.Tensor:
+    """A cached byte buffer of at least nbytes per (device, stream): calls on
+    one stream are ordered, so reusing its buffer is safe (grown on demand)."""
+    key = (torch.device(device).index, int(stream_handle))
+    ws = _WORKSPACE.get(key)
+    if ws is None or ws.numel() < nbytes:
+        if ws is not None:                   # growing: the old buffer may still be in use
+            torch.cuda.synchronize(device)
+        ws = torch.empty(max(nbytes, 1), dtype=torch.uint8, device=device)
+        _WORKSPACE[key] = ws
+    return ws
+
+
 def convolve_chain(x: torch.Tensor, first, second, mode="clamp", constant=0.0, shift1=0,
                    shift2=0, out=None, out_dtype=None, roi=None, offset=(0, 0),
-                   stream=None) -> torch.Tensor:
-    """Fused second (*) (first (*) x) in one pass (e.g. Gaussian -> Sobel); equal
-    bit for bit to two convolve() calls (u8: the intermediate is u8)."""
+                   stream=None, fused=False) -> torch.Tensor:
+    """second (*) (first (*) x) (e.g. Gaussian -> Sobel), equal bit for bit to
+    two convolve() calls (u8: the intermediate is u8).  Default: the library
+    picks the faster route with a cached workspace (lop_convolve_chain_execute_ws:
+    two passes through L2 on B200); fused=True: the one-pass fused kernel
+    (lop_convolve_chain_execute)."""
     mdt = _lib.LOP_F32 if x.dtype == torch.float32 else _lib.LOP_I32
     a1, m1 = _host_mask(first, mdt)
     a2, m2 = _host_mask(second, mdt)
@@ -187,9 +206,21 @@ def convolve_chain(x: torch.Tensor, first, second, mode="clamp", constant=0.0, s
     if out is None:
         out = torch.empty(x.shape, dtype=out_dtype or x.dtype, device=x.device)
     size = (m1.size_x + m2.size_x - 1, m1.size_y + m2.size_y - 1)
-    return _execute("chain", x, out, mode, constant, size, roi, offset, stream, (0, 0, 0, 0),
-                    lambda is_, acc, s: lib.lop_convolve_chain_execute(
-                        is_, acc, ctypes.byref(m1), ctypes.byref(m2), s))
+    if fused:
+        return _execute("chain", x, out, mode, constant, size, roi, offset, stream, (0, 0, 0, 0),
+                        lambda is_, acc, s: lib.lop_convolve_chain_execute(
+                            is_, acc, ctypes.byref(m1), ctypes.byref(m2), s))
+
+    def call(is_, acc, s):
+        nb = ctypes.c_int64(0)
+        st = lib.lop_convolve_chain_workspace_bytes(is_, acc, ctypes.byref(m1), ctypes.byref(m2),
+                                                    ctypes.byref(nb))
+        if st != _lib.LOP_OK:
+            return st
+        ws = _workspace(x.device, s or 0, nb.value)
+        return lib.lop_convolve_chain_execute_ws(is_, acc, ctypes.byref(m1), ctypes.byref(m2),
+                                                 ws.data_ptr(), nb.value, s)
+    return _execute("chain", x, out, mode, constant, size, roi, offset, stream, (0, 0, 0, 0), call)
 
 
 _REDUCE = {"sum": _lib.LOP_REDUCE_SUM, "min": _lib.LOP_REDUCE_MIN, "max": _lib.LOP_REDUCE_MAX}

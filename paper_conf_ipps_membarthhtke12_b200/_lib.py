@@ -69,6 +69,14 @@ SIGNATURES = {
     "lop_convolve_chain_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
                                            ctypes.POINTER(lop_accessor), ctypes.POINTER(lop_mask),
                                            ctypes.POINTER(lop_mask), c_vp]),
+    "lop_convolve_chain_workspace_bytes": (c_i32, [ctypes.POINTER(lop_iteration_space),
+                                                   ctypes.POINTER(lop_accessor),
+                                                   ctypes.POINTER(lop_mask),
+                                                   ctypes.POINTER(lop_mask),
+                                                   ctypes.POINTER(c_i64)]),
+    "lop_convolve_chain_execute_ws": (c_i32, [ctypes.POINTER(lop_iteration_space),
+                                              ctypes.POINTER(lop_accessor), ctypes.POINTER(lop_mask),
+                                              ctypes.POINTER(lop_mask), c_vp, c_i64, c_vp]),
     "lop_reduce_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
                                    ctypes.POINTER(lop_accessor), ctypes.POINTER(lop_mask),
                                    c_i32, c_vp]),

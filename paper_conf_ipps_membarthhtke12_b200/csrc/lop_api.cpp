@@ -231,6 +231,33 @@ lop_status prepare(const lop_iteration_space *is, const lop_accessor *in, Prepar
                       (int64_t)c.roi_y0 + c.roi_h - 1 + c.off_y + c.ry);
 }
 
+// Bilateral kernel choice (the paper's configuration
+// exploration, §V-D / Fig. 4): the symmetric pair-sharing kernel
+// (84 exps / px at 13x13, but warps stream rows with an R-row warm-up and
+// 2 x ceil(R/4) halo lanes) against the unshared separable kernel (168 exps /
+// px, no warm-up), from the B200 sweep profiles/r02/sweep_bilateral_pair_vs_sep.jsonl
+// (tools/sweep_bilateral.py): pair wins on small launches (latency-bound,
+// fewer exps per warp step) and on large ones with windows of 7x7 and up;
+// the unshared kernel in between and for 3x3 / 5x5 beyond 768^2 / 512^2.
+// Keyed to the WHOLE launch's work -- width x GLOBAL height x frames, never
+// the iteration space or the band -- so ROI launches, row-band views (every
+// rank of a band split) and pipeline chunks of one image take the same kernel
+// as the whole-image call and stay bit-identical to it.  (A batch of frames
+// and the same frames launched one by one may differ; both meet the 1e-5
+// contract.)
+int pair_preferred(const lop::Common &c, int dflt)
+{
+    if (!dflt) return 0;
+    const double px = (double)c.in.W * (double)c.in.GH * (double)c.batch;
+    const int r = c.rx;
+    static const double lo[8] = {0, 768.0 * 768, 512.0 * 512, 512.0 * 512, 384.0 * 384,
+                                 256.0 * 256, 256.0 * 256, 256.0 * 256};   // pair at or below
+    static const double hi[8] = {0, 1e300, 1e300, 4096.0 * 4096, 3072.0 * 3072,
+                                 3072.0 * 3072, 2048.0 * 2048, 2048.0 * 2048};  // pair at or above
+    if (r < 1 || r > 7) return dflt;
+    return px <= lo[r] || px >= hi[r] ? 1 : 0;
+}
+
 lop_status launched(cudaError_t e, const char *what)
 {
     if (e != cudaSuccess) return cuda_fail(e, what);
@@ -410,8 +437,9 @@ lop_status lop_bilateral_execute(const lop_iteration_space *is, const lop_access
     if (const char *env = std::getenv("LOP_BILATERAL_SCALED")) scaled = std::atoi(env) != 0;
     if (scaled) npoly = 0;
     // symmetric pair-sharing: square separable windows, scaled
-    // exponent; LOP_BILATERAL_PAIR overrides
-    int pair = kDefaultPair;
+    // exponent, chosen per launch by the measured configuration space
+    // (pair_preferred); LOP_BILATERAL_PAIR overrides
+    int pair = pair_preferred(c, kDefaultPair);
     if (const char *env = std::getenv("LOP_BILATERAL_PAIR")) pair = std::atoi(env) != 0;
     pair = pair && sepform && scaled && c.rx == c.ry && c.rx >= 1 && c.rx <= lop::kTiledMaxRX;
     const double alpha_d = std::sqrt(kLog2e / (2.0 * (double)sigma_r * (double)sigma_r));
@@ -731,9 +759,12 @@ lop_status chain_stage(const lop::Common &c, const lop_mask *m, int32_t img_dtyp
 }
 }  // namespace
 
-lop_status lop_convolve_chain_execute(const lop_iteration_space *is, const lop_accessor *in,
-                                      const lop_mask *first, const lop_mask *second,
-                                      void *cuda_stream)
+namespace {
+// Shared validation of the chain calls: both stages factored, the accessor's
+// window = the combined footprint, whole images.
+lop_status chain_prepare(const lop_iteration_space *is, const lop_accessor *in,
+                         const lop_mask *first, const lop_mask *second, Prepared &pp,
+                         lop::ConvChain &p)
 {
     if (!first || !second) return fail(LOP_ERR_INVALID, "mask is NULL");
     if (in && in->bc &&
@@ -743,7 +774,6 @@ lop_status lop_convolve_chain_execute(const lop_iteration_space *is, const lop_a
                     "boundary condition window %d x %d must be the combined footprint %d x %d",
                     in->bc->size_x, in->bc->size_y, first->size_x + second->size_x - 1,
                     first->size_y + second->size_y - 1);
-    Prepared pp;
     lop_status st = prepare(is, in, pp);
     if (st) return st;
     const lop::Common &c = pp.c;
@@ -752,19 +782,92 @@ lop_status lop_convolve_chain_execute(const lop_iteration_space *is, const lop_a
         (ii.global_height && ii.global_height != ii.height))
         return fail(LOP_ERR_UNSUPPORTED, "fused chains take whole images (no band views)");
     const int32_t idt = ii.dtype, odt = is->image.dtype;
-    static thread_local lop::ConvChain p;
     if (idt == LOP_F32 && odt == LOP_F32) p.kind = 0;
     else if (idt == LOP_U8 && odt == LOP_U8) p.kind = 1;
     else if (idt == LOP_U8 && odt == LOP_I32) p.kind = 2;
     else return fail(LOP_ERR_INVALID, "unsupported dtype combination %d -> %d", idt, odt);
     st = chain_stage(c, first, idt, p.s1, "first");
     if (st) return st;
-    st = chain_stage(c, second, idt, p.s2, "second");
+    return chain_stage(c, second, idt, p.s2, "second");
+}
+
+// Intermediate image of the two-pass route: the whole input extent in the
+// input's dtype, rows 16-byte aligned.
+int64_t chain_ws_pitch(const lop_image &ii) { return ((int64_t)ii.width * elem_size(ii.dtype) + 15) & ~(int64_t)15; }
+int64_t chain_ws_bytes(const lop_image &ii) { return chain_ws_pitch(ii) * ii.height * ii.batch; }
+}  // namespace
+
+lop_status lop_convolve_chain_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                      const lop_mask *first, const lop_mask *second,
+                                      void *cuda_stream)
+{
+    Prepared pp;
+    static thread_local lop::ConvChain p;
+    lop_status st = chain_prepare(is, in, first, second, pp, p);
     if (st) return st;
     cudaError_t e = lop::launch_conv_chain(p, static_cast<cudaStream_t>(cuda_stream));
     if (e == cudaErrorNotSupported)
         return fail(LOP_ERR_UNSUPPORTED, "no fused chain instance for this mask pair");
     return launched(e, "conv_chain launch");
+}
+
+lop_status lop_convolve_chain_workspace_bytes(const lop_iteration_space *is, const lop_accessor *in,
+                                              const lop_mask *first, const lop_mask *second,
+                                              int64_t *bytes)
+{
+    if (!bytes) return fail(LOP_ERR_INVALID, "bytes is NULL");
+    Prepared pp;
+    static thread_local lop::ConvChain p;
+    lop_status st = chain_prepare(is, in, first, second, pp, p);
+    if (st) return st;
+    *bytes = chain_ws_bytes(in->bc->image);
+    return LOP_OK;
+}
+
+lop_status lop_convolve_chain_execute_ws(const lop_iteration_space *is, const lop_accessor *in,
+                                         const lop_mask *first, const lop_mask *second,
+                                         void *d_workspace, int64_t workspace_bytes,
+                                         void *cuda_stream)
+{
+    Prepared pp;
+    static thread_local lop::ConvChain p;
+    lop_status st = chain_prepare(is, in, first, second, pp, p);
+    if (st) return st;
+    const lop_image &ii = in->bc->image;
+    bool two_pass = d_workspace && workspace_bytes >= chain_ws_bytes(ii);
+    if (const char *env = std::getenv("LOP_CHAIN_FUSED")) two_pass = two_pass && std::atoi(env) == 0;
+    if (!two_pass) return lop_convolve_chain_execute(is, in, first, second, cuda_stream);
+    // Two passes through the workspace (DESIGN.md §6 "Fused chain"): on B200
+    // the intermediate of a 4096^2 image (64 MiB f32 / 16 MiB u8) stays in the
+    // 126 MB L2 between the passes, and the two HBM-bound separable kernels
+    // beat the fused kernel; bit-identical to it by construction (the fused
+    // kernel reproduces exactly these two passes).
+    lop_image g = ii;                                       // G: whole input extent
+    g.data = d_workspace;
+    g.stride_bytes = chain_ws_pitch(ii);
+    g.batch_stride_bytes = g.stride_bytes * ii.height;
+    {
+        cudaPointerAttributes attr;
+        if (cudaPointerGetAttributes(&attr, d_workspace) != cudaSuccess ||
+            (attr.type != cudaMemoryTypeDevice && attr.type != cudaMemoryTypeManaged)) {
+            cudaGetLastError();
+            return fail(LOP_ERR_INVALID, "workspace must be device memory");
+        }
+    }
+    lop_iteration_space is1{};
+    is1.image = g;
+    lop_boundary_condition bc1 = *in->bc;
+    bc1.size_x = first->size_x;
+    bc1.size_y = first->size_y;
+    lop_accessor a1{&bc1, 0, 0};
+    st = lop_convolve_execute(&is1, &a1, first, cuda_stream);
+    if (st) return st;
+    lop_boundary_condition bc2 = *in->bc;
+    bc2.image = g;
+    bc2.size_x = second->size_x;
+    bc2.size_y = second->size_y;
+    lop_accessor a2{&bc2, in->offset_x, in->offset_y};
+    return lop_convolve_execute(is, &a2, second, cuda_stream);
 }
 
 // ------------------------------------- local operator over several accessors

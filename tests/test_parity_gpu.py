@@ -227,8 +227,9 @@ def test_bilateral_step_edge_preserved(lop, monkeypatch):
     assert torch.equal(out, img)
 
 
+@pytest.mark.parametrize("kernel", ["auto", "1", "0"])
 @pytest.mark.parametrize("mode", MODES)
-def test_bilateral_step_edge_bit_exact_default_path(lop, mode):
+def test_bilateral_step_edge_bit_exact_default_path(lop, mode, kernel, monkeypatch):
     """SURVEY §8(c) step-edge pin, bit-exact, on the default (scaled, pair)
     kernel: sigma_r chosen so that alpha = sqrt(log2(e) / (2 sigma_r^2)) = 32
     exactly in f32.  Then J = 32 I is exact for I in {0, .5, 1}, every
@@ -239,6 +240,8 @@ def test_bilateral_step_edge_bit_exact_default_path(lop, mode):
     sigma_r = float(np.float32(math.sqrt(math.log2(math.e) / 2048.0)))
     alpha = np.float32(math.sqrt(math.log2(math.e) / (2.0 * sigma_r * sigma_r)))
     assert alpha == np.float32(32.0)                      # the library's alpha_d -> float
+    if kernel != "auto":                                  # pair-sharing / unshared kernel
+        monkeypatch.setenv("LOP_BILATERAL_PAIR", kernel)
     img = synthetic.levels(300, 517, seed=11)
     out = lop.bilateral(img.cuda(), 3.0, sigma_r, mode, constant=0.5).cpu()
     if mode == "undefined":
@@ -594,16 +597,17 @@ def _chain_pairs(dtype):
     return [(g5, k5, sx, 0), (g3, k3, g5, k5), (box, 3, sy, 0), (g5, k5, g3, k3)]
 
 
+@pytest.mark.parametrize("fused", [True, False])
 @pytest.mark.parametrize("shape", [(1, 1), (5, 7), (37, 70), (130, 1100), (77, 2050)])
 @pytest.mark.parametrize("mode", MODES)
-def test_chain_equals_two_passes_and_oracle(lop, shape, mode):
+def test_chain_equals_two_passes_and_oracle(lop, shape, mode, fused):
     """lop.convolve_chain == two lop.convolve passes bit for bit (f32 and u8), and
     == the oracle's composition (f32 within 1e-5 x mask gain, u8 exact)."""
     H, W = shape
     img = synthetic.uniform(H, W, seed=H + 7 * W)
     u8 = synthetic.uniform_u8(H, W, seed=H * 3 + W)
     for m1, k1, m2, k2 in _chain_pairs("f32"):
-        fused = lop.convolve_chain(img.cuda(), m1, m2, mode, constant=0.5)
+        fused = lop.convolve_chain(img.cuda(), m1, m2, mode, constant=0.5, fused=fused)
         two = lop.convolve(lop.convolve(img.cuda(), m1, mode, constant=0.5), m2, mode,
                            constant=0.5)
         if mode != "undefined":
@@ -618,7 +622,7 @@ def test_chain_equals_two_passes_and_oracle(lop, shape, mode):
         _cmp_float(fused.cpu().numpy(), ref, valid, tol=2e-5)
     for m1, k1, m2, k2 in _chain_pairs("u8"):
         for odt, npdt in ((torch.uint8, np.uint8), (torch.int32, np.int32)):
-            fused = lop.convolve_chain(u8.cuda(), m1, m2, mode, constant=200, shift1=k1,
+            fused = lop.convolve_chain(u8.cuda(), m1, m2, mode, constant=200, shift1=k1, fused=fused,
                                        shift2=k2, out_dtype=odt).cpu()
             mid = lop.convolve(u8.cuda(), m1, mode, constant=200, shift=k1)
             two = lop.convolve(mid, m2, mode, constant=200, shift=k2, out_dtype=odt).cpu()
@@ -629,15 +633,16 @@ def test_chain_equals_two_passes_and_oracle(lop, shape, mode):
                 assert (fused.numpy() == ref).all()
 
 
-def test_chain_roi_offset_and_validation(lop):
+@pytest.mark.parametrize("fused", [True, False])
+def test_chain_roi_offset_and_validation(lop, fused):
     img = synthetic.angio(90, 600, seed=3).cuda()
     g5, k5 = lop.gaussian_mask(5, np.float32)
     sx = lop.sobel_mask(0, np.float32)
-    full = lop.convolve_chain(img, g5, sx, "mirror")
+    full = lop.convolve_chain(img, g5, sx, "mirror", fused=fused)
     out = torch.full_like(img, -1.0)
-    lop.convolve_chain(img, g5, sx, "mirror", out=out, roi=(13, 7, 500, 70))
+    lop.convolve_chain(img, g5, sx, "mirror", out=out, roi=(13, 7, 500, 70), fused=fused)
     assert torch.equal(out[7:77, 13:513], full[7:77, 13:513])
-    off = lop.convolve_chain(img, g5, sx, "clamp", offset=(2, -3))
+    off = lop.convolve_chain(img, g5, sx, "clamp", offset=(2, -3), fused=fused)
     two = lop.convolve(lop.convolve(img, g5, "clamp"), sx, "clamp", offset=(2, -3))
     assert torch.equal(off, two)
     with pytest.raises(lop.LopError, match="separable"):
@@ -663,9 +668,9 @@ def test_chain_stream_equals_tiles(lop, rows, mode, monkeypatch):
             for odt in ((None,) if x.dtype == torch.float32 else (torch.uint8, torch.int32)):
                 kw = dict(constant=cval, shift1=k1, shift2=k2, out_dtype=odt)
                 monkeypatch.setenv("LOP_CHAIN_STREAM", "1")
-                fused = lop.convolve_chain(x, m1, m2, mode, **kw)
+                fused = lop.convolve_chain(x, m1, m2, mode, fused=True, **kw)
                 monkeypatch.setenv("LOP_CHAIN_STREAM", "0")
-                tiles = lop.convolve_chain(x, m1, m2, mode, **kw)
+                tiles = lop.convolve_chain(x, m1, m2, mode, fused=True, **kw)
                 assert torch.equal(fused, tiles), (mode, x.dtype, odt)
                 if mode != "undefined":
                     mid = lop.convolve(x, m1, mode, constant=cval, shift=k1)
@@ -686,7 +691,8 @@ def test_chain_stream_roi_offset(lop, mode, roi, offset, monkeypatch):
         for st in ("1", "0"):
             monkeypatch.setenv("LOP_CHAIN_STREAM", st)
             o = torch.full_like(x, -7.0)
-            lop.convolve_chain(x, m1, m2, mode, constant=0.5, out=o, roi=roi, offset=offset)
+            lop.convolve_chain(x, m1, m2, mode, constant=0.5, out=o, roi=roi, offset=offset,
+                               fused=True)
             outs.append(o)
         assert torch.equal(outs[0], outs[1]), (mode, roi, offset)
         x0, y0, w, h = roi
@@ -982,3 +988,28 @@ def test_bilateral_factored_user_mask(lop, size, monkeypatch):
     out = lop.bilateral(img.cuda(), 0.0, 0.1, "clamp", mask=cm2)
     ref, _ = oracle.bilateral_f32(img.numpy(), 0.0, 0.1, "clamp", cmask=cm2.astype(np.float64))
     _cmp_float(out.cpu().numpy(), ref)
+
+
+def test_bilateral_kernel_choice_by_whole_launch_size(lop, monkeypatch):
+    """N1 (DESIGN.md §6 "Kernel choice"): the pair-sharing or the unshared
+    kernel is chosen from width x global height x frames and the window
+    (profiles/r02/sweep_bilateral_pair_vs_sep.jsonl) -- the auto result equals
+    the forced kernel's bit for bit, and band views / ROI launches of the same
+    image take the same kernel as the whole-image call."""
+    def run(img, force=None, **kw):
+        if force is None:
+            monkeypatch.delenv("LOP_BILATERAL_PAIR", raising=False)
+        else:
+            monkeypatch.setenv("LOP_BILATERAL_PAIR", force)
+        return lop.bilateral(img, 3.0, 0.1, "mirror", size=13, **kw)
+    for S, expect in ((256, "1"), (1024, "0"), (2048, "1")):
+        img = synthetic.angio(S, S, seed=S).cuda()
+        whole = run(img)
+        assert torch.equal(whole, run(img, expect)), S
+        assert not torch.equal(whole, run(img, "1" if expect == "0" else "0")), S
+        # ROI and a band view (halo rows in place) of the same image: same kernel
+        roi = run(img, roi=(5, S // 3, S - 9, S // 4))
+        assert torch.equal(roi[S // 3:S // 3 + S // 4, 5:S - 4], whole[S // 3:S // 3 + S // 4, 5:S - 4])
+        y0, y1 = S // 2, S // 2 + S // 8
+        band = run(img[y0:y1], band=(6, 6, y0, S))
+        assert torch.equal(band, whole[y0:y1]), S

@@ -116,7 +116,7 @@ def test_config5_32768_whole_image_and_p8_bands(lop, c5_image, mode):
     torch.cuda.empty_cache()
 
 
-def test_config4_last_frames_of_1024(lop):
+def test_config4_last_frames_of_1024(lop, monkeypatch):
     """Config 4: 1024 frames of 1024^2 in one batched launch (bench.py's
     N = 1 step); the last frames -- beyond 2^32 bytes -- against the oracle
     (frame 1023 every output, frames 1020-1022 sampled), and bit-identical to
@@ -136,6 +136,9 @@ def test_config4_last_frames_of_1024(lop):
         got = out[f].cpu().numpy()[ys, xs]
         ref, _ = oracle.bilateral_f32_points(host, 3.0, 5.0, "clamp", xs, ys, size=13)
         _cmp(got, ref)
+    # one 1024^2 frame alone takes the unshared kernel (N1 rule, whole-launch
+    # size); forced to the batch's pair kernel it reproduces the batch bit for bit
+    monkeypatch.setenv("LOP_BILATERAL_PAIR", "1")
     for f in (0, 1023):
         assert torch.equal(out[f], lop.bilateral(frames[f].contiguous(), 3.0, 5.0, "clamp",
                                                  size=13))

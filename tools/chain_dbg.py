@@ -12,8 +12,8 @@ else:
     x = torch.stack([synthetic.uniform_u8(67, 1040, seed=s + 80) for s in range(2)]).cuda(); pairs = _chain_pairs("u8"); cval = 99
 for m1, k1, m2, k2 in pairs:
     os.environ["LOP_CHAIN_STREAM"] = "1"
-    a = lop.convolve_chain(x, m1, m2, mode, constant=cval, shift1=k1, shift2=k2)
+    a = lop.convolve_chain(x, m1, m2, mode, constant=cval, shift1=k1, shift2=k2, fused=True)
     torch.cuda.synchronize()
     os.environ["LOP_CHAIN_STREAM"] = "0"
-    b = lop.convolve_chain(x, m1, m2, mode, constant=cval, shift1=k1, shift2=k2)
+    b = lop.convolve_chain(x, m1, m2, mode, constant=cval, shift1=k1, shift2=k2, fused=True)
     print(mode, which, m1.shape, m2.shape, torch.equal(a, b), flush=True)

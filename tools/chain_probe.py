@@ -16,7 +16,7 @@ sxf = lop.sobel_mask(0, np.float32)
 gi, gk = lop.gaussian_mask(5, np.int32)
 sxi = lop.sobel_mask(0, np.int32)
 for _ in range(2):
-    lop.convolve_chain(img, gf, sxf, "clamp")
-    lop.convolve_chain(u8, gi, sxi, "clamp", shift1=gk, out_dtype=torch.int32)
+    lop.convolve_chain(img, gf, sxf, "clamp", fused=True)
+    lop.convolve_chain(u8, gi, sxi, "clamp", shift1=gk, out_dtype=torch.int32, fused=True)
 torch.cuda.synchronize()
 print("ok")

@@ -62,8 +62,8 @@ for H, W in ((13, 17), (70, 257), (67, 1040)):
         gi, gk = lop.gaussian_mask(5, np.int32)
         for st in ("0", "1"):
             os.environ["LOP_CHAIN_STREAM"] = st
-            lop.convolve_chain(img, gf, lop.sobel_mask(0, np.float32), mode, constant=0.5)
-            lop.convolve_chain(u8, gi, lop.sobel_mask(1, np.int32), mode, constant=9, shift1=gk,
+            lop.convolve_chain(img, gf, lop.sobel_mask(0, np.float32, fused=True), mode, constant=0.5)
+            lop.convolve_chain(u8, gi, lop.sobel_mask(1, np.int32, fused=True), mode, constant=9, shift1=gk,
                                out_dtype=torch.int32)
             n += 2
         os.environ.pop("LOP_CHAIN_STREAM")

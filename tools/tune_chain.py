@@ -51,11 +51,11 @@ def timed(fn):
 
 
 cases = {
-    "f32_fused": lambda k, s: lop.convolve_chain(fi[k], gf, sxf, "clamp", out=fo[k], stream=s),
+    "f32_fused": lambda k, s: lop.convolve_chain(fi[k], gf, sxf, "clamp", out=fo[k], stream=s, fused=True),
     "f32_two_pass": lambda k, s: lop.convolve(lop.convolve(fi[k], gf, "clamp", out=mf, stream=s),
                                               sxf, "clamp", out=fo[k], stream=s),
     "u8_i32_fused": lambda k, s: lop.convolve_chain(ui[k], gi, sxi, "clamp", shift1=gk,
-                                                    out=io[k], stream=s),
+                                                    out=io[k], stream=s, fused=True),
     "u8_i32_two_pass": lambda k, s: lop.convolve(lop.convolve(ui[k], gi, "clamp", shift=gk,
                                                               out=mu, stream=s),
                                                  sxi, "clamp", out=io[k], stream=s),
