@@ -597,21 +597,21 @@ def _chain_pairs(dtype):
     return [(g5, k5, sx, 0), (g3, k3, g5, k5), (box, 3, sy, 0), (g5, k5, g3, k3)]
 
 
-@pytest.mark.parametrize("fused", [True, False])
+@pytest.mark.parametrize("route", [True, False])
 @pytest.mark.parametrize("shape", [(1, 1), (5, 7), (37, 70), (130, 1100), (77, 2050)])
 @pytest.mark.parametrize("mode", MODES)
-def test_chain_equals_two_passes_and_oracle(lop, shape, mode, fused):
+def test_chain_equals_two_passes_and_oracle(lop, shape, mode, route):
     """lop.convolve_chain == two lop.convolve passes bit for bit (f32 and u8), and
     == the oracle's composition (f32 within 1e-5 x mask gain, u8 exact)."""
     H, W = shape
     img = synthetic.uniform(H, W, seed=H + 7 * W)
     u8 = synthetic.uniform_u8(H, W, seed=H * 3 + W)
     for m1, k1, m2, k2 in _chain_pairs("f32"):
-        fused = lop.convolve_chain(img.cuda(), m1, m2, mode, constant=0.5, fused=fused)
+        got = lop.convolve_chain(img.cuda(), m1, m2, mode, constant=0.5, fused=route)
         two = lop.convolve(lop.convolve(img.cuda(), m1, mode, constant=0.5), m2, mode,
                            constant=0.5)
         if mode != "undefined":
-            assert torch.equal(fused, two), (mode, shape)
+            assert torch.equal(got, two), (mode, shape)
         g, _ = oracle.convolve_f32(img.numpy(), m1.astype(np.float64), mode, 0.5)
         ref, _ = oracle.convolve_f32(g.astype(np.float32), m2.astype(np.float64), mode, 0.5)
         valid = np.ones_like(ref, bool)
@@ -619,18 +619,18 @@ def test_chain_equals_two_passes_and_oracle(lop, shape, mode, fused):
             r = (m1.shape[0] // 2) + (m2.shape[0] // 2)
             valid[:] = False
             valid[r:H - r, r:W - r] = True
-        _cmp_float(fused.cpu().numpy(), ref, valid, tol=2e-5)
+        _cmp_float(got.cpu().numpy(), ref, valid, tol=2e-5)
     for m1, k1, m2, k2 in _chain_pairs("u8"):
         for odt, npdt in ((torch.uint8, np.uint8), (torch.int32, np.int32)):
-            fused = lop.convolve_chain(u8.cuda(), m1, m2, mode, constant=200, shift1=k1, fused=fused,
+            got = lop.convolve_chain(u8.cuda(), m1, m2, mode, constant=200, shift1=k1, fused=route,
                                        shift2=k2, out_dtype=odt).cpu()
             mid = lop.convolve(u8.cuda(), m1, mode, constant=200, shift=k1)
             two = lop.convolve(mid, m2, mode, constant=200, shift=k2, out_dtype=odt).cpu()
             if mode != "undefined":
-                assert torch.equal(fused, two), (mode, shape, odt)
+                assert torch.equal(got, two), (mode, shape, odt)
                 g, _ = oracle.convolve_u8(u8.numpy(), m1, k1, mode, cval=200)
                 ref, _ = oracle.convolve_u8(g, m2, k2, mode, cval=200, out_dtype=npdt)
-                assert (fused.numpy() == ref).all()
+                assert (got.numpy() == ref).all()
 
 
 @pytest.mark.parametrize("fused", [True, False])
