@@ -82,13 +82,27 @@ __device__ __forceinline__ uint32_t smem_addr(const void *p)
 }
 
 // Wait for phase `parity` of an mbarrier (try_wait loop; hardware sleep).
+// LOP_MBAR_SUSPEND_NS: a suspend-time hint for try_wait (the thread sleeps up
+// to that long unless the phase completes first), so waiting warps do not
+// spin on the issue slots of the warps that are computing; 0 = no hint.
+#ifndef LOP_MBAR_SUSPEND_NS
+#define LOP_MBAR_SUSPEND_NS 0
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity)
 {
+#if LOP_MBAR_SUSPEND_NS > 0
+    asm volatile(
+        "{\n\t.reg .pred P;\n"
+        "WAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared.b64 P, [%0], %1, %2;\n\t"
+        "@!P bra WAIT_%=;\n}" ::"r"(smem_addr(bar)), "r"(parity), "n"(LOP_MBAR_SUSPEND_NS) : "memory");
+#else
     asm volatile(
         "{\n\t.reg .pred P;\n"
         "WAIT_%=:\n\t"
         "mbarrier.try_wait.parity.shared.b64 P, [%0], %1;\n\t"
         "@!P bra WAIT_%=;\n}" ::"r"(smem_addr(bar)), "r"(parity) : "memory");
+#endif
 }
 
 __device__ __forceinline__ float ex2_approx(float x)

@@ -23,13 +23,15 @@
 // cudaOccupancyMaxActiveBlocksPerMultiprocessor, then the fewest threads in
 // border CTAs with y-preferred tilings.
 // Summation order (SUM, f32): per accessor, per window row a left-to-right
-// partial sum (first tap M*g, then FMA), rows folded top to bottom (FADD),
+// partial sum (FMA from +0), rows folded top to bottom (FADD),
 // accessors folded in order (FADD).  MIN / MAX: exact, taps with M != 0.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
 #include <climits>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <type_traits>
 
@@ -83,8 +85,10 @@ struct LocalAccum {
     {
         const V g = tap_g<FN>(v, c);
         if (OP == RED_SUM) {
-            if (std::is_same<V, float>::value) rs = first ? __fmul_rn(M, g) : __fmaf_rn(M, g, rs);
-            else rs = first ? M * g : rs + M * g;
+            // every tap an FMA into the row partial sum, which starts at +0 (so the
+            // first tap is M*g exactly, up to the sign of a zero product)
+            if (std::is_same<V, float>::value) rs = __fmaf_rn(M, g, rs);
+            else rs = rs + M * g;
         } else if (M != (V)0) {
             const V f = std::is_same<V, float>::value ? (V)__fmul_rn(M, g) : M * g;
             total = OP == RED_MIN ? min(total, f) : max(total, f);
@@ -92,7 +96,10 @@ struct LocalAccum {
     }
     __device__ __forceinline__ void end_row(bool first_row)
     {
-        if (OP == RED_SUM) acck = first_row ? rs : (std::is_same<V, float>::value ? (V)__fadd_rn(acck, rs) : acck + rs);
+        if (OP == RED_SUM) {
+            acck = first_row ? rs : (std::is_same<V, float>::value ? (V)__fadd_rn(acck, rs) : acck + rs);
+            rs = (V)0;
+        }
     }
     __device__ __forceinline__ void end_accessor(bool first_acc)
     {
@@ -124,6 +131,71 @@ __device__ __forceinline__ bool local_interior(const LocalAcc &a, int x0, int y0
     return ix0 >= 0 && ix0 + w + 2 * a.rx <= a.in.W && gy >= 0 && gy + h + 2 * a.ry <= a.in.GH;
 }
 
+// Stage rows [r_lo, r_hi) x pitch columns of accessor a's footprint (input
+// origin (ix0, iy0)) into t (row pitch `pitch`, in elements).  Warps take
+// rows, lanes columns (no per-element division); interior tiles load without
+// boundary handling, 16 bytes at a time when aligned.
+template <bool U8>
+__device__ __forceinline__ void local_stage(const LocalAcc &a, int b, int ix0, int iy0, int r_lo,
+                                            int r_hi, int pitch, bool interior,
+                                            typename std::conditional<U8, int, float>::type *t)
+{
+    using V = typename std::conditional<U8, int, float>::type;
+    const int lane = (threadIdx.y * blockDim.x + threadIdx.x) & 31;
+    const int warp = (threadIdx.y * blockDim.x + threadIdx.x) >> 5;
+    const int nwarps = (blockDim.x * blockDim.y + 31) >> 5;
+    const char *fb = a.in.data + (int64_t)b * a.in.bstride;
+    const bool vec = interior && (pitch & 3) == 0 && (ix0 & 3) == 0 && (a.in.stride & (U8 ? 3 : 15)) == 0 &&
+                     ((reinterpret_cast<uintptr_t>(fb) & (U8 ? 3 : 15)) == 0);
+    if constexpr (!U8) {
+        if (vec) {
+            // f32 interior: 16-byte asynchronous copies (LDGSTS), all in flight at
+            // once, waited for here (the caller's __syncthreads follows)
+            const int nv = pitch >> 2, tid = threadIdx.y * blockDim.x + threadIdx.x;
+            const int nthr = blockDim.x * blockDim.y, total = (r_hi - r_lo) * nv;
+            int r = r_lo + tid / nv, x4 = tid % nv;               // one division per thread
+            const int dr = nthr / nv, dx = nthr % nv;
+            for (int i = tid; i < total; i += nthr) {
+                const char *src = fb + (int64_t)(iy0 + r) * a.in.stride + (int64_t)(ix0 + 4 * x4) * 4;
+                const uint32_t dst = (uint32_t)__cvta_generic_to_shared(t + r * pitch + 4 * x4);
+                asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+                r += dr;
+                x4 += dx;
+                if (x4 >= nv) { x4 -= nv; ++r; }
+            }
+            asm volatile("cp.async.commit_group;\n\tcp.async.wait_all;" ::: "memory");
+            return;
+        }
+    }
+    for (int r = r_lo + warp; r < r_hi; r += nwarps) {
+        V *trow = t + r * pitch;
+        if (interior) {
+            const char *rp = fb + (int64_t)(iy0 + r) * a.in.stride;
+            if (vec) {                                   // u8: 4-byte words, 4 in flight per lane
+                for (int x = 4 * lane; x < pitch; x += 512) {
+                    uint32_t w[4];
+#pragma unroll
+                    for (int u = 0; u < 4; ++u)
+                        w[u] = x + 128 * u < pitch
+                                   ? __ldg(reinterpret_cast<const uint32_t *>(rp + ix0 + x + 128 * u)) : 0u;
+#pragma unroll
+                    for (int u = 0; u < 4; ++u)
+                        if (x + 128 * u < pitch)
+                            *reinterpret_cast<int4 *>(trow + x + 128 * u) =
+                                make_int4(w[u] & 0xFF, (w[u] >> 8) & 0xFF, (w[u] >> 16) & 0xFF, w[u] >> 24);
+                }
+            } else {
+                for (int x = lane; x < pitch; x += 32) {
+                    if constexpr (U8) trow[x] = (int)__ldg(reinterpret_cast<const uint8_t *>(rp) + ix0 + x);
+                    else trow[x] = __ldg(reinterpret_cast<const float *>(rp) + ix0 + x);
+                }
+            }
+        } else {
+            for (int x = lane; x < pitch; x += 32) trow[x] = local_read<U8>(a, b, ix0 + x, iy0 + r);
+        }
+    }
+}
+
 // ------------------------------------------------------------------ tiled
 template <bool U8, int OP, int FN>
 __global__ void __launch_bounds__(1024) local_tiled_kernel(const __grid_constant__ LocalParams p)
@@ -145,20 +217,7 @@ __global__ void __launch_bounds__(1024) local_tiled_kernel(const __grid_constant
         const LocalAcc &a = p.acc[k];
         const int sw = tw + 2 * a.rx, sh = rows + 2 * a.ry;
         const int ix0 = tx0 + a.off_x - a.rx, iy0 = ty0 + a.off_y - a.ry;
-        const bool interior = local_interior(a, tx0, ty0, tw, rows);
-        const char *fb = a.in.data + (int64_t)b * a.in.bstride;
-        for (int i = tid; i < sw * sh; i += nthr) {
-            const int r = i / sw, x = i - r * sw;
-            V v;
-            if (interior) {
-                const char *rp = fb + (int64_t)(iy0 + r) * a.in.stride;
-                if constexpr (U8) v = (int)__ldg(reinterpret_cast<const uint8_t *>(rp) + ix0 + x);
-                else v = __ldg(reinterpret_cast<const float *>(rp) + ix0 + x);
-            } else {
-                v = local_read<U8>(a, b, ix0 + x, iy0 + r);
-            }
-            sm[base + i] = v;
-        }
+        local_stage<U8>(a, b, ix0, iy0, 0, sh, sw, local_interior(a, tx0, ty0, tw, rows), sm + base);
         base += sw * sh;
     }
     __syncthreads();
@@ -207,6 +266,135 @@ __global__ void __launch_bounds__(1024) local_tiled_kernel(const __grid_constant
         if (j < nj) local_store<U8>(c, b, x, ty0 + y0 + j, (float)acc[j].total, (int)acc[j].total);
 }
 
+// ----------------------------------------------------- small-window tiled
+// Every accessor's window <= 7 x 7 (the common case: 3x3, 5x5 stencils).
+// Register blocking: a thread computes 4 columns x 4 rows.  Per accessor k and
+// window row yf (runtime, warp-uniform loop) the 7 coefficients of the row are
+// read once (uniform, from the kernel parameter block: the mask embedded in a
+// 7 x 7 slot), then for each of the 4 output rows the staged row segment of
+// 12 values (columns c0 .. c0 + 11 = c0 - 4 .. c0 + 7 of the input) comes in
+// as 3 LDS.128 and feeds 7 x 4 taps, the tap loop unrolled over the slot with
+// warp-uniform predicates for the accessor's own window.  Each output sees
+// exactly the generic kernel's sequence of operations (accessor, window row,
+// left-to-right taps).  Staging: per accessor the tile's rows +- ry_k and
+// columns +- 4; rows past the iteration space are zero-filled, not fetched.
+namespace local {
+constexpr int SR = kLocalSmallR, SW = kLocalSmallW;
+constexpr int SX = 4;                        // output columns per thread
+// staged columns left / right for a launch whose largest x radius is <= RXM
+// (>= RXM, a multiple of 4 so that rows stay 16-byte aligned)
+template <int RXM> struct Halo { static constexpr int HX = (RXM + 3) & ~3; };
+inline int rxm_bucket(int rx) { return rx <= 1 ? 1 : rx <= 2 ? 2 : rx <= 3 ? 3 : 7; }
+}  // namespace local
+
+template <bool U8, int OP, int FN, int RXM>
+__global__ void __launch_bounds__(256) local_small_kernel(const __grid_constant__ LocalParams p)
+{
+    using V = typename std::conditional<U8, int, float>::type;
+    using V4 = typename std::conditional<U8, int4, float4>::type;
+    constexpr int OY = local::OUT_Y, SR = local::SR, SW = local::SW, SX = local::SX;
+    constexpr int HX = local::Halo<RXM>::HX, NV = (SX + 2 * HX) / 4;    // float4 per row segment
+    extern __shared__ float4 smem4[];
+    V *sm = reinterpret_cast<V *>(smem4);
+    const Common &c = p.c;
+    const int tw = SX * blockDim.x, th = OY * blockDim.y;
+    const int pitch = tw + 2 * HX;
+    const int b = blockIdx.z;
+    const int tx0 = c.roi_x0 + blockIdx.x * tw, ty0 = c.roi_y0 + blockIdx.y * th;
+    const int roi_x1 = c.roi_x0 + c.roi_w, roi_y1 = c.roi_y0 + c.roi_h;
+    const int rows = min(th, roi_y1 - ty0);
+    int base = 0;
+#pragma unroll 1
+    for (int k = 0; k < p.n; ++k) {
+        const LocalAcc &a = p.acc[k];
+        const int ix0 = tx0 + a.off_x - HX, iy0 = ty0 + a.off_y - a.ry;
+        const int sh = rows + 2 * a.ry;                                 // fetched rows
+        const int gy = iy0 + a.in.gy0;
+        const bool interior = ix0 >= 0 && ix0 + pitch <= a.in.W && gy >= 0 && gy + sh <= a.in.GH;
+        local_stage<U8>(a, b, ix0, iy0, 0, sh, pitch, interior, sm + base);
+        // rows of a partial last tile row: zero (computed, never stored)
+        for (int i = threadIdx.y * blockDim.x + threadIdx.x + sh * pitch; i < (th + 2 * a.ry) * pitch;
+             i += blockDim.x * blockDim.y)
+            sm[base + i] = (V)0;
+        base += (th + 2 * a.ry) * pitch;
+    }
+    __syncthreads();
+
+    const int c0 = SX * threadIdx.x;                       // tile-relative first column
+    const int r0 = OY * threadIdx.y;                       // tile-relative first row
+    const int x0 = tx0 + c0;
+    LocalAccum<V, OP> acc[OY][SX];
+#pragma unroll
+    for (int j = 0; j < OY; ++j)
+#pragma unroll
+        for (int q = 0; q < SX; ++q) acc[j][q].init();
+    base = 0;
+#pragma unroll 1
+    for (int k = 0; k < p.n; ++k) {
+        const LocalAcc &a = p.acc[k];
+        const int rx = a.rx, ry = a.ry;
+        const V *t = sm + base + c0;                        // column c0 - HX of the input
+        const V *mk = (const V *)(U8 ? (const void *)p.ms.i[k] : (const void *)p.ms.f[k]);
+        V cen[OY][SX];
+        if (FN == local::FN_ABSDIFF || FN == local::FN_SQDIFF) {
+#pragma unroll
+            for (int j = 0; j < OY; ++j) {
+                const V4 w = *reinterpret_cast<const V4 *>(t + (r0 + j + ry) * pitch + HX);
+                cen[j][0] = w.x; cen[j][1] = w.y; cen[j][2] = w.z; cen[j][3] = w.w;
+            }
+        }
+#pragma unroll 1
+        for (int yf = -ry; yf <= ry; ++yf) {
+            V M[2 * RXM + 1];
+#pragma unroll
+            for (int xf = -RXM; xf <= RXM; ++xf) M[xf + RXM] = mk[(yf + SR) * SW + xf + SR];
+#pragma unroll
+            for (int j = 0; j < OY; ++j) {
+                const V4 *rp = reinterpret_cast<const V4 *>(t + (r0 + j + yf + ry) * pitch);
+                V v[4 * NV];
+#pragma unroll
+                for (int i = 0; i < NV; ++i) {
+                    const V4 w = rp[i];
+                    v[4 * i] = w.x; v[4 * i + 1] = w.y; v[4 * i + 2] = w.z; v[4 * i + 3] = w.w;
+                }
+#pragma unroll
+                for (int xf = -RXM; xf <= RXM; ++xf) {
+                    if (xf < -rx || xf > rx) continue;               // warp-uniform
+#pragma unroll
+                    for (int q = 0; q < SX; ++q)
+                        acc[j][q].template tap<FN>(M[xf + RXM], v[HX + q + xf], cen[j][q], xf == -rx);
+                }
+#pragma unroll
+                for (int q = 0; q < SX; ++q) acc[j][q].end_row(yf == -ry);
+            }
+        }
+#pragma unroll
+        for (int j = 0; j < OY; ++j)
+#pragma unroll
+            for (int q = 0; q < SX; ++q) acc[j][q].end_accessor(k == 0);
+        base += (th + 2 * ry) * pitch;
+    }
+    if (x0 >= roi_x1) return;
+    const bool vec = x0 + SX <= roi_x1 && ((x0 & 3) == 0) && ((c.out.stride & 15) == 0) &&
+                     ((reinterpret_cast<uintptr_t>(c.out.data + (int64_t)b * c.out.bstride) & 15) == 0);
+#pragma unroll
+    for (int j = 0; j < OY; ++j) {
+        if (r0 + j >= rows) break;
+        const int y = ty0 + r0 + j;
+        char *orow = c.out.data + (int64_t)b * c.out.bstride + (int64_t)y * c.out.stride;
+        if (vec) {
+            if constexpr (U8) *reinterpret_cast<int4 *>(reinterpret_cast<int32_t *>(orow) + x0) =
+                make_int4(acc[j][0].total, acc[j][1].total, acc[j][2].total, acc[j][3].total);
+            else *reinterpret_cast<float4 *>(reinterpret_cast<float *>(orow) + x0) =
+                make_float4(acc[j][0].total, acc[j][1].total, acc[j][2].total, acc[j][3].total);
+        } else {
+#pragma unroll
+            for (int q = 0; q < SX; ++q)
+                if (x0 + q < roi_x1) local_store<U8>(c, b, x0 + q, y, (float)acc[j][q].total, (int)acc[j][q].total);
+        }
+    }
+}
+
 // ---------------------------------------------------------------- generic
 template <bool U8, int OP, int FN>
 __global__ void __launch_bounds__(1024) local_generic_kernel(const __grid_constant__ LocalParams p)
@@ -250,6 +438,15 @@ __global__ void __launch_bounds__(1024) local_generic_kernel(const __grid_consta
 // --------------------------------------------------------------- launcher
 namespace {
 
+size_t small_smem(const LocalParams &p, int bx, int by)
+{
+    const int rxm = local::rxm_bucket(p.c.rx), hx = (rxm + 3) & ~3;
+    size_t n = 0;
+    for (int k = 0; k < p.n; ++k)
+        n += (size_t)(local::SX * bx + 2 * hx) * (local::OUT_Y * by + 2 * p.acc[k].ry);
+    return n * 4;
+}
+
 size_t tiled_smem(const LocalParams &p, int bx, int by)
 {
     size_t n = 0;
@@ -262,8 +459,9 @@ size_t tiled_smem(const LocalParams &p, int bx, int by)
 // SIMD width): tiling y-preferred (32 x T/32) with border handling, x-preferred
 // (T x 1) without; resource limits from the kernel's attributes and the
 // device's opt-in shared memory; occupancy from the CUDA occupancy API.
+// tiled: 0 generic (1 x 1 outputs per thread), 1 tiled (1 x 4), 2 small (2 x 4)
 template <typename K>
-cudaError_t choose_config(K kernel, const LocalParams &p, bool tiled, int &bx, int &by)
+cudaError_t choose_config(K kernel, const LocalParams &p, int tiled, int &bx, int &by)
 {
     const int dev = current_device();
     cudaFuncAttributes fa;
@@ -284,9 +482,10 @@ cudaError_t choose_config(K kernel, const LocalParams &p, bool tiled, int &bx, i
         lop_config_candidate &cd = cand[n++];
         cd.block_x = border ? 32 : t;
         cd.block_y = border ? t / 32 : 1;
-        cd.out_x = 1;
+        cd.out_x = tiled == 2 ? local::SX : 1;
         cd.out_y = tiled ? local::OUT_Y : 1;
-        const size_t smem = tiled ? tiled_smem(p, cd.block_x, cd.block_y) : 0;
+        const size_t smem = tiled == 2 ? small_smem(p, cd.block_x, cd.block_y)
+                                       : (tiled ? tiled_smem(p, cd.block_x, cd.block_y) : 0);
         cd.valid = t <= fa.maxThreadsPerBlock && smem <= (size_t)smem_max;
         cd.occupancy = 0.0;
         if (cd.valid) {
@@ -308,30 +507,60 @@ cudaError_t choose_config(K kernel, const LocalParams &p, bool tiled, int &bx, i
     return cudaSuccess;
 }
 
+// the small-window instance for the launch's largest x radius
 template <bool U8, int OP, int FN>
-cudaError_t launch_local_t(const LocalParams &p, bool tiled, cudaStream_t stream)
+auto small_kernel_ptr(const LocalParams &p) -> decltype(&local_small_kernel<U8, OP, FN, 1>)
 {
+    switch (local::rxm_bucket(p.c.rx)) {
+    case 1: return local_small_kernel<U8, OP, FN, 1>;
+    case 2: return local_small_kernel<U8, OP, FN, 2>;
+    case 3: return local_small_kernel<U8, OP, FN, 3>;
+    default: return local_small_kernel<U8, OP, FN, 7>;
+    }
+}
+
+template <bool U8, int OP, int FN>
+cudaError_t launch_local_t(const LocalParams &p, bool tiled_ok, cudaStream_t stream)
+{
+    const int kind = !tiled_ok ? 0 : (p.small ? 2 : 1);
     // configuration cache: the last geometry per (thread, instance)
-    struct Key { int dev, w, h, batch, n, tiled; int r[4 * kLocalMaxAcc]; };
+    struct Key { int dev, w, h, batch, n, kind; int r[4 * kLocalMaxAcc]; };
     static thread_local Key last{};
     static thread_local int last_bx = 0, last_by = 0;
     Key key{};
     key.dev = current_device(); key.w = p.c.roi_w; key.h = p.c.roi_h; key.batch = p.c.batch;
-    key.n = p.n; key.tiled = tiled;
+    key.n = p.n; key.kind = kind;
     for (int k = 0; k < p.n; ++k) {
         key.r[4 * k] = p.acc[k].rx; key.r[4 * k + 1] = p.acc[k].ry;
         key.r[4 * k + 2] = p.acc[k].off_x; key.r[4 * k + 3] = p.acc[k].off_y;
     }
     int bx = 0, by = 0;
-    if (last_bx && !memcmp(&key, &last, sizeof key)) {
+    if (const char *env = std::getenv("LOP_LOCAL_CFG")) {          // exploration (Fig. 4 sweep)
+        if (std::sscanf(env, "%d:%d", &bx, &by) != 2 || bx < 1 || by < 1 || bx * by > 1024) bx = by = 0;
+    }
+    if (bx) {
+    } else if (last_bx && !memcmp(&key, &last, sizeof key)) {
         bx = last_bx; by = last_by;
     } else {
-        cudaError_t e = tiled ? choose_config(local_tiled_kernel<U8, OP, FN>, p, true, bx, by)
-                              : choose_config(local_generic_kernel<U8, OP, FN>, p, false, bx, by);
+        cudaError_t e = kind == 2 ? choose_config(small_kernel_ptr<U8, OP, FN>(p), p, 2, bx, by)
+                      : kind == 1 ? choose_config(local_tiled_kernel<U8, OP, FN>, p, 1, bx, by)
+                                  : choose_config(local_generic_kernel<U8, OP, FN>, p, 0, bx, by);
         if (e != cudaSuccess) return e;
         last = key; last_bx = bx; last_by = by;
+        if (std::getenv("LOP_DEBUG_SELECT"))
+            fprintf(stderr, "[lop] local kernel %d: Algorithm 2 chose %d x %d threads for %d x %d\n",
+                    kind, bx, by, p.c.roi_w, p.c.roi_h);
     }
-    if (tiled) {
+    if (kind == 2) {
+        const size_t smem = small_smem(p, bx, by);
+        auto kern = small_kernel_ptr<U8, OP, FN>(p);
+        static PerDevice configured_b[8];                       // one cache per instance (bucket)
+        cudaError_t e = ensure_smem(kern, smem, configured_b[local::rxm_bucket(p.c.rx)]);
+        if (e != cudaSuccess) return e;
+        const int tw = local::SX * bx, th = local::OUT_Y * by;
+        dim3 grid((p.c.roi_w + tw - 1) / tw, (p.c.roi_h + th - 1) / th, p.c.batch);
+        kern<<<grid, dim3(bx, by), smem, stream>>>(p);
+    } else if (kind == 1) {
         const size_t smem = tiled_smem(p, bx, by);
         static PerDevice configured;
         cudaError_t e = ensure_smem(local_tiled_kernel<U8, OP, FN>, smem, configured);

@@ -956,6 +956,23 @@ lop_status lop_local_execute(const lop_iteration_space *is, const lop_accessor *
         return fail(LOP_ERR_UNSUPPORTED, "integer masks too large: the result may overflow int32");
     p.c.rx = rx;                                     // the largest window (L556-L558)
     p.c.ry = ry;
+    // small-window path: every mask embedded centred in a 7 x 7 slot
+    p.small = rx <= lop::kLocalSmallR && ry <= lop::kLocalSmallR;
+    if (const char *env = std::getenv("LOP_LOCAL_SMALL")) p.small = p.small && std::atoi(env) != 0;
+    if (p.small) {
+        constexpr int SR = lop::kLocalSmallR, SW = lop::kLocalSmallW;
+        std::memset(&p.ms, 0, sizeof p.ms);
+        for (int k = 0; k < n_inputs; ++k) {
+            const lop::LocalAcc &a = p.acc[k];
+            const int sx = 2 * a.rx + 1;
+            for (int yf = -a.ry; yf <= a.ry; ++yf)
+                for (int xf = -a.rx; xf <= a.rx; ++xf) {
+                    const int src = a.moff + (yf + a.ry) * sx + xf + a.rx, dst = (yf + SR) * SW + xf + SR;
+                    if (p.u8) p.ms.i[k][dst] = p.m.i[src];
+                    else p.ms.f[k][dst] = p.m.f[src];
+                }
+        }
+    }
     const bool tiled = g_variant != LOP_VARIANT_GENERIC;
     return launched(lop::launch_local(p, tiled, static_cast<cudaStream_t>(cuda_stream)),
                     "local launch");

@@ -186,10 +186,17 @@ struct LocalAcc {
     int32_t cval_i;
     int32_t moff;
 };
+constexpr int kLocalSmallR = 7;                               // register-blocked path: radii <= 7
+constexpr int kLocalSmallW = 2 * kLocalSmallR + 1;
 struct LocalParams {
     Common c;                    // output, ROI, batch, largest radii
     int32_t n, op, fn, u8;
+    int32_t small;               // every radius <= kLocalSmallR: masks also in ms (15 x 15 slots)
     LocalAcc acc[kLocalMaxAcc];
+    union {                      // mask k embedded centred in a 15 x 15 slot (zeros outside)
+        float f[kLocalMaxAcc][kLocalSmallW * kLocalSmallW];
+        int32_t i[kLocalMaxAcc][kLocalSmallW * kLocalSmallW];
+    } ms;
     union {
         float f[kLocalMaxTaps];
         int32_t i[kLocalMaxTaps];

@@ -50,14 +50,18 @@ def _cmp_float(gpu, ref, valid=None, tol=TOL):
     return err
 
 
-def _sample_points(H, W, n_random, r, seed):
+def _sample_points(H, W, n_random, r, seed, dense_borders=False):
+    """All outputs within r + 2 of a border (dense_borders) or every 64th of
+    them, the corner neighbourhoods, and n_random interior points."""
     rng = np.random.default_rng(seed)
     pts = set()
+    step_x = 1 if dense_borders else max(1, W // 64)
+    step_y = 1 if dense_borders else max(1, H // 64)
     for y in list(range(min(H, r + 2))) + list(range(max(0, H - r - 2), H)):
-        for x in range(0, W, max(1, W // 64)):
+        for x in range(0, W, step_x):
             pts.add((y, x))
     for x in list(range(min(W, r + 2))) + list(range(max(0, W - r - 2), W)):
-        for y in range(0, H, max(1, H // 64)):
+        for y in range(0, H, step_y):
             pts.add((y, x))
     for cy in (0, H - 1):
         for cx in (0, W - 1):
@@ -193,7 +197,8 @@ def test_config2_bilateral_4096_sampled(lop, mode):
     img = synthetic.angio(H, W, seed=synthetic.config_seed(2), device="cuda")
     out = lop.bilateral(img, 3.0, 5.0, mode, constant=0.0).cpu().numpy()
     host = img.cpu().numpy()
-    ys, xs = _sample_points(H, W, 4000, 6, seed=2)
+    # every output of the border strips (8 rows / columns per side) + corners + random interior
+    ys, xs = _sample_points(H, W, 4000, 6, seed=2, dense_borders=True)
     ref, valid = oracle.bilateral_f32_points(host, 3.0, 5.0, mode, xs, ys, cval=0.0)
     _cmp_float(out[ys, xs], ref, valid if mode == "undefined" else None)
     # small sigma_r exercises the range term (reading c3)
