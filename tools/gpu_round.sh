@@ -31,7 +31,7 @@ for w in $WHAT; do
       timeout 300 ./tools/peaks > "$OUT/peaks.txt" 2>&1
       echo "peaks exit $?" >> "$OUT/status.txt" ;;
     ncu)
-      timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"bilateral|conv" -c 40 --csv \
+      timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"bilateral|conv|local" -c 60 --csv \
         --log-file "$OUT/launches.csv" python bench.py --steps 20 --warmup 3 --no-extras \
         --no-cpu-baseline --e2e-steps 0 --no-partitioned > "$OUT/ncu_launch_bench.log" 2>&1
       echo "ncu exit $?" >> "$OUT/status.txt" ;;
