@@ -81,6 +81,9 @@ def parse(argv=None):
     ap.add_argument("--e2e-steps", type=int, default=10)
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--dry-run", action="store_true", help="launch plumbing only (gloo, no GPU)")
+    ap.add_argument("--backend", choices=["nccl", "gloo"], default="nccl",
+                    help="process-group backend (gloo: ranks may share one GPU -- a test of "
+                         "the N > 1 code path on a single-GPU box; halos are host-staged)")
     return ap.parse_args(argv)
 
 
@@ -139,10 +142,18 @@ class Dist:
         self.local = int(os.environ.get("LOCAL_RANK", "0"))
         self.backend = None
 
+    def device_index(self) -> int:
+        """This rank's GPU: LOCAL_RANK (nccl); modulo the visible GPUs for gloo,
+        whose ranks may share one GPU."""
+        import torch
+        n = torch.cuda.device_count()
+        return self.local if self.backend != "gloo" or n == 0 else self.local % n
+
     def init(self, backend="nccl"):
         import torch
         import torch.distributed as dist
         if self.world > 1 and not dist.is_initialized():
+            self.backend = backend
             if backend == "nccl":
                 torch.cuda.set_device(self.local)
             dist.init_process_group(backend, device_id=(torch.device("cuda", self.local)
@@ -486,12 +497,12 @@ def run_lop(args, dist, peaks):
     import synthetic
     import paper_conf_ipps_membarthhtke12_b200 as lop
 
-    dev = torch.device("cuda", dist.local)
+    dev = torch.device("cuda", dist.device_index())
     torch.cuda.set_device(dev)
     stream = torch.cuda.current_stream(dev)
     K, W = args.steps, max(3, args.warmup)
     wl = WORKLOADS[args.workload](args, dist, lop, synthetic, dev, stream)
-    clocks = ClockSampler(dist.local)
+    clocks = ClockSampler(dist.device_index())
     clocks.start()
     total_ms, per, launches = time_steps(wl["step"], K, W, dist, stream, lop)
     # keep the GPU busy a little longer so the sampler sees the clocks under load
@@ -543,14 +554,14 @@ def run_e2e(args, dist, lop, base, dev):
     # single synchronous image: 1024-row chunks (ramped); a frame stream: 2048-row
     # chunks (the fill / drain is paid once per stream; tools/pipe_frames_sweep.py)
     one = host_in[0]
-    pipe1 = lop.Pipeline(Wd, H, device=dist.local, chunk_rows=1024)
+    pipe1 = lop.Pipeline(Wd, H, device=dist.device_index(), chunk_rows=1024)
     pipe1.bilateral(one, host_out[0], SIGMA_D, SIGMA_R, args.mode, size=WINDOW)
     dist.barrier()
     t0 = time.perf_counter()
     pipe1.bilateral(one, host_out[0], SIGMA_D, SIGMA_R, args.mode, size=WINDOW)
     t_single = dist.max(time.perf_counter() - t0)
     pipe1.close()
-    pipe = lop.Pipeline(Wd, H, device=dist.local, chunk_rows=2048)
+    pipe = lop.Pipeline(Wd, H, device=dist.device_index(), chunk_rows=2048)
     # warm-up over every frame: the first DMA touching each pinned page is slower
     pipe.bilateral_frames(host_in, host_out, SIGMA_D, SIGMA_R, args.mode, size=WINDOW)
     dist.barrier()
@@ -845,7 +856,7 @@ def main(argv=None):
     if not torch.cuda.is_available():
         print(json.dumps({"error": "bench.py needs a CUDA device (no CPU fallback)"}))
         return 1
-    dist.init("nccl")
+    dist.init(args.backend)
     peaks = load_peaks()
     res = run_lop(args, dist, peaks)
     if dist.rank == 0:
