@@ -265,19 +265,21 @@ _TAP = {"product": _lib.LOP_TAP_PRODUCT, "absdiff": _lib.LOP_TAP_ABSDIFF,
 
 
 def local(inputs, masks, op="sum", fn="product", modes="clamp", constants=0.0, offsets=None,
-          out=None, roi=None, stream=None) -> torch.Tensor:
+          out=None, roi=None, stream=None, band=None) -> torch.Tensor:
     """Local operator over several Accessors with a per-tap function
     (lop_local_execute; Listing 9):
     out = op over k, taps of fn(M_k, Read_k(x+ox_k+xf, y+oy_k+yf), centre_k).
     inputs: up to 4 CUDA images of one shape and dtype (float32 -> float32,
     uint8 -> int32); masks: one 2D host mask per input (its window);
-    modes / constants / offsets: per input (or one value for all)."""
+    modes / constants / offsets: per input (or one value for all); band: per input
+    (halo_top, halo_bottom, global_y0, global_height) for row-band views."""
     K = len(inputs)
     if K != len(masks):
         raise ValueError("one mask per input")
     modes = [modes] * K if isinstance(modes, (str, int)) else list(modes)
     constants = [constants] * K if np.isscalar(constants) else list(constants)
     offsets = [(0, 0)] * K if offsets is None else list(offsets)
+    band = [(0, 0, 0, 0)] * K if band is None else list(band)
     x0 = inputs[0]
     mdt = _lib.LOP_F32 if x0.dtype == torch.float32 else _lib.LOP_I32
     if out is None:
@@ -287,7 +289,7 @@ def local(inputs, masks, op="sum", fn="product", modes="clamp", constants=0.0, o
     for k in range(K):
         arr, m = _host_mask(masks[k], mdt)
         bc = _lib.lop_boundary_condition()
-        bc.image = image_view(inputs[k])
+        bc.image = image_view(inputs[k], *band[k])
         bc.mode = _mode(modes[k])
         bc.size_x, bc.size_y = m.size_x, m.size_y
         bc.constant = float(constants[k])
@@ -298,7 +300,7 @@ def local(inputs, masks, op="sum", fn="product", modes="clamp", constants=0.0, o
     acc_arr = (ctypes.POINTER(_lib.lop_accessor) * K)(*[ctypes.pointer(a) for a in accs])
     m_arr = (ctypes.POINTER(_lib.lop_mask) * K)(*[ctypes.pointer(m) for m in ms])
     is_ = _lib.lop_iteration_space()
-    is_.image = image_view(out)
+    is_.image = image_view(out, 0, 0, band[0][2], band[0][3])
     if roi is not None:
         is_.x0, is_.y0, is_.width, is_.height = (int(v) for v in roi)
     with torch.cuda.device(x0.device):

@@ -1,4 +1,4 @@
-// local.cu -- local operator over several Accessors with a per-tap function
+// local_impl.cuh -- local operator over several Accessors with a per-tap function
 // (include/lop.h lop_local_execute):
 //   PAPER.md L556-L558  "In case multiple Accessors are used within one
 //                        kernel, the largest window size specified is taken"
@@ -25,6 +25,9 @@
 // Summation order (SUM, f32): per accessor, per window row a left-to-right
 // partial sum (FMA from +0), rows folded top to bottom (FADD),
 // accessors folded in order (FADD).  MIN / MAX: exact, taps with M != 0.
+// Instantiated by local_f32.cu and local_u8.cu (two translation units, so the
+// ~70 kernel instances each compile in parallel).
+#pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -599,10 +602,5 @@ cudaError_t launch_local_u8(const LocalParams &p, bool tiled, cudaStream_t s)
 }
 
 }  // namespace
-
-cudaError_t launch_local(const LocalParams &p, bool tiled, cudaStream_t stream)
-{
-    return p.u8 ? launch_local_u8<true>(p, tiled, stream) : launch_local_u8<false>(p, tiled, stream);
-}
 
 }  // namespace lop

@@ -142,6 +142,29 @@ def test_local_roi_frames_and_band_views(lop):
     assert float(np.abs(whole.cpu().numpy() - ref).max()) <= TOL
 
 
+@pytest.mark.parametrize("mode", MODES)
+def test_local_band_views_bit_identical(lop, mode):
+    """Row bands of both accessors (halo rows in place; REPEAT ring rows at
+    the ends) reproduce the whole-image output bit for bit -- the largest
+    window (7 rows here) sets the halo the band must hold (L556-L558)."""
+    rng = np.random.default_rng(13)
+    H, W = 120, 150
+    a = synthetic.angio(H, W, seed=31).cuda()
+    b = synthetic.uniform(H, W, seed=32).cuda()
+    masks = _masks(rng, [(3, 5), (7, 3)], False)
+    kw = dict(op="sum", fn="sqdiff", modes=[mode, mode], constants=[0.5, 0.25])
+    whole = lop.local([a, b], masks, **kw)
+    r = 3                                                   # the largest window: 7 rows
+    for y0, y1 in ((0, 17), (17, 64), (64, 120)):
+        top = r if (y0 > 0 or mode == "repeat") else 0
+        bot = r if (y1 < H or mode == "repeat") else 0
+        rows = [(y % H) for y in range(y0 - top, y1 + bot)]
+        ba = a[rows].contiguous()[top:top + (y1 - y0)]
+        bb = b[rows].contiguous()[top:top + (y1 - y0)]
+        out = lop.local([ba, bb], masks, band=[(top, bot, y0, H)] * 2, **kw)
+        assert torch.equal(out, whole[y0:y1]), (mode, y0, y1)
+
+
 def test_local_4096_sampled(lop):
     """The bench case: two 4096^2 f32 frames, SUM of PRODUCT with a 5x5 and a
     3x3 mask (a temporal-spatial average of consecutive angiography frames)."""
