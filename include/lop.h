@@ -259,8 +259,8 @@ lop_status lop_global_reduce_execute(const lop_iteration_space *is, int32_t op, 
  * halo is the largest window (L556-L558).  All images share the output's
  * width / height / batch.
  * dtypes: every input F32 with F32 masks -> F32 output (SUM accumulated in
- * f32 in a fixed order: per accessor, per window row a left-to-right partial
- * sum, rows top to bottom, accessors in order); or every input U8 with I32
+ * f32 in a fixed order: per accessor one FMA chain over its taps, window rows
+ * top to bottom, taps left to right; accessors in order); or every input U8 with I32
  * masks -> I32 output (exact integers; the worst-case magnitude must fit
  * int32, else LOP_ERR_UNSUPPORTED).
  * Kernel configuration: Algorithm 2 on B200 terms --

@@ -22,9 +22,9 @@
 // The CTA shape of both comes from Algorithm 2 (select.cpp): occupancy from
 // cudaOccupancyMaxActiveBlocksPerMultiprocessor, then the fewest threads in
 // border CTAs with y-preferred tilings.
-// Summation order (SUM, f32): per accessor, per window row a left-to-right
-// partial sum (FMA from +0), rows folded top to bottom (FADD),
-// accessors folded in order (FADD).  MIN / MAX: exact, taps with M != 0.
+// Summation order (SUM, f32): per accessor one FMA chain from +0 over its
+// taps, window rows top to bottom and taps left to right; the accessors'
+// sums added in order (FADD).  MIN / MAX: exact, taps with M != 0.
 // Instantiated by local_f32.cu and local_u8.cu (two translation units, so the
 // ~70 kernel instances each compile in parallel).
 #pragma once
@@ -69,7 +69,7 @@ __device__ __forceinline__ int tap_g(int v, int c)
     return v;
 }
 
-// Per-output accumulator: SUM keeps (total, accessor sum, row partial);
+// Per-output accumulator: SUM keeps (total, running accessor sum);
 // MIN / MAX a running extreme initialised to the identity.
 template <typename V, int OP>
 struct LocalAccum {
@@ -97,16 +97,15 @@ struct LocalAccum {
             total = OP == RED_MIN ? min(total, f) : max(total, f);
         }
     }
-    __device__ __forceinline__ void end_row(bool first_row)
-    {
-        if (OP == RED_SUM) {
-            acck = first_row ? rs : (std::is_same<V, float>::value ? (V)__fadd_rn(acck, rs) : acck + rs);
-            rs = (V)0;
-        }
-    }
+    // one FMA chain per accessor over its taps (yf outer, xf inner); the
+    // accessors' sums are added in order
+    __device__ __forceinline__ void end_row(bool) {}
     __device__ __forceinline__ void end_accessor(bool first_acc)
     {
-        if (OP == RED_SUM) total = first_acc ? acck : (std::is_same<V, float>::value ? (V)__fadd_rn(total, acck) : total + acck);
+        if (OP == RED_SUM) {
+            total = first_acc ? rs : (std::is_same<V, float>::value ? (V)__fadd_rn(total, rs) : total + rs);
+            rs = (V)0;
+        }
     }
 };
 
@@ -306,21 +305,60 @@ __global__ void __launch_bounds__(256) local_small_kernel(const __grid_constant_
     const int tx0 = c.roi_x0 + blockIdx.x * tw, ty0 = c.roi_y0 + blockIdx.y * th;
     const int roi_x1 = c.roi_x0 + c.roi_w, roi_y1 = c.roi_y0 + c.roi_h;
     const int rows = min(th, roi_y1 - ty0);
+    const int tid = threadIdx.y * blockDim.x + threadIdx.x;
+    // f32 interior footprints: one cp.async.bulk per staged row (TMA bulk
+    // engine, issued by one thread, completing on `sbar`); the rest element-wise
+    __shared__ __align__(8) uint64_t sbar;
+    if (tid == 0) {
+        asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&sbar)));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    auto bulk_ok = [&](const LocalAcc &a, int ix0, int iy0, int sh) {
+        if constexpr (U8) return false;
+        const char *fb = a.in.data + (int64_t)b * a.in.bstride;
+        const int gy = iy0 + a.in.gy0;
+        return ix0 >= 0 && ix0 + pitch <= a.in.W && gy >= 0 && gy + sh <= a.in.GH && (ix0 & 3) == 0 &&
+               (a.in.stride & 15) == 0 && (reinterpret_cast<uintptr_t>(fb) & 15) == 0;
+    };
+    if (tid == 0) {
+        uint32_t nbytes = 0;
+        for (int k = 0; k < p.n; ++k) {
+            const LocalAcc &a = p.acc[k];
+            const int ix0 = tx0 + a.off_x - HX, iy0 = ty0 + a.off_y - a.ry, sh = rows + 2 * a.ry;
+            if (bulk_ok(a, ix0, iy0, sh)) nbytes += (uint32_t)(sh * pitch * 4);
+        }
+        asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;" ::"r"(smem_addr(&sbar)), "r"(nbytes)
+                     : "memory");
+    }
     int base = 0;
 #pragma unroll 1
     for (int k = 0; k < p.n; ++k) {
         const LocalAcc &a = p.acc[k];
         const int ix0 = tx0 + a.off_x - HX, iy0 = ty0 + a.off_y - a.ry;
         const int sh = rows + 2 * a.ry;                                 // fetched rows
-        const int gy = iy0 + a.in.gy0;
-        const bool interior = ix0 >= 0 && ix0 + pitch <= a.in.W && gy >= 0 && gy + sh <= a.in.GH;
-        local_stage<U8>(a, b, ix0, iy0, 0, sh, pitch, interior, sm + base);
+        if (bulk_ok(a, ix0, iy0, sh)) {
+            if (tid == 0) {
+                const char *src = a.in.data + (int64_t)b * a.in.bstride + (int64_t)iy0 * a.in.stride +
+                                  (int64_t)ix0 * 4;
+                for (int r = 0; r < sh; ++r)
+                    asm volatile(
+                        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                        ::"r"(smem_addr(sm + base + r * pitch)), "l"(src + (int64_t)r * a.in.stride),
+                          "r"(pitch * 4), "r"(smem_addr(&sbar))
+                        : "memory");
+            }
+        } else {
+            const int gy = iy0 + a.in.gy0;
+            const bool interior = ix0 >= 0 && ix0 + pitch <= a.in.W && gy >= 0 && gy + sh <= a.in.GH;
+            local_stage<U8>(a, b, ix0, iy0, 0, sh, pitch, interior, sm + base);
+        }
         // rows of a partial last tile row: zero (computed, never stored)
-        for (int i = threadIdx.y * blockDim.x + threadIdx.x + sh * pitch; i < (th + 2 * a.ry) * pitch;
-             i += blockDim.x * blockDim.y)
+        for (int i = tid + sh * pitch; i < (th + 2 * a.ry) * pitch; i += blockDim.x * blockDim.y)
             sm[base + i] = (V)0;
         base += (th + 2 * a.ry) * pitch;
     }
+    mbar_wait(&sbar, 0);
     __syncthreads();
 
     const int c0 = SX * threadIdx.x;                       // tile-relative first column
