@@ -449,10 +449,14 @@ __global__ void __launch_bounds__(tiled::NT, 3) bilateral_sep_kernel(const __gri
 #define LOP_PAIR_NW 2
 #endif
 #ifndef LOP_PAIR_MAXREG
-#define LOP_PAIR_MAXREG 168
+#define LOP_PAIR_MAXREG 160   // 160 / 164 / 168: same 12 warps/SM; 160 schedules best (profiles/r02)
+#endif
+#ifndef LOP_PAIR_DY_UNROLL
+#define LOP_PAIR_DY_UNROLL 1
 #endif
 namespace pair {
 constexpr int NW = LOP_PAIR_NW;                        // warps per CTA
+constexpr int kDyUnroll = LOP_PAIR_DY_UNROLL;          // packed row-pair loop unroll (1: rolled)
 template <int R> struct Shape {
     static constexpr int HLN = (R + 3) / 4;            // halo lanes each side
     static constexpr int HL = 4 * HLN;                 // halo columns each side
@@ -758,7 +762,7 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
             fold4(cy, rd, rp, D[0], P[0]);
             fold4(cy, qd, qp, D[0], P[0]);
         }
-#pragma unroll 1
+#pragma unroll pair::kDyUnroll
         for (int dy = 1; dy + 1 <= R; dy += 2) {                 // row pairs (dy, dy+1): packed
             if (dy + 1 < kmin) continue;
             const int sl = slot0 + dy >= NR ? slot0 + dy - NR : slot0 + dy;
