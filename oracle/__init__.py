@@ -90,9 +90,9 @@ def _load():
                                                         dbl, i32, dbl, vp, vp, i64, vp, vp]
             pa = ctypes.POINTER(ctypes.c_void_p)
             lib.oracle_local_f32.argtypes = [i32, pa, vp, i64, i64, pa, vp, vp, vp, vp, vp, vp,
-                                             i32, i32, i64, i64, vp, vp]
+                                             vp, vp, i32, i32, i64, i64, vp, vp]
             lib.oracle_local_u8.argtypes = [i32, pa, vp, i64, i64, pa, vp, vp, vp, vp, vp, vp,
-                                            i32, i32, i64, i64, vp, vp]
+                                            vp, vp, i32, i32, i64, i64, vp, vp]
             _lib = lib
     return _lib
 
@@ -240,7 +240,10 @@ def global_reduce(img, op, roi=None):
     """Global operator: one value for all pixels of the
     region (x0, y0, w, h) of a 2D image or a (B, H, W) stack.  "sum" is the
     correctly rounded exact sum (math.fsum over the float values; exact integer
-    for u8), "min" / "max" the extreme pixel value."""
+    for u8), "min" / "max" the extreme pixel value, "sumsq" the correctly
+    rounded exact sum of squares (the square of an f32 value is exact in
+    double) -- a merge of two pixels a, b -> a^2 + b^2 summed over the image
+    ("operations that merge/reduce two pixels"; reading c26)."""
     import math
     a = np.asarray(img)
     if a.ndim == 2:
@@ -252,6 +255,10 @@ def global_reduce(img, op, roi=None):
         if a.dtype == np.uint8:
             return float(int(a.astype(np.int64).sum()))
         return math.fsum(float(v) for v in a.ravel())
+    if op == "sumsq":
+        if a.dtype == np.uint8:
+            return float(int((a.astype(np.int64) ** 2).sum()))
+        return math.fsum(float(v) * float(v) for v in a.ravel())
     if op == "min":
         return float(min(a.ravel().tolist()))
     if op == "max":
@@ -349,12 +356,15 @@ TAP_FNS = {"product": 0, "absdiff": 1, "sqdiff": 2, "square": 3}
 
 
 def local(imgs, masks, op="sum", fn="product", modes="clamp", cvals=0.0, offsets=None,
-          rows=None):
+          rows=None, point=None):
     """Local operator over K accessors (N2; Listing 9):
     out = op over k, taps of fn(M_k, Read_k(x+ox_k+xf, y+oy_k+yf), centre_k).
     imgs: K images of one shape and dtype (float32 -> double result, uint8 ->
     exact int64); masks: K 2D masks (odd sizes, float for f32, int for u8);
-    modes / cvals / offsets: one per accessor (or a single value for all)."""
+    modes / cvals / offsets: one per accessor (or a single value for all);
+    point: per accessor (scale, offset) of a point-operator prologue
+    Read'_k = scale * Read_k + offset applied to every read of accessor k
+    (reading c27) -- None = identity."""
     K = len(imgs)
     assert K == len(masks) and K >= 1
     u8 = np.asarray(imgs[0]).dtype == np.uint8
@@ -375,18 +385,23 @@ def local(imgs, masks, op="sum", fn="product", modes="clamp", cvals=0.0, offsets
     oxs = np.array([o[0] for o in offsets], np.int32)
     oys = np.array([o[1] for o in offsets], np.int32)
     mds = np.array([_mode(md) for md in modes], np.int32)
+    point = [(1, 0)] * K if point is None else list(point)
     y0, y1 = (0, H) if rows is None else rows
     valid = np.empty((y1 - y0, W), np.uint8)
     if u8:
         cv = np.array([int(c) for c in cvals], np.int64)
+        pa = np.array([int(a) for a, _ in point], np.int64)
+        pb = np.array([int(b) for _, b in point], np.int64)
         out = np.empty((y1 - y0, W), np.int64)
         fnc = _load().oracle_local_u8
     else:
         cv = np.array([float(c) for c in cvals], np.float64)
+        pa = np.array([float(a) for a, _ in point], np.float64)
+        pb = np.array([float(b) for _, b in point], np.float64)
         out = np.empty((y1 - y0, W), np.float64)
         fnc = _load().oracle_local_f32
     fnc(K, ctypes.cast(img_ptrs, ctypes.POINTER(ctypes.c_void_p)), _ptr(strides), W, H,
         ctypes.cast(m_ptrs, ctypes.POINTER(ctypes.c_void_p)), _ptr(mws), _ptr(mhs), _ptr(oxs),
-        _ptr(oys), _ptr(mds), _ptr(cv), LOCAL_OPS[op], TAP_FNS[fn], y0, y1, _ptr(out),
-        _ptr(valid))
+        _ptr(oys), _ptr(mds), _ptr(cv), _ptr(pa), _ptr(pb), LOCAL_OPS[op], TAP_FNS[fn], y0, y1,
+        _ptr(out), _ptr(valid))
     return out, valid.astype(bool)

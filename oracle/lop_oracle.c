@@ -417,6 +417,8 @@ void oracle_bilateral_f32_points(const float *img, int64_t W, int64_t H, int64_t
 /* taps with M != 0, reading c18):                                       */
 /*   out(x, y) = op_{k, yf, xf} f(M_k(xf, yf),                          */
 /*                  Read_k(x + ox_k + xf, y + oy_k + yf), c_k)           */
+/* Point-operator prologue (reading c27): every read */
+/* of accessor k is Read'_k = pa_k * Read_k + pb_k (centre included).    */
 /* Undefined mode: the output is valid iff no read of any accessor      */
 /* (its whole window, centre included) leaves its image (reading c9).   */
 /* f32 images: double arithmetic; u8 images: exact int64.               */
@@ -444,19 +446,21 @@ static int64_t tap_fn_i64(int fn, int64_t M, int64_t v, int64_t c)
 static double local_px_f32(int K, const float *const *imgs, const int64_t *strides, int64_t W,
                            int64_t H, const double *const *masks, const int *mws, const int *mhs,
                            const int *oxs, const int *oys, const int *modes, const double *cvals,
-                           int op, int fn, int64_t x, int64_t y, uint8_t *valid)
+                           const double *pa, const double *pb, int op, int fn, int64_t x,
+                           int64_t y, uint8_t *valid)
 {
     int undef = 0, first = 1;
     double acc = 0.0;
     for (int k = 0; k < K; ++k) {
         const int m = mws[k] / 2, n = mhs[k] / 2;
         const int64_t cx = x + oxs[k], cy = y + oys[k];
-        const double c = read_f32(imgs[k], W, H, strides[k], cx, cy, modes[k], cvals[k], &undef);
+        const double c = pa[k] * read_f32(imgs[k], W, H, strides[k], cx, cy, modes[k], cvals[k],
+                                          &undef) + pb[k];
         for (int yf = -n; yf <= n; ++yf)
             for (int xf = -m; xf <= m; ++xf) {
                 const double M = masks[k][(yf + n) * mws[k] + (xf + m)];
-                const double v = read_f32(imgs[k], W, H, strides[k], cx + xf, cy + yf, modes[k],
-                                          cvals[k], &undef);
+                const double v = pa[k] * read_f32(imgs[k], W, H, strides[k], cx + xf, cy + yf,
+                                                  modes[k], cvals[k], &undef) + pb[k];
                 if (op == 0) {
                     acc += tap_fn_f64(fn, M, v, c);
                 } else if (M != 0.0) {
@@ -473,19 +477,21 @@ static double local_px_f32(int K, const float *const *imgs, const int64_t *strid
 static int64_t local_px_u8(int K, const uint8_t *const *imgs, const int64_t *strides, int64_t W,
                            int64_t H, const int32_t *const *masks, const int *mws, const int *mhs,
                            const int *oxs, const int *oys, const int *modes, const int64_t *cvals,
-                           int op, int fn, int64_t x, int64_t y, uint8_t *valid)
+                           const int64_t *pa, const int64_t *pb, int op, int fn, int64_t x,
+                           int64_t y, uint8_t *valid)
 {
     int undef = 0, first = 1;
     int64_t acc = 0;
     for (int k = 0; k < K; ++k) {
         const int m = mws[k] / 2, n = mhs[k] / 2;
         const int64_t cx = x + oxs[k], cy = y + oys[k];
-        const int64_t c = read_u8(imgs[k], W, H, strides[k], cx, cy, modes[k], cvals[k], &undef);
+        const int64_t c = pa[k] * read_u8(imgs[k], W, H, strides[k], cx, cy, modes[k], cvals[k],
+                                          &undef) + pb[k];
         for (int yf = -n; yf <= n; ++yf)
             for (int xf = -m; xf <= m; ++xf) {
                 const int64_t M = masks[k][(yf + n) * mws[k] + (xf + m)];
-                const int64_t v = read_u8(imgs[k], W, H, strides[k], cx + xf, cy + yf, modes[k],
-                                          cvals[k], &undef);
+                const int64_t v = pa[k] * read_u8(imgs[k], W, H, strides[k], cx + xf, cy + yf,
+                                                  modes[k], cvals[k], &undef) + pb[k];
                 if (op == 0) {
                     acc += tap_fn_i64(fn, M, v, c);
                 } else if (M != 0) {
@@ -502,27 +508,29 @@ static int64_t local_px_u8(int K, const uint8_t *const *imgs, const int64_t *str
 void oracle_local_f32(int K, const float *const *imgs, const int64_t *strides, int64_t W,
                       int64_t H, const double *const *masks, const int *mws, const int *mhs,
                       const int *oxs, const int *oys, const int *modes, const double *cvals,
-                      int op, int fn, int64_t y0, int64_t y1, double *out, uint8_t *valid)
+                      const double *pa, const double *pb, int op, int fn, int64_t y0, int64_t y1,
+                      double *out, uint8_t *valid)
 {
 #pragma omp parallel for schedule(dynamic, 1)
     for (int64_t y = y0; y < y1; ++y)
         for (int64_t x = 0; x < W; ++x) {
             int64_t o = (y - y0) * W + x;
             out[o] = local_px_f32(K, imgs, strides, W, H, masks, mws, mhs, oxs, oys, modes, cvals,
-                                  op, fn, x, y, &valid[o]);
+                                  pa, pb, op, fn, x, y, &valid[o]);
         }
 }
 
 void oracle_local_u8(int K, const uint8_t *const *imgs, const int64_t *strides, int64_t W,
                      int64_t H, const int32_t *const *masks, const int *mws, const int *mhs,
                      const int *oxs, const int *oys, const int *modes, const int64_t *cvals,
-                     int op, int fn, int64_t y0, int64_t y1, int64_t *out, uint8_t *valid)
+                     const int64_t *pa, const int64_t *pb, int op, int fn, int64_t y0, int64_t y1,
+                     int64_t *out, uint8_t *valid)
 {
 #pragma omp parallel for schedule(dynamic, 1)
     for (int64_t y = y0; y < y1; ++y)
         for (int64_t x = 0; x < W; ++x) {
             int64_t o = (y - y0) * W + x;
             out[o] = local_px_u8(K, imgs, strides, W, H, masks, mws, mhs, oxs, oys, modes, cvals,
-                                 op, fn, x, y, &valid[o]);
+                                 pa, pb, op, fn, x, y, &valid[o]);
         }
 }

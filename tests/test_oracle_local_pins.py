@@ -136,3 +136,55 @@ def test_undefined_valid_region_is_the_largest_window():
     ok = (xs + 1 >= 0) & (xs + 3 <= 11) & (ys - 1 >= 0) & (ys + 1 <= 11)
     ok &= (xs - 2 >= 0) & (xs + 2 <= 11) & (ys - 3 >= 0) & (ys + 3 <= 11)
     assert np.array_equal(valid, ok)
+
+
+# ---------------------------------------- point-operator prologue (reading c27) ----
+
+@pytest.mark.parametrize("mode", MODES)
+def test_point_prologue_is_the_local_operator_of_the_mapped_image(mode):
+    """Read'_k = a Read_k + b: the result equals the
+    operator applied to the explicitly mapped image a I + b with the
+    constant mapped too (a boundary constant is a pixel value), for every
+    op / tap function -- checked against scipy on the mapped image."""
+    img = _img(9, 13, 21).astype(np.float64)
+    a, b = 2.5, -0.75
+    mask = np.random.default_rng(22).random((3, 5))
+    got, _ = oracle.local([img.astype(np.float32)], [mask], "sum", "product", mode, 0.2,
+                          point=[(a, b)])
+    f32 = img.astype(np.float32).astype(np.float64)
+    ref = ndi.correlate(a * f32 + b, mask, mode=SCIPY_MODE[mode], cval=a * 0.2 + b)
+    assert np.allclose(got, ref, rtol=0, atol=1e-12)
+    # SQDIFF about the mapped centre: a^2 times the unmapped result (b cancels)
+    g1, _ = oracle.local([img.astype(np.float32)], [mask], "sum", "sqdiff", mode, 0.2,
+                         point=[(a, b)])
+    g0, _ = oracle.local([img.astype(np.float32)], [mask], "sum", "sqdiff", mode, 0.2)
+    assert np.allclose(g1, a * a * g0, rtol=1e-13, atol=1e-13)
+
+
+def test_point_prologue_u8_integer_and_per_accessor():
+    rng = np.random.default_rng(23)
+    u = rng.integers(0, 256, (10, 12)).astype(np.uint8)
+    v = rng.integers(0, 256, (10, 12)).astype(np.uint8)
+    m = np.ones((3, 3), np.int32)
+    got, _ = oracle.local([u, v], [m, m], "sum", "product", "clamp", point=[(-1, 255), (3, 0)])
+    ref = (ndi.correlate(255 - u.astype(np.int64), m.astype(np.int64), mode="nearest")
+           + ndi.correlate(3 * v.astype(np.int64), m.astype(np.int64), mode="nearest"))
+    assert np.array_equal(got, ref)
+
+
+# ------------------------------------ global merge: sum of squares (reading c26) ----
+
+def test_global_sumsq_exact():
+    """sum of squares: the exact sum (fractions.Fraction) of v^2 correctly
+    rounded; a constant image v gives v^2 N; u8 an exact integer; a ramp the
+    closed form sum_{k<n} k^2 = (n-1) n (2n-1) / 6."""
+    from fractions import Fraction
+    img = np.random.default_rng(24).random((17, 19)).astype(np.float32)
+    exact = sum(Fraction(float(x)) ** 2 for x in img.ravel())
+    assert oracle.global_reduce(img, "sumsq") == float(exact)
+    assert oracle.global_reduce(np.full((7, 9), 0.5, np.float32), "sumsq") == 0.25 * 63
+    n = 2000
+    ramp = np.arange(n, dtype=np.float32).reshape(40, 50)
+    assert oracle.global_reduce(ramp, "sumsq") == (n - 1) * n * (2 * n - 1) / 6
+    u8 = (np.arange(512) % 256).astype(np.uint8).reshape(2, 16, 16)
+    assert oracle.global_reduce(u8, "sumsq") == 2 * 255 * 256 * 511 / 6
