@@ -201,7 +201,12 @@ lop_status lop_convolve_chain_execute_ws(const lop_iteration_space *is, const lo
  * (LOP_ERR_INVALID otherwise).  Window: odd, up to 63 x 63, equal to the
  * BoundaryCondition's; boundary modes as for every local operator (Table I).
  * Exact: every output is an input value or the constant. */
-typedef enum { LOP_REDUCE_SUM = 0, LOP_REDUCE_MIN = 1, LOP_REDUCE_MAX = 2 } lop_reduce_op;
+typedef enum {
+    LOP_REDUCE_SUM = 0,
+    LOP_REDUCE_MIN = 1,
+    LOP_REDUCE_MAX = 2,
+    LOP_REDUCE_SUMSQ = 3        /* global operators only (lop_global_reduce_execute) */
+} lop_reduce_op;
 lop_status lop_reduce_execute(const lop_iteration_space *is, const lop_accessor *in,
                               const lop_mask *domain, int32_t op, void *cuda_stream);
 
@@ -224,14 +229,18 @@ lop_status lop_convolve2_execute(const lop_iteration_space *is, const lop_access
                                  void *cuda_stream);
 
 /* Global operator (one output for all pixels, "e.g. the
- * sum of all pixels"): SUM, MIN or MAX of the pixels of the
+ * sum of all pixels"): SUM, MIN, MAX or SUMSQ of the pixels of the
  * region (x0, y0, width, height) of is->image (here the INPUT; width/height 0
  * = to the image edge), over all frames of a batch.  The result is one double
  * written to device memory d_result; d_work is a device scratch array of
  * LOP_GLOBAL_WORK_DOUBLES doubles owned by the caller, ZERO-initialised before
  * its first use (its last element is an arrival counter that every call leaves
  * at zero again; calls sharing one d_work must be ordered on one stream).
- * F32 (sum accumulated in double) or U8 (exact integer sum).  Deterministic:
+ * SUMSQ merges two pixels a, b into a^2 + b^2 ("operations
+ * that merge/reduce two pixels"; reading c26): the sum of squares, which with
+ * SUM gives a region's mean and variance.
+ * F32 (sums accumulated in double; an f32 value's square is exact in double) or
+ * U8 (exact integer sums).  Deterministic:
  * fixed partition and fixed reduction trees, so the same input gives the same
  * bits on every run.  Asynchronous on cuda_stream (one kernel launch). */
 #define LOP_GLOBAL_WORK_DOUBLES 1025
@@ -275,6 +284,23 @@ typedef enum {
 lop_status lop_local_execute(const lop_iteration_space *is, const lop_accessor *const *inputs,
                              const lop_mask *const *masks, int32_t n_inputs, int32_t op,
                              int32_t tap_fn, void *cuda_stream);
+/* The same local operator with a point-operator prologue per accessor
+ * (point operators precede local ones in an image
+ * pipeline; reading c27): every read of accessor k -- the window taps, its
+ * centre c_k and, in LOP_CONSTANT mode, the boundary constant -- is replaced by
+ *   Read'_k = scale[k] * Read_k + offset[k]
+ * before the tap function (window/level, inversion, gain) without the mapped
+ * image making a round trip through HBM.  scale / offset: n_inputs host
+ * doubles each (NULL = 1 / 0 for every accessor).  F32 inputs: scale and
+ * offset are rounded to f32 and applied as one f32 FMA when the footprint is
+ * staged; U8 inputs: integers with |scale|, |offset| <= 2^16 (exact int32
+ * arithmetic; LOP_ERR_INVALID otherwise), and the result's worst case must
+ * fit int32 (LOP_ERR_UNSUPPORTED otherwise).  lop_local_execute is this call
+ * with scale = offset = NULL. */
+lop_status lop_local_execute_point(const lop_iteration_space *is, const lop_accessor *const *inputs,
+                                   const lop_mask *const *masks, int32_t n_inputs, int32_t op,
+                                   int32_t tap_fn, const double *scale, const double *offset,
+                                   void *cuda_stream);
 
 /* Algorithm 2, the kernel-configuration heuristic, as a
  * pure host function (no CUDA call; the library feeds it cudaOccupancy*

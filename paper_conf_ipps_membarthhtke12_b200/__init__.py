@@ -242,7 +242,8 @@ def reduce(x: torch.Tensor, domain, op="min", mode="clamp", constant=0.0, out=No
 
 def global_reduce(x: torch.Tensor, op="sum", roi=None, out=None, work=None,
                   stream=None) -> torch.Tensor:
-    """Global operator: "sum" / "min" / "max" of the pixels
+    """Global operator: "sum" / "min" / "max" / "sumsq"
+    (the sum of squares; reading c26) of the pixels
     of ``roi`` over all frames, as a 1-element float64 CUDA tensor (written
     asynchronously; deterministic).  ``work``: a reusable zero-initialised
     float64 scratch tensor of LOP_GLOBAL_WORK_DOUBLES elements."""
@@ -255,24 +256,28 @@ def global_reduce(x: torch.Tensor, op="sum", roi=None, out=None, work=None,
     if roi is not None:
         is_.x0, is_.y0, is_.width, is_.height = (int(v) for v in roi)
     with torch.cuda.device(x.device):
-        _check(lib.lop_global_reduce_execute(ctypes.byref(is_), _REDUCE[op], out.data_ptr(),
+        _check(lib.lop_global_reduce_execute(ctypes.byref(is_), _GLOBAL[op], out.data_ptr(),
                                              work.data_ptr(), _stream_handle(x, stream)))
     return out
 
 
+_GLOBAL = dict(_REDUCE, sumsq=_lib.LOP_REDUCE_SUMSQ)
 _TAP = {"product": _lib.LOP_TAP_PRODUCT, "absdiff": _lib.LOP_TAP_ABSDIFF,
         "sqdiff": _lib.LOP_TAP_SQDIFF, "square": _lib.LOP_TAP_SQUARE}
 
 
 def local(inputs, masks, op="sum", fn="product", modes="clamp", constants=0.0, offsets=None,
-          out=None, roi=None, stream=None, band=None) -> torch.Tensor:
+          out=None, roi=None, stream=None, band=None, point=None) -> torch.Tensor:
     """Local operator over several Accessors with a per-tap function
     (lop_local_execute; Listing 9):
     out = op over k, taps of fn(M_k, Read_k(x+ox_k+xf, y+oy_k+yf), centre_k).
     inputs: up to 4 CUDA images of one shape and dtype (float32 -> float32,
     uint8 -> int32); masks: one 2D host mask per input (its window);
     modes / constants / offsets: per input (or one value for all); band: per input
-    (halo_top, halo_bottom, global_y0, global_height) for row-band views."""
+    (halo_top, halo_bottom, global_y0, global_height) for row-band views;
+    point: per input (scale, offset) of a point-operator prologue
+    Read' = scale * Read + offset (lop_local_execute_point; PAPER.md
+    L107-L122, reading c27), None = identity."""
     K = len(inputs)
     if K != len(masks):
         raise ValueError("one mask per input")
@@ -304,8 +309,16 @@ def local(inputs, masks, op="sum", fn="product", modes="clamp", constants=0.0, o
     if roi is not None:
         is_.x0, is_.y0, is_.width, is_.height = (int(v) for v in roi)
     with torch.cuda.device(x0.device):
-        _check(lib.lop_local_execute(ctypes.byref(is_), acc_arr, m_arr, K, _REDUCE[op], _TAP[fn],
-                                     _stream_handle(x0, stream)))
+        if point is None:
+            _check(lib.lop_local_execute(ctypes.byref(is_), acc_arr, m_arr, K, _REDUCE[op],
+                                         _TAP[fn], _stream_handle(x0, stream)))
+        else:
+            if len(point) != K:
+                raise ValueError("one (scale, offset) per input")
+            sc = (ctypes.c_double * K)(*[float(a) for a, _ in point])
+            of = (ctypes.c_double * K)(*[float(b) for _, b in point])
+            _check(lib.lop_local_execute_point(ctypes.byref(is_), acc_arr, m_arr, K, _REDUCE[op],
+                                               _TAP[fn], sc, of, _stream_handle(x0, stream)))
     del keep
     return out
 

@@ -16,7 +16,7 @@ LOP_OK, LOP_ERR_INVALID, LOP_ERR_UNSUPPORTED, LOP_ERR_CUDA = 0, -1, -2, -3
 LOP_U8, LOP_I32, LOP_F32 = 0, 1, 2
 LOP_UNDEFINED, LOP_CLAMP, LOP_REPEAT, LOP_MIRROR, LOP_CONSTANT = 0, 1, 2, 3, 4
 LOP_VARIANT_AUTO, LOP_VARIANT_GENERIC, LOP_VARIANT_TILED = 0, 1, 2
-LOP_REDUCE_SUM, LOP_REDUCE_MIN, LOP_REDUCE_MAX = 0, 1, 2
+LOP_REDUCE_SUM, LOP_REDUCE_MIN, LOP_REDUCE_MAX, LOP_REDUCE_SUMSQ = 0, 1, 2, 3
 LOP_COMBINE_L2, LOP_COMBINE_L1, LOP_COMBINE_SUMSQ = 0, 1, 2
 LOP_GLOBAL_WORK_DOUBLES = 1025
 LOP_TAP_PRODUCT, LOP_TAP_ABSDIFF, LOP_TAP_SQDIFF, LOP_TAP_SQUARE = 0, 1, 2, 3
@@ -89,6 +89,10 @@ SIGNATURES = {
                                   ctypes.POINTER(ctypes.POINTER(lop_accessor)),
                                   ctypes.POINTER(ctypes.POINTER(lop_mask)), c_i32, c_i32, c_i32,
                                   c_vp]),
+    "lop_local_execute_point": (c_i32, [ctypes.POINTER(lop_iteration_space),
+                                        ctypes.POINTER(ctypes.POINTER(lop_accessor)),
+                                        ctypes.POINTER(ctypes.POINTER(lop_mask)), c_i32, c_i32,
+                                        c_i32, c_vp, c_vp, c_vp]),
     "lop_alg2_select": (c_i32, [c_vp, c_i32, c_i32, c_i32, c_i32, c_i32, c_i32,
                                 ctypes.POINTER(c_i64)]),
     "lop_mask_closeness": (c_i32, [c_flt, c_i32, c_i32, c_vp]),

@@ -43,10 +43,25 @@ def headers():
     return hs + [os.path.join(INCLUDE, "lop.h")]
 
 
+def deps(src: str, seen=None) -> set:
+    """The in-tree headers `src` includes, transitively (#include "...")."""
+    import re
+    seen = set() if seen is None else seen
+    with open(src) as f:
+        for name in re.findall(r'^\s*#\s*include\s+"([^"]+)"', f.read(), re.M):
+            for d in (CSRC, INCLUDE):
+                h = os.path.join(d, name)
+                if os.path.exists(h) and h not in seen:
+                    seen.add(h)
+                    deps(h, seen)
+                    break
+    return seen
+
+
 def _compile(src: str, force: bool, verbose: bool) -> str:
     unit = os.path.splitext(os.path.basename(src))[0]
     obj = os.path.join(BUILD, unit + ".o")
-    newest_dep = max([os.path.getmtime(src)] + [os.path.getmtime(h) for h in headers()])
+    newest_dep = max([os.path.getmtime(src)] + [os.path.getmtime(h) for h in deps(src)])
     if not force and os.path.exists(obj) and os.path.getmtime(obj) >= newest_dep:
         return obj
     cmd = [nvcc(), *ARCH, "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC",

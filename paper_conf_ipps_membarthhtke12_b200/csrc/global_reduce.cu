@@ -1,8 +1,11 @@
 // global_reduce.cu -- global operators ("global operators
 // (e.g., reduction operators) produce one output for the operator applied to
 // all pixels of the image (e.g., compute the sum of all pixels)"; SURVEY §8(f)
-// N3 "global reductions (sum/min/max)"): SUM, MIN or MAX over the pixels of a
-// region of interest (all frames of a batch).
+// N3 "global reductions (sum/min/max)"): SUM, MIN, MAX or SUMSQ over the pixels
+// of a region of interest (all frames of a batch).  SUMSQ is the merge
+// a, b -> a^2 + b^2 of PAPER.md L956-L959 ("operations that merge/reduce two
+// pixels"; reading c26): f32 squares are exact in double, u8 squares are
+// byte dot products of a word with itself (IDP4A), exact.
 //
 // Deterministic: a fixed number of CTAs (kGlobalParts, independent of the GPU)
 // each reduce a fixed contiguous block of rows -- every thread a fixed set of
@@ -57,12 +60,16 @@ __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_c
     const int64_t rows = (int64_t)c.batch * c.roi_h;
     const int64_t r0 = rows * blockIdx.x / kGlobalParts, r1 = rows * (blockIdx.x + 1) / kGlobalParts;
     constexpr bool F = sizeof(T) == 4;
-    // per-thread accumulators in the cheapest exact form: f32 SUM in double;
-    // f32 MIN / MAX in float (exact); u8 SUM in int32 by byte dot products
-    // (IDP4A); u8 MIN / MAX on bytes in 16-bit lanes
+    // per-thread accumulators in the cheapest exact form: f32 SUM / SUMSQ in
+    // double; f32 MIN / MAX in float (exact); u8 SUM in int32 by byte dot
+    // products (IDP4A); u8 SUMSQ by dot products of a word with itself, per
+    // batch of loads in 32 bits (<= 128 x 255^2) then in 64; u8 MIN / MAX on
+    // bytes in 16-bit lanes
+    constexpr bool SQ = OP == RED_SUMSQ;
     double dacc = 0.0;
     float facc = OP == RED_MIN ? __int_as_float(0x7f800000) : -__int_as_float(0x7f800000);
     unsigned int iacc = 0;
+    unsigned long long lacc = 0;
     // u8 MIN / MAX: even and odd bytes in the 16-bit lanes of two accumulators
     // (native VIMNMX.U16x2; __vminu4 / __vmaxu4 are emulated on sm_100)
     uint32_t eacc = OP == RED_MIN ? 0x00FF00FFu : 0u, oacc = eacc;
@@ -72,6 +79,7 @@ __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_c
             w = OP == RED_MIN ? (w | ~keep) : (w & keep);
         }
         if (OP == RED_SUM) iacc = __dp4a(w, 0x01010101u, iacc);   // unsigned bytes, exact
+        else if (SQ) iacc = __dp4a(w, w, iacc);                    // sum of the 4 squares
         else {
             const uint32_t e = w & 0x00FF00FFu, o = (w >> 8) & 0x00FF00FFu;
             eacc = OP == RED_MIN ? __vminu2(eacc, e) : __vmaxu2(eacc, e);
@@ -80,6 +88,7 @@ __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_c
     };
     auto add_f = [&](float v) {
         if (OP == RED_SUM) dacc += (double)v;
+        else if (SQ) dacc = fma((double)v, (double)v, dacc);      // exact square, one rounding
         else facc = OP == RED_MIN ? fminf(facc, v) : fmaxf(facc, v);
     };
     constexpr int V = 16 / (int)sizeof(T);                       // elements per 16-B load
@@ -100,7 +109,7 @@ __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_c
     };
     const char *rowp = row_at(b, y);
     // Identity element of the operator (partial groups are padded with it).
-    const float fid = OP == RED_SUM ? 0.0f : (OP == RED_MIN ? __int_as_float(0x7f800000)
+    const float fid = OP == RED_SUM || SQ ? 0.0f : (OP == RED_MIN ? __int_as_float(0x7f800000)
                                                            : -__int_as_float(0x7f800000));
     const uint32_t bid = OP == RED_MIN ? 0xFFFFFFFFu : 0u;
     const uint32_t idw = F ? __float_as_uint(fid) : bid;
@@ -139,10 +148,12 @@ __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_c
                 add_word(q[u].x, 4); add_word(q[u].y, 4); add_word(q[u].z, 4); add_word(q[u].w, 4);
             }
         }
+        if constexpr (!F && SQ) { lacc += iacc; iacc = 0; }
     }
     double acc;
-    if constexpr (F) acc = OP == RED_SUM ? dacc : (double)facc;
+    if constexpr (F) acc = OP == RED_SUM || SQ ? dacc : (double)facc;
     else if (OP == RED_SUM) acc = (double)iacc;                   // exact (partials < 2^31)
+    else if (SQ) acc = (double)lacc;                              // exact (partials < 2^53)
     else {
         const uint32_t l = OP == RED_MIN ? __vminu2(eacc, oacc) : __vmaxu2(eacc, oacc);
         const uint32_t m = OP == RED_MIN ? min(l & 0xFFFFu, l >> 16) : max(l & 0xFFFFu, l >> 16);
@@ -202,6 +213,7 @@ cudaError_t launch_global_op(const GlobalReduce &p, cudaStream_t stream)
     case RED_SUM: return launch_global_t<T, RED_SUM>(p, stream);
     case RED_MIN: return launch_global_t<T, RED_MIN>(p, stream);
     case RED_MAX: return launch_global_t<T, RED_MAX>(p, stream);
+    case RED_SUMSQ: return launch_global_t<T, RED_SUMSQ>(p, stream);
     default: return cudaErrorNotSupported;
     }
 }

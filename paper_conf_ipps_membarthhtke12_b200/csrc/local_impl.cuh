@@ -7,6 +7,10 @@
 //                        of a per-tap function (reading c22: a fixed set).
 //   out(x, y) = op_{k, yf, xf} f(M_k(xf, yf), Read_k(x + ox_k + xf,
 //                                 y + oy_k + yf), Read_k(x + ox_k, y + oy_k))
+// with an optional point-operator prologue per accessor (
+// reading c27): Read'_k = a_k Read_k + b_k, applied once per staged element
+// (tiled kernels: in shared memory after staging, so the boundary constant is
+// mapped too) or per read (generic kernel) -- the same value either way.
 //
 // Two kernels with the same per-output arithmetic in the same order (so the
 // outputs are bit-identical, tested):
@@ -124,6 +128,20 @@ __device__ __forceinline__ auto local_read(const LocalAcc &a, int b, int ix, int
     else return read_f32(a.in, b, ix, iy, a.mode, a.cval_f);
 }
 
+// Point-operator prologue (reading c27): f32 one FMA (a, b rounded to f32),
+// u8 exact int32 (|a|, |b| <= 2^16 checked by the API).
+__device__ __forceinline__ float local_point(const LocalAcc &a, float v) { return __fmaf_rn(a.pa_f, v, a.pb_f); }
+__device__ __forceinline__ int local_point(const LocalAcc &a, int v) { return a.pa_i * v + a.pb_i; }
+
+// Map the n staged elements t[0..n) of accessor a in place (all threads of
+// the CTA; the caller synchronises before and after).
+template <typename V>
+__device__ __forceinline__ void local_point_stage(const LocalAcc &a, V *t, int n)
+{
+    const int tid = threadIdx.y * blockDim.x + threadIdx.x, nthr = blockDim.x * blockDim.y;
+    for (int i = tid; i < n; i += nthr) t[i] = local_point(a, t[i]);
+}
+
 // Is accessor a's footprint of output rectangle [x0, x0+w) x [y0, y0+h)
 // inside the image (global rows, columns)?  Then no boundary handling.
 __device__ __forceinline__ bool local_interior(const LocalAcc &a, int x0, int y0, int w, int h)
@@ -212,7 +230,6 @@ __global__ void __launch_bounds__(1024) local_tiled_kernel(const __grid_constant
     const int tx0 = c.roi_x0 + blockIdx.x * tw, ty0 = c.roi_y0 + blockIdx.y * th;
     const int roi_x1 = c.roi_x0 + c.roi_w, roi_y1 = c.roi_y0 + c.roi_h;
     const int rows = min(th, roi_y1 - ty0);               // output rows of this tile
-    const int tid = threadIdx.y * blockDim.x + threadIdx.x, nthr = blockDim.x * blockDim.y;
     // stage every accessor's footprint (only the rows the tile's outputs need)
     int base = 0;
     for (int k = 0; k < p.n; ++k) {
@@ -223,6 +240,16 @@ __global__ void __launch_bounds__(1024) local_tiled_kernel(const __grid_constant
         base += sw * sh;
     }
     __syncthreads();
+    if (p.any_point) {                                     // point-operator prologue
+        base = 0;
+        for (int k = 0; k < p.n; ++k) {
+            const LocalAcc &a = p.acc[k];
+            const int n = (tw + 2 * a.rx) * (rows + 2 * a.ry);
+            if (a.point) local_point_stage(a, sm + base, n);
+            base += n;
+        }
+        __syncthreads();
+    }
 
     const int x = tx0 + threadIdx.x;
     const int y0 = OY * threadIdx.y;                       // first output row (tile-relative)
@@ -360,6 +387,16 @@ __global__ void __launch_bounds__(256) local_small_kernel(const __grid_constant_
     }
     mbar_wait(&sbar, 0);
     __syncthreads();
+    if (p.any_point) {                                     // point-operator prologue
+        base = 0;
+        for (int k = 0; k < p.n; ++k) {
+            const LocalAcc &a = p.acc[k];
+            const int n = (th + 2 * a.ry) * pitch;
+            if (a.point) local_point_stage(a, sm + base, n);
+            base += n;
+        }
+        __syncthreads();
+    }
 
     const int c0 = SX * threadIdx.x;                       // tile-relative first column
     const int r0 = OY * threadIdx.y;                       // tile-relative first row
@@ -456,13 +493,17 @@ __global__ void __launch_bounds__(1024) local_generic_kernel(const __grid_consta
         // boundary resolution (Algorithm 2 counts the others' threads)
         const bool interior = local_interior(a, bx0, by0, blockDim.x, blockDim.y);
         const char *fb = a.in.data + (int64_t)b * a.in.bstride;
-        auto rd = [&](int xx, int yy) -> V {
+        auto rd0 = [&](int xx, int yy) -> V {
             if (interior) {
                 const char *rp = fb + (int64_t)yy * a.in.stride;
                 if constexpr (U8) return (int)__ldg(reinterpret_cast<const uint8_t *>(rp) + xx);
                 else return __ldg(reinterpret_cast<const float *>(rp) + xx);
             }
             return local_read<U8>(a, b, xx, yy);
+        };
+        auto rd = [&](int xx, int yy) -> V {
+            const V v = rd0(xx, yy);
+            return a.point ? local_point(a, v) : v;
         };
         const V cen = rd(ix, iy);
         const V *mk = (const V *)(U8 ? (const void *)(p.m.i + a.moff) : (const void *)(p.m.f + a.moff));

@@ -600,8 +600,8 @@ lop_status lop_global_reduce_execute(const lop_iteration_space *is, int32_t op, 
 {
     static_assert(lop::kGlobalCounter + 1 == LOP_GLOBAL_WORK_DOUBLES, "work size");
     if (!is) return fail(LOP_ERR_INVALID, "iteration space is NULL");
-    if (op != LOP_REDUCE_SUM && op != LOP_REDUCE_MIN && op != LOP_REDUCE_MAX)
-        return fail(LOP_ERR_INVALID, "unknown reduction %d (SUM, MIN, MAX)", op);
+    if (op != LOP_REDUCE_SUM && op != LOP_REDUCE_MIN && op != LOP_REDUCE_MAX && op != LOP_REDUCE_SUMSQ)
+        return fail(LOP_ERR_INVALID, "unknown reduction %d (SUM, MIN, MAX, SUMSQ)", op);
     if (!d_result || !d_work) return fail(LOP_ERR_INVALID, "d_result / d_work is NULL");
     lop_status st = check_image(is->image, "image");
     if (st) return st;
@@ -628,7 +628,8 @@ lop_status lop_global_reduce_execute(const lop_iteration_space *is, int32_t op, 
         return fail(LOP_ERR_INVALID, "region [%d,%d)+%dx%d outside the %d x %d image", is->x0,
                     is->y0, p.c.roi_w, p.c.roi_h, im.width, im.height);
     p.c.batch = im.batch;
-    p.op = op == LOP_REDUCE_SUM ? lop::RED_SUM : (op == LOP_REDUCE_MIN ? lop::RED_MIN : lop::RED_MAX);
+    p.op = op == LOP_REDUCE_SUM ? lop::RED_SUM : op == LOP_REDUCE_MIN ? lop::RED_MIN
+         : op == LOP_REDUCE_MAX ? lop::RED_MAX : lop::RED_SUMSQ;
     p.u8 = im.dtype == LOP_U8;
     p.work = d_work;
     p.result = d_result;
@@ -875,6 +876,15 @@ lop_status lop_local_execute(const lop_iteration_space *is, const lop_accessor *
                              const lop_mask *const *masks, int32_t n_inputs, int32_t op,
                              int32_t tap_fn, void *cuda_stream)
 {
+    return lop_local_execute_point(is, inputs, masks, n_inputs, op, tap_fn, nullptr, nullptr,
+                                   cuda_stream);
+}
+
+lop_status lop_local_execute_point(const lop_iteration_space *is, const lop_accessor *const *inputs,
+                                   const lop_mask *const *masks, int32_t n_inputs, int32_t op,
+                                   int32_t tap_fn, const double *scale, const double *offset,
+                                   void *cuda_stream)
+{
     if (!inputs || !masks) return fail(LOP_ERR_INVALID, "inputs / masks is NULL");
     if (n_inputs < 1 || n_inputs > LOP_MAX_ACCESSORS)
         return fail(LOP_ERR_INVALID, "n_inputs %d outside 1..%d", n_inputs, LOP_MAX_ACCESSORS);
@@ -889,7 +899,7 @@ lop_status lop_local_execute(const lop_iteration_space *is, const lop_accessor *
     int taps = 0, rx = 0, ry = 0;
     bool any_tap = false;
     double bound = 0.0;                               // worst-case |out| (integer path)
-    const double gmax = tap_fn == LOP_TAP_SQDIFF || tap_fn == LOP_TAP_SQUARE ? 255.0 * 255.0 : 255.0;
+    p.any_point = 0;
     for (int k = 0; k < n_inputs; ++k) {
         Prepared pp;
         lop_status st = prepare(is, inputs[k], pp);
@@ -929,6 +939,31 @@ lop_status lop_local_execute(const lop_iteration_space *is, const lop_accessor *
         a.cval_f = c.cval_f;
         a.cval_i = c.cval_i;
         a.moff = taps;
+        // point-operator prologue Read' = pa * Read + pb (reading c27)
+        const double pa = scale ? scale[k] : 1.0, pb = offset ? offset[k] : 0.0;
+        if (!std::isfinite(pa) || !std::isfinite(pb))
+            return fail(LOP_ERR_INVALID, "accessor %d: point operator %g * v + %g not finite", k, pa, pb);
+        double lo = 0.0, hi = 255.0;                  // range of the (mapped) reads, u8 path
+        if (p.u8) {
+            if (pa != std::floor(pa) || pb != std::floor(pb) || std::fabs(pa) > 65536.0 ||
+                std::fabs(pb) > 65536.0)
+                return fail(LOP_ERR_INVALID,
+                            "accessor %d: U8 point operator needs integers |scale|, |offset| <= 2^16", k);
+            a.pa_i = (int32_t)pa;
+            a.pb_i = (int32_t)pb;
+            a.point = a.pa_i != 1 || a.pb_i != 0;
+            lo = std::min(pb, 255.0 * pa + pb);
+            hi = std::max(pb, 255.0 * pa + pb);
+        } else {
+            a.pa_f = (float)pa;
+            a.pb_f = (float)pb;
+            a.point = a.pa_f != 1.0f || a.pb_f != 0.0f;
+        }
+        p.any_point |= a.point;
+        const double vmax = std::max(std::fabs(lo), std::fabs(hi));
+        const double gmax = tap_fn == LOP_TAP_SQDIFF ? (hi - lo) * (hi - lo)
+                          : tap_fn == LOP_TAP_SQUARE ? vmax * vmax
+                          : tap_fn == LOP_TAP_ABSDIFF ? hi - lo : vmax;
         double l1 = 0.0, mx = 0.0;
         for (int i = 0; i < sx * sy; ++i) {
             if (p.u8) {

@@ -109,7 +109,7 @@ struct ConvSep {
 // Local reduction over a mask domain (Listing 9's convolve(mask, <reduction>, f)
 // with the MIN / MAX reductions; reduce.cu): out = min / max of Read(x+xf, y+yf)
 // over the taps where the mask is non-zero.  dom[yf + ry] bit (xf + rx) = tap.
-enum ReduceOp { RED_SUM = 0, RED_MIN = 1, RED_MAX = 2 };
+enum ReduceOp { RED_SUM = 0, RED_MIN = 1, RED_MAX = 2, RED_SUMSQ = 3 };   // SUMSQ: global only
 struct ReduceParams {
     Common c;
     int32_t op;                      // RED_MIN / RED_MAX
@@ -128,7 +128,7 @@ constexpr int kGlobalCounter = 1024;                         // + 1 = LOP_GLOBAL
 static_assert(kGlobalParts <= kGlobalCounter && kGlobalParts % 256 == 0, "global parts");
 struct GlobalReduce {
     Common c;                    // c.in: the image; c.roi_*: the region; c.batch
-    int32_t op;                  // RED_SUM / RED_MIN / RED_MAX
+    int32_t op;                  // RED_SUM / RED_MIN / RED_MAX / RED_SUMSQ
     int32_t u8;
     double *work;                // kGlobalParts doubles, arrival counter at [kGlobalCounter]
     double *result;              // 1 double (device)
@@ -185,6 +185,9 @@ struct LocalAcc {
     float cval_f;
     int32_t cval_i;
     int32_t moff;
+    int32_t point;               // point-operator prologue Read' = pa * Read + pb (reading c27)
+    float pa_f, pb_f;            // f32 images
+    int32_t pa_i, pb_i;          // u8 images (exact)
 };
 constexpr int kLocalSmallR = 7;                               // register-blocked path: radii <= 7
 constexpr int kLocalSmallW = 2 * kLocalSmallR + 1;
@@ -192,6 +195,7 @@ struct LocalParams {
     Common c;                    // output, ROI, batch, largest radii
     int32_t n, op, fn, u8;
     int32_t small;               // every radius <= kLocalSmallR: masks also in ms (15 x 15 slots)
+    int32_t any_point;           // some accessor has a point-operator prologue
     LocalAcc acc[kLocalMaxAcc];
     union {                      // mask k embedded centred in a 15 x 15 slot (zeros outside)
         float f[kLocalMaxAcc][kLocalSmallW * kLocalSmallW];

@@ -197,3 +197,69 @@ def test_local_validation(lop):
         lop.local([x], [m], out=x)
     with pytest.raises(lop.LopError, match="overflow"):
         lop.local([u], [np.full((31, 31), 4000, np.int32)], "sum", "square")
+
+
+# ------------------------------- point-operator prologue (reading c27, N3) ----
+
+@pytest.mark.parametrize("shape", [(1, 1), (5, 6), (67, 131), (260, 517)])
+@pytest.mark.parametrize("fn", FNS)
+def test_local_point_prologue_f32(lop, shape, fn):
+    """Read'_k = a_k Read_k + b_k on every read of accessor k (centre and
+    boundary constant included) against oracle.local(point=...), all modes,
+    both tiled kernels and the generic kernel (bit-identical to each other)."""
+    H, W = shape
+    rng = np.random.default_rng(H + W)
+    a, b = synthetic.uniform(H, W, seed=31), synthetic.uniform(H, W, seed=32)
+    masks = _masks(rng, [(5, 5), (3, 7)], False)
+    point = [(-0.5, 0.75), (1.0, -0.25)]                    # f32-exact scale / offset
+    for modes, offs in ((["clamp", "constant"], [(0, 0), (1, -1)]),
+                        (["mirror", "repeat"], [(-2, 0), (0, 2)]),
+                        (["undefined", "undefined"], [(0, 0), (0, 0)])):
+        outs = []
+        for variant in ("auto", "generic"):
+            lop.set_variant(variant)
+            outs.append(lop.local([a.cuda(), b.cuda()], masks, "sum", fn, modes, [0.25, 0.5], offs,
+                                  point=point))
+        lop.set_variant("auto")
+        assert torch.equal(outs[0], outs[1]), modes
+        ref, valid = oracle.local([a.numpy(), b.numpy()], masks, "sum", fn, modes, [0.25, 0.5],
+                                  offs, point=point)
+        _compare(outs[0].cpu().numpy(), ref, valid, False, modes)
+    # windows wider than 7 take the tiled (not the register-blocked) kernel
+    big = _masks(rng, [(11, 9)], False)
+    for op in OPS:
+        got = lop.local([a.cuda()], big, op, fn, "mirror", point=[(2.0, -1.0)])
+        ref, valid = oracle.local([a.numpy()], big, op, fn, "mirror", point=[(2.0, -1.0)])
+        _compare(got.cpu().numpy(), ref, valid, False, ["mirror"])
+
+
+@pytest.mark.parametrize("op", OPS)
+@pytest.mark.parametrize("fn", FNS)
+def test_local_point_prologue_u8_exact(lop, op, fn):
+    """u8: integer prologues (inversion 255 - v, gain 3 v) are exact."""
+    rng = np.random.default_rng(41)
+    H, W = 45, 133
+    imgs = [synthetic.uniform_u8(H, W, seed=s) for s in (43, 44)]
+    masks = _masks(rng, [(3, 3), (5, 5)], True)
+    point = [(-1, 255), (3, -7)]
+    got = lop.local([t.cuda() for t in imgs], masks, op, fn, ["clamp", "constant"], [0, 200],
+                    [(0, 0), (2, -1)], point=point)
+    ref, valid = oracle.local([t.numpy() for t in imgs], masks, op, fn, ["clamp", "constant"],
+                              [0, 200], [(0, 0), (2, -1)], point=point)
+    _compare(got.cpu().numpy(), ref, valid, True, [])
+
+
+def test_local_point_prologue_identity_and_validation(lop):
+    """scale 1 / offset 0 is bit-identical to lop_local_execute; non-integer
+    u8 prologues and int32 overflow are rejected."""
+    x = synthetic.angio(64, 96, seed=5).cuda()
+    m = [np.full((3, 3), 1.0 / 9, np.float32)]
+    assert torch.equal(lop.local([x], m, point=[(1.0, 0.0)]), lop.local([x], m))
+    u = synthetic.uniform_u8(16, 16, seed=6).cuda()
+    mi = [np.ones((3, 3), np.int32)]
+    with pytest.raises(lop.LopError):
+        lop.local([u], mi, point=[(0.5, 0)])
+    with pytest.raises(lop.LopError):
+        lop.local([u], [np.full((31, 31), 1000, np.int32)], fn="square", point=[(4, 0)])
+    with pytest.raises(ValueError):
+        lop.local([u], mi, point=[(1, 0), (1, 0)])

@@ -1018,3 +1018,37 @@ def test_bilateral_kernel_choice_by_whole_launch_size(lop, monkeypatch):
         y0, y1 = S // 2, S // 2 + S // 8
         band = run(img[y0:y1], band=(6, 6, y0, S))
         assert torch.equal(band, whole[y0:y1]), S
+
+
+@pytest.mark.parametrize("shape", [(1, 1), (7, 5), (130, 1031), (1024, 2048)])
+def test_global_sumsq(lop, shape):
+    """SUMSQ merge (reading c26): u8 exact; f32 within
+    1e-12 relative of the exact sum of squares; deterministic; regions and
+    frames (ragged / misaligned column groups)."""
+    H, W = shape
+    img = synthetic.uniform(H, W, seed=H + 2 * W)
+    u8 = synthetic.uniform_u8(H, W, seed=H * W + 3)
+    g = lop.global_reduce(img.cuda(), "sumsq").item()
+    ref = oracle.global_reduce(img.numpy(), "sumsq")
+    assert abs(g - ref) <= 1e-12 * max(1.0, abs(ref)), (g, ref)
+    assert lop.global_reduce(img.cuda(), "sumsq").item() == g
+    assert lop.global_reduce(u8.cuda(), "sumsq").item() == oracle.global_reduce(u8.numpy(), "sumsq")
+    full = torch.full((H, W), 255, dtype=torch.uint8)           # the largest squares
+    assert lop.global_reduce(full.cuda(), "sumsq").item() == 255.0 * 255.0 * H * W
+    if H > 10 and W > 10:
+        roi = (3, 5, W - 7, H - 9)
+        frames = torch.stack([img, img * -0.5, img + 0.25]).cuda()
+        g = lop.global_reduce(frames, "sumsq", roi=roi).item()
+        ref = oracle.global_reduce(frames.cpu().numpy(), "sumsq", roi=roi)
+        assert abs(g - ref) <= 1e-12 * max(1.0, abs(ref)), (g, ref)
+        uframes = torch.stack([u8, 255 - u8, u8 // 2]).cuda()
+        assert (lop.global_reduce(uframes, "sumsq", roi=roi).item() ==
+                oracle.global_reduce(uframes.cpu().numpy(), "sumsq", roi=roi))
+
+
+def test_global_sumsq_u8_4096_frames_exact(lop):
+    """u8 SUMSQ over 16 x 4096^2 frames of 255 (2^28 pixels): the exact
+    integer 255^2 * 2^28 (> 2^32: the 64-bit per-thread accumulation)."""
+    x = torch.full((16, 4096, 4096), 255, dtype=torch.uint8, device="cuda")
+    assert lop.global_reduce(x, "sumsq").item() == 255.0 ** 2 * 16 * 4096 * 4096
+    assert lop.global_reduce(x, "sum").item() == 255.0 * 16 * 4096 * 4096
