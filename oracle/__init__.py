@@ -24,6 +24,10 @@ Parity status (details in DESIGN.md "Oracle pins"):
                                         correlate, hand-computed 3x3 examples,
                                         step-edge preservation, constant image,
                                         convexity, flip symmetry
+  pyr_reduce / pyr_expand       pinned: scipy correlate + decimation; np.pad +
+                                        zero insertion (tests/test_oracle_pyramid_pins.py)
+  multires_bilateral            pinned: perfect reconstruction, constant image,
+                                        one level == bilateral_f32
 """
 from __future__ import annotations
 
@@ -93,6 +97,9 @@ def _load():
                                              vp, vp, i32, i32, i64, i64, vp, vp]
             lib.oracle_local_u8.argtypes = [i32, pa, vp, i64, i64, pa, vp, vp, vp, vp, vp, vp,
                                             vp, vp, i32, i32, i64, i64, vp, vp]
+            lib.oracle_pyr_reduce_f64.argtypes = [vp, i64, i64, i32, dbl, vp]
+            lib.oracle_pyr_expand_f64.argtypes = [vp, i64, i64, i64, i64, i32, dbl, vp]
+            lib.oracle_bilateral_f64.argtypes = [vp, i64, i64, i32, i32, dbl, dbl, i32, dbl, vp]
             _lib = lib
     return _lib
 
@@ -405,3 +412,81 @@ def local(imgs, masks, op="sum", fn="product", modes="clamp", cvals=0.0, offsets
         _ptr(oys), _ptr(mds), _ptr(cv), _ptr(pa), _ptr(pb), LOCAL_OPS[op], TAP_FNS[fn], y0, y1,
         _ptr(out), _ptr(valid))
     return out, valid.astype(bool)
+
+
+# ------------------------------------------------ multiresolution filter (N4) ----
+# PAPER.md L309-L314 ("a multiresolution filter (see [7]) is applied to an
+# image: the image gets upsampled multiple times", Mirror at the borders);
+# reading c28: a Laplacian pyramid (REDUCE / EXPAND with the 5x5 binomial)
+# whose band-pass levels are bilateral-filtered, then reconstructed.
+
+PYRAMID_MODES = ("clamp", "repeat", "mirror", "constant")
+
+
+def pyr_size(n: int) -> int:
+    """Size of the next coarser level: ceil(n / 2)."""
+    return (int(n) + 1) // 2
+
+
+def pyr_reduce(img, mode="mirror", cval=0.0):
+    """REDUCE (lop_oracle.c oracle_pyr_reduce_f64): the 5x5 binomial at every
+    second pixel; double result of size ceil(H/2) x ceil(W/2)."""
+    assert _mode(mode) != UNDEFINED
+    g = np.ascontiguousarray(img, np.float64)
+    H, W = g.shape
+    out = np.empty((pyr_size(H), pyr_size(W)), np.float64)
+    _load().oracle_pyr_reduce_f64(_ptr(g), W, H, _mode(mode), float(cval), _ptr(out))
+    return out
+
+
+def pyr_expand(coarse, shape, mode="mirror", cval=0.0):
+    """EXPAND (oracle_pyr_expand_f64) of a coarse level to ``shape`` = (H, W),
+    ceil(H/2) x ceil(W/2) = coarse.shape."""
+    assert _mode(mode) != UNDEFINED
+    g = np.ascontiguousarray(coarse, np.float64)
+    H, W = shape
+    assert g.shape == (pyr_size(H), pyr_size(W))
+    out = np.empty((H, W), np.float64)
+    _load().oracle_pyr_expand_f64(_ptr(g), g.shape[1], g.shape[0], W, H, _mode(mode), float(cval),
+                                  _ptr(out))
+    return out
+
+
+def bilateral_f64(img, sigma_d, sigma_r, mode, cval=0.0, size=None):
+    """Alg. 1 on a double image (oracle_bilateral_f64), window 4*sigma_d+1."""
+    g = np.ascontiguousarray(img, np.float64)
+    H, W = g.shape
+    if size is None:
+        size = 2 * int(round(2 * sigma_d)) + 1
+    out = np.empty((H, W), np.float64)
+    _load().oracle_bilateral_f64(_ptr(g), W, H, size, size, float(sigma_d), float(sigma_r),
+                                 _mode(mode), float(cval), _ptr(out))
+    return out
+
+
+def multires_bilateral(img, levels, sigma_d, sigma_r, mode="mirror", cval=0.0):
+    """Multiresolution bilateral filter (N4, reading c28), step by step:
+      G_0 = I;  G_{l+1} = REDUCE(G_l)                       l = 0 .. L-2
+      B_l = G_l - EXPAND(G_{l+1}) (band-pass), B_{L-1} = G_{L-1} (low-pass)
+      F_l = bilateral(B_l; sigma_d, sigma_r[l]) if sigma_r[l] > 0 else B_l
+      R_{L-1} = F_{L-1};  R_l = F_l + EXPAND(R_{l+1});  result R_0.
+    Every level uses ``mode``; in CONSTANT mode the Gaussian levels (REDUCE /
+    EXPAND reads and the low-pass level) read ``cval``, the band-pass levels 0
+    (the band-pass of a constant image).  sigma_r: one value per level."""
+    L = int(levels)
+    assert L >= 1 and len(sigma_r) == L
+    G = [np.asarray(img, np.float64)]
+    for _ in range(L - 1):
+        G.append(pyr_reduce(G[-1], mode, cval))
+    B = [G[l] - pyr_expand(G[l + 1], G[l].shape, mode, cval) for l in range(L - 1)] + [G[-1]]
+    F = []
+    for l in range(L):
+        if sigma_r[l] > 0:
+            F.append(bilateral_f64(B[l], sigma_d, sigma_r[l], mode,
+                                   cval if l == L - 1 else 0.0))
+        else:
+            F.append(B[l])
+    R = F[-1]
+    for l in range(L - 2, -1, -1):
+        R = F[l] + pyr_expand(R, F[l].shape, mode, cval)
+    return R

@@ -534,3 +534,97 @@ void oracle_local_u8(int K, const uint8_t *const *imgs, const int64_t *strides, 
                                  pa, pb, op, fn, x, y, &valid[o]);
         }
 }
+
+/* ------------------------------------------------------------------ */
+/* Multiresolution filter: PAPER.md L309-L314 -- "a */
+/* multiresolution filter (see [7]) ... the image gets upsampled       */
+/* multiple times", with Mirror at the borders -- read as a Laplacian  */
+/* pyramid whose band-pass levels are filtered by the bilateral filter */
+/* (reading c28).  Images here are double (the pyramid's intermediate  */
+/* levels are not f32 data in the oracle).                             */
+/*   w = [1 4 6 4 1] / 16 (the binomial of the paper's Gaussian)       */
+/*   REDUCE: G'(x, y) = sum_{j=-2..2} sum_{i=-2..2} w(i) w(j)          */
+/*                      Read_G(2x + i, 2y + j),                        */
+/*           G' of size ceil(W/2) x ceil(H/2)                          */
+/*   EXPAND: E(x, y) = sum_{j=-2..2} sum_{i=-2..2} 4 w(i) w(j)         */
+/*                     Read_G'((x - i) / 2, (y - j) / 2)               */
+/*           over the taps with x - i and y - j even; Read applies the */
+/*           boundary mode at the level being read.                    */
+/* Modes: Clamp / Repeat / Mirror / Constant (Undefined has no pyramid */
+/* meaning: its reads would leave every border output unspecified).   */
+/* ------------------------------------------------------------------ */
+
+static double read_f64(const double *img, int64_t W, int64_t H, int64_t x, int64_t y, int mode,
+                       double cval)
+{
+    if (x >= 0 && x < W && y >= 0 && y < H)
+        return img[y * W + x];
+    if (mode == OR_CONSTANT)
+        return cval;
+    return img[oracle_map_index(y, H, mode) * W + oracle_map_index(x, W, mode)];
+}
+
+static const double PYR_W[5] = {1.0 / 16, 4.0 / 16, 6.0 / 16, 4.0 / 16, 1.0 / 16};
+
+void oracle_pyr_reduce_f64(const double *g, int64_t W, int64_t H, int mode, double cval,
+                           double *out)
+{
+    const int64_t Wc = (W + 1) / 2, Hc = (H + 1) / 2;
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t y = 0; y < Hc; ++y)
+        for (int64_t x = 0; x < Wc; ++x) {
+            double acc = 0.0;
+            for (int j = -2; j <= 2; ++j)
+                for (int i = -2; i <= 2; ++i)
+                    acc += PYR_W[i + 2] * PYR_W[j + 2] *
+                           read_f64(g, W, H, 2 * x + i, 2 * y + j, mode, cval);
+            out[y * Wc + x] = acc;
+        }
+}
+
+/* floor((v) / 2) for the even v the caller passes (exact for negatives) */
+static int64_t half_even(int64_t v) { return v >= 0 ? v / 2 : -((-v) / 2); }
+
+void oracle_pyr_expand_f64(const double *gc, int64_t Wc, int64_t Hc, int64_t W, int64_t H,
+                           int mode, double cval, double *out)
+{
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t y = 0; y < H; ++y)
+        for (int64_t x = 0; x < W; ++x) {
+            double acc = 0.0;
+            for (int j = -2; j <= 2; ++j) {
+                if ((y - j) % 2 != 0) continue;
+                for (int i = -2; i <= 2; ++i) {
+                    if ((x - i) % 2 != 0) continue;
+                    acc += 4.0 * PYR_W[i + 2] * PYR_W[j + 2] *
+                           read_f64(gc, Wc, Hc, half_even(x - i), half_even(y - j), mode, cval);
+                }
+            }
+            out[y * W + x] = acc;
+        }
+}
+
+/* Bilateral filter of a double image: Alg. 1 exactly as bilateral_px     */
+/* (closeness from Eq. (1), similarity Eq. (2)), for the pyramid levels.  */
+void oracle_bilateral_f64(const double *img, int64_t W, int64_t H, int mw, int mh,
+                          double sigma_d, double sigma_r, int mode, double cval, double *out)
+{
+    const int m = mw / 2, n = mh / 2;
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int64_t y = 0; y < H; ++y)
+        for (int64_t x = 0; x < W; ++x) {
+            const double center = img[y * W + x];
+            double p = 0.0, k = 0.0;
+            for (int yf = -n; yf <= n; ++yf)
+                for (int xf = -m; xf <= m; ++xf) {
+                    const double v = read_f64(img, W, H, x + xf, y + yf, mode, cval);
+                    const double dist = sqrt((double)(xf * xf + yf * yf));
+                    const double c = exp(-0.5 * (dist / sigma_d) * (dist / sigma_d));
+                    const double dp = fabs(v - center);
+                    const double s = exp(-0.5 * (dp / sigma_r) * (dp / sigma_r));
+                    k = k + c * s;
+                    p = p + c * s * v;
+                }
+            out[y * W + x] = p / k;
+        }
+}
