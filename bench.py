@@ -646,6 +646,21 @@ def extras(lop, synthetic, dev, stream, peaks):
     stream.wait_stream(s2)
     ms = timed(lambda: g.replay(), 10, False)
     out["config1_bilateral_256_3x3_graph_Mpx_s"] = round(256 * 256 * 100 / ms / 1e3, 1)
+    # multiresolution filter (N4, reading c28): 4 levels, 13 x 13 window, Mirror; the
+    # bilateral levels dominate (SFU-bound), so report the time and the share of the
+    # level-0 bilateral alone
+    levels, srs = 4, [0.05, 0.08, 0.12, 0.0]
+    ws = torch.empty(lop.multires_workspace_bytes(tuple(img.shape), levels), dtype=torch.uint8,
+                     device=dev)
+    ms_mr = timed(lambda: lop.multires_bilateral(img, levels, 3.0, srs, "mirror", out=res,
+                                                 workspace=ws, stream=stream), 10, False)
+    ms_b0 = timed(lambda: lop.bilateral(img, 3.0, 0.05, "mirror", size=13, out=res,
+                                        stream=stream), 10, False)
+    out["multires_bilateral_4096_4levels_13x13"] = {
+        "ms": round(ms_mr, 4), "Mpx_s": round(H * Wd / ms_mr / 1e3, 1),
+        "level0_bilateral_ms": round(ms_b0, 4),
+        "level0_share": round(ms_b0 / ms_mr, 3),
+        "launches": 3 * (levels - 1) + sum(1 for v in srs if v > 0)}
     return out
 
 
@@ -731,6 +746,16 @@ def conv_extras(lop, synthetic, dev, stream, hbm, img, timed):
                                                           stream=s), 4),
         ("global_max_u8", lambda k, s: lop.global_reduce(u_in[k], "max", out=gres, work=gwork,
                                                          stream=s), 1)]
+    # Laplacian-pyramid steps of the multiresolution filter (N4, reading c28):
+    # REDUCE 4096^2 -> 2048^2 (4 B read per fine pixel + 4 B per coarse = 5 B / fine px),
+    # band-pass EXPAND with the fine addend (coarse 1 B + addend 4 B + out 4 B = 9 B / fine px)
+    red = [torch.empty(2048, 2048, device=dev) for _ in range(sets)]
+    cases += [
+        ("pyramid_reduce_f32", lambda k, s: lop.pyramid_reduce(f_in[k], "mirror", out=red[k],
+                                                               stream=s), 5),
+        ("pyramid_expand_bandpass_f32",
+         lambda k, s: lop.pyramid_expand(red[k], img.shape, "mirror", addend=f_in[k], sign=-1.0,
+                                         out=f_out[k], stream=s), 9)]
     res = {}
     H, W = img.shape
     for name, fn, bpp in cases:

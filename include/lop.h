@@ -302,6 +302,53 @@ lop_status lop_local_execute_point(const lop_iteration_space *is, const lop_acce
                                    int32_t tap_fn, const double *scale, const double *offset,
                                    void *cuda_stream);
 
+/* ---- Multiresolution filter ----
+ * "a multiresolution filter (see [7]) is applied to an
+ * image: the image gets upsampled multiple times", Mirror at the borders
+ * avoiding artifacts.  Reading c28: a Laplacian pyramid with the
+ * binomial w = [1 4 6 4 1] / 16 whose levels are bilateral-filtered.
+ * Pyramid levels are whole F32 images (no ROI, no band views), batch allowed
+ * (all frames at once); modes CLAMP / REPEAT / MIRROR / CONSTANT (UNDEFINED
+ * is rejected: every border output of a pyramid level would be unspecified).
+ *
+ * REDUCE: is->image (the coarse level, ceil(W/2) x ceil(H/2), same batch)
+ *   G'(x, y) = sum_{i,j=-2..2} w(i) w(j) Read(2x + i, 2y + j)
+ * of the accessor's image (W x H) with its BoundaryCondition (mode,
+ * constant; window 5 x 5; offset 0).  One kernel launch. */
+lop_status lop_pyramid_reduce_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                      void *cuda_stream);
+/* EXPAND: is->image (the fine level, W x H) receives
+ *   out(x, y) = addend(x, y) + sign * E(x, y),
+ *   E(x, y) = sum 4 w(i) w(j) Read((x - i) / 2, (y - j) / 2) over the i, j in
+ *             -2..2 with x - i and y - j even,
+ * Read: the accessor's image, the coarse level (ceil(W/2) x ceil(H/2)), with
+ * its BoundaryCondition (window 5 x 5, offset 0).  addend: NULL (out = sign
+ * E) or an F32 image of the output's size; it may be the output itself (in
+ * place: each output reads only its own addend pixel) but must not partially
+ * overlap it.  sign -1 gives a band-pass level G - EXPAND(G'), +1 the
+ * reconstruction step.  One kernel launch. */
+lop_status lop_pyramid_expand_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                      const lop_image *addend, float sign, void *cuda_stream);
+/* The whole filter, reading c28:
+ *   G_0 = input, G_{l+1} = REDUCE(G_l)            (l < levels - 1)
+ *   B_l = G_l - EXPAND(G_{l+1}), B_{levels-1} = G_{levels-1}
+ *   F_l = bilateral(B_l; sigma_d, sigma_r[l]) (window = the BoundaryCondition's
+ *         size, closeness Eq. 1), or F_l = B_l when sigma_r[l] <= 0
+ *   R_{levels-1} = F_{levels-1}, R_l = F_l + EXPAND(R_{l+1}); out = R_0.
+ * in: the F32 input through its BoundaryCondition (mode for every level; in
+ * CONSTANT mode the Gaussian levels read the constant and the band-pass
+ * levels 0); is->image: the F32 output, same size and batch, whole image.
+ * levels: 1 .. 16 (1 = the bilateral filter itself); sigma_r: `levels` host
+ * floats.  d_workspace: device memory of at least
+ * lop_multires_workspace_bytes() bytes (16-B aligned), owned by the caller.
+ * At most 4 * levels kernel launches on cuda_stream, nothing synchronised. */
+lop_status lop_multires_workspace_bytes(int32_t width, int32_t height, int32_t batch,
+                                        int32_t levels, int64_t *bytes);
+lop_status lop_multires_bilateral_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                          int32_t levels, float sigma_d, const float *sigma_r,
+                                          void *d_workspace, int64_t workspace_bytes,
+                                          void *cuda_stream);
+
 /* Algorithm 2, the kernel-configuration heuristic, as a
  * pure host function (no CUDA call; the library feeds it cudaOccupancy*
  * figures).  cand[i] describes configuration i: threads per CTA, its tiling

@@ -323,6 +323,73 @@ def local(inputs, masks, op="sum", fn="product", modes="clamp", constants=0.0, o
     return out
 
 
+# ------------------------------------------------ multiresolution filter (N4) ----
+
+def _pyr_half(n: int) -> int:
+    return (int(n) + 1) // 2
+
+
+def pyramid_reduce(x: torch.Tensor, mode="mirror", constant=0.0, out=None,
+                   stream=None) -> torch.Tensor:
+    """REDUCE (lop_pyramid_reduce_execute; reading c28): the 5x5 binomial at
+    every second pixel of a float32 (H, W) / (B, H, W) image -> ceil(H/2) x
+    ceil(W/2)."""
+    if out is None:
+        out = torch.empty(x.shape[:-2] + (_pyr_half(x.shape[-2]), _pyr_half(x.shape[-1])),
+                          dtype=x.dtype, device=x.device)
+    return _execute("pyr_reduce", x, out, mode, constant, (5, 5), None, (0, 0), stream,
+                    (0, 0, 0, 0), lambda is_, acc, s: lib.lop_pyramid_reduce_execute(is_, acc, s))
+
+
+def pyramid_expand(coarse: torch.Tensor, shape, mode="mirror", constant=0.0, addend=None,
+                   sign=1.0, out=None, stream=None) -> torch.Tensor:
+    """EXPAND (lop_pyramid_expand_execute; reading c28) of a coarse level to
+    ``shape`` = (H, W): out = addend + sign * EXPAND(coarse) (addend None ->
+    sign * EXPAND); ``out`` may be ``addend`` (in place)."""
+    H, W = (int(v) for v in shape)
+    if out is None:
+        out = torch.empty(coarse.shape[:-2] + (H, W), dtype=coarse.dtype, device=coarse.device)
+    add = ctypes.byref(image_view(addend)) if addend is not None else None
+    return _execute("pyr_expand", coarse, out, mode, constant, (5, 5), None, (0, 0), stream,
+                    (0, 0, 0, 0), lambda is_, acc, s: lib.lop_pyramid_expand_execute(
+                        is_, acc, add, float(sign), s))
+
+
+def multires_workspace_bytes(shape, levels: int) -> int:
+    b = 1 if len(shape) == 2 else int(shape[0])
+    n = ctypes.c_int64(0)
+    _check(lib.lop_multires_workspace_bytes(int(shape[-1]), int(shape[-2]), b, int(levels),
+                                            ctypes.byref(n)))
+    return n.value
+
+
+def multires_bilateral(x: torch.Tensor, levels: int, sigma_d: float, sigma_r, mode="mirror",
+                       constant=0.0, size=None, out=None, workspace=None,
+                       stream=None) -> torch.Tensor:
+    """Multiresolution bilateral filter (lop_multires_bilateral_execute; PAPER.md
+    L309-L314, reading c28): Laplacian pyramid of ``levels`` levels, level l
+    bilateral-filtered with (sigma_d, sigma_r[l]) (sigma_r[l] <= 0: unfiltered),
+    reconstructed.  ``workspace``: a uint8 CUDA tensor of at least
+    multires_workspace_bytes(x.shape, levels) bytes (allocated if None)."""
+    levels = int(levels)
+    sr = [float(v) for v in (sigma_r if np.ndim(sigma_r) else [sigma_r] * levels)]
+    if len(sr) != levels:
+        raise ValueError("one sigma_r per level")
+    if size is None:
+        size = _default_window(sigma_d)
+    size_xy = (size, size) if isinstance(size, int) else tuple(size)
+    need = multires_workspace_bytes(tuple(x.shape), levels)
+    if workspace is None:
+        workspace = torch.empty(max(need, 1), dtype=torch.uint8, device=x.device)
+    if out is None:
+        out = torch.empty_like(x)
+    srs = (ctypes.c_float * levels)(*sr)
+    return _execute("multires", x, out, mode, constant, size_xy, None, (0, 0), stream,
+                    (0, 0, 0, 0), lambda is_, acc, s: lib.lop_multires_bilateral_execute(
+                        is_, acc, levels, float(sigma_d), srs, workspace.data_ptr(),
+                        workspace.numel(), s))
+
+
 def alg2_select(candidates, width, height, rx, ry, simd_width=32):
     """Algorithm 2 over candidate configurations, each a
     dict(block_x, block_y, out_x=1, out_y=1, valid=True, occupancy);

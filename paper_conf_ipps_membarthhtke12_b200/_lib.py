@@ -93,6 +93,15 @@ SIGNATURES = {
                                         ctypes.POINTER(ctypes.POINTER(lop_accessor)),
                                         ctypes.POINTER(ctypes.POINTER(lop_mask)), c_i32, c_i32,
                                         c_i32, c_vp, c_vp, c_vp]),
+    "lop_pyramid_reduce_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
+                                           ctypes.POINTER(lop_accessor), c_vp]),
+    "lop_pyramid_expand_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
+                                           ctypes.POINTER(lop_accessor), ctypes.POINTER(lop_image),
+                                           c_flt, c_vp]),
+    "lop_multires_workspace_bytes": (c_i32, [c_i32, c_i32, c_i32, c_i32, ctypes.POINTER(c_i64)]),
+    "lop_multires_bilateral_execute": (c_i32, [ctypes.POINTER(lop_iteration_space),
+                                               ctypes.POINTER(lop_accessor), c_i32, c_flt, c_vp,
+                                               c_vp, c_i64, c_vp]),
     "lop_alg2_select": (c_i32, [c_vp, c_i32, c_i32, c_i32, c_i32, c_i32, c_i32,
                                 ctypes.POINTER(c_i64)]),
     "lop_mask_closeness": (c_i32, [c_flt, c_i32, c_i32, c_vp]),

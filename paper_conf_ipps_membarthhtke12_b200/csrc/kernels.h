@@ -34,4 +34,8 @@ cudaError_t launch_conv_chain(const ConvChain &p, cudaStream_t stream);
 // staging) or generic; the CTA shape from Algorithm 2 (select.cpp).
 cudaError_t launch_local(const LocalParams &p, bool tiled, cudaStream_t stream);
 
+// Laplacian-pyramid REDUCE and EXPAND (+ addend) (pyramid.cu).
+cudaError_t launch_pyr_reduce(const PyrParams &p, cudaStream_t stream);
+cudaError_t launch_pyr_expand(const PyrParams &p, cudaStream_t stream);
+
 }  // namespace lop

@@ -1014,3 +1014,276 @@ lop_status lop_local_execute_point(const lop_iteration_space *is, const lop_acce
 }
 
 }  // extern "C"
+
+// ------------------------------------------ multiresolution filter (N4, c28)
+namespace {
+
+int pyr_half(int n) { return (n + 1) / 2; }
+
+// Whole, unbanded F32 image (pyramid levels).
+lop_status pyr_check_level(const lop_image &im, const char *name)
+{
+    lop_status st = check_image(im, name);
+    if (st) return st;
+    if (im.dtype != LOP_F32) return fail(LOP_ERR_INVALID, "%s: pyramid levels are F32 images", name);
+    if (im.halo_top || im.halo_bottom || im.global_y0 ||
+        (im.global_height && im.global_height != im.height))
+        return fail(LOP_ERR_INVALID, "%s: pyramid levels are whole images (no band views)", name);
+    return LOP_OK;
+}
+
+// Common validation of REDUCE / EXPAND; reduce: the output is the coarse level.
+lop_status pyr_prepare(const lop_iteration_space *is, const lop_accessor *in, bool reduce,
+                       lop::PyrParams &p)
+{
+    if (!is) return fail(LOP_ERR_INVALID, "iteration space is NULL");
+    if (!in || !in->bc) return fail(LOP_ERR_INVALID, "accessor / boundary condition is NULL");
+    const lop_boundary_condition &bc = *in->bc;
+    lop_status st = pyr_check_level(bc.image, "input");
+    if (st) return st;
+    st = pyr_check_level(is->image, "output");
+    if (st) return st;
+    const lop_image &ii = bc.image, &oi = is->image;
+    if (bc.mode < LOP_CLAMP || bc.mode > LOP_CONSTANT)
+        return fail(LOP_ERR_INVALID, "pyramid boundary mode %d: CLAMP, REPEAT, MIRROR or CONSTANT", bc.mode);
+    if (bc.size_x != 5 || bc.size_y != 5)
+        return fail(LOP_ERR_INVALID, "pyramid window must be 5 x 5 (the binomial), got %d x %d", bc.size_x,
+                    bc.size_y);
+    if (in->offset_x || in->offset_y) return fail(LOP_ERR_INVALID, "pyramid accessors take no offset");
+    if (!std::isfinite(bc.constant)) return fail(LOP_ERR_INVALID, "constant is not finite");
+    if (is->x0 || is->y0 || (is->width && is->width != oi.width) || (is->height && is->height != oi.height))
+        return fail(LOP_ERR_INVALID, "pyramid levels are computed whole (no ROI)");
+    if (ii.batch != oi.batch) return fail(LOP_ERR_INVALID, "input/output batch differ");
+    const lop_image &fine = reduce ? ii : oi, &coarse = reduce ? oi : ii;
+    if (coarse.width != pyr_half(fine.width) || coarse.height != pyr_half(fine.height))
+        return fail(LOP_ERR_INVALID, "coarse level %d x %d is not ceil(%d/2) x ceil(%d/2)", coarse.width,
+                    coarse.height, fine.width, fine.height);
+    st = check_disjoint(ii, oi);
+    if (st) return st;
+    std::memset(&p, 0, sizeof p);
+    p.in = make_geom(ii);
+    p.out.data = static_cast<char *>(oi.data);
+    p.out.stride = oi.stride_bytes;
+    p.out.bstride = oi.batch > 1 ? oi.batch_stride_bytes : 0;
+    p.out.W = oi.width;
+    p.out.H = oi.height;
+    p.mode = bc.mode;
+    p.cval = (float)bc.constant;
+    p.batch = oi.batch;
+    p.sign = 1.0f;
+    return LOP_OK;
+}
+
+struct PyrLevel {
+    int32_t w, h;
+    int64_t stride, frame, bytes;     // row pitch, frame bytes, all frames (256-B rounded)
+};
+
+PyrLevel pyr_level(int32_t w, int32_t h, int32_t batch)
+{
+    PyrLevel L;
+    L.w = w;
+    L.h = h;
+    L.stride = ((int64_t)w * 4 + 15) & ~(int64_t)15;
+    L.frame = L.stride * h;
+    L.bytes = (L.frame * batch + 255) & ~(int64_t)255;
+    return L;
+}
+
+lop_image pyr_view(void *data, const PyrLevel &L, int32_t batch)
+{
+    lop_image im;
+    std::memset(&im, 0, sizeof im);
+    im.data = data;
+    im.width = L.w;
+    im.height = L.h;
+    im.stride_bytes = L.stride;
+    im.dtype = LOP_F32;
+    im.batch = batch;
+    im.batch_stride_bytes = L.frame;
+    return im;
+}
+
+// Workspace: the Gaussian levels 1 .. L-1, then T0 (band-pass level 0, later
+// the filtered levels 1 .. L-1).
+int64_t multires_layout(int32_t w, int32_t h, int32_t batch, int32_t levels, PyrLevel *lv,
+                        int64_t *goff, int64_t *t0off, int64_t *foff)
+{
+    lv[0] = pyr_level(w, h, batch);
+    for (int l = 1; l < levels; ++l) lv[l] = pyr_level(pyr_half(lv[l - 1].w), pyr_half(lv[l - 1].h), batch);
+    int64_t off = 0;
+    for (int l = 1; l < levels; ++l) { goff[l] = off; off += lv[l].bytes; }
+    *t0off = off;
+    int64_t fsum = 0;
+    for (int l = 1; l < levels; ++l) { foff[l] = off + fsum; fsum += lv[l].bytes; }
+    return off + std::max(levels > 1 ? lv[0].bytes : (int64_t)0, fsum);
+}
+
+constexpr int kMaxLevels = 16;
+
+}  // namespace
+
+extern "C" {
+
+lop_status lop_pyramid_reduce_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                      void *cuda_stream)
+{
+    lop::PyrParams p;
+    lop_status st = pyr_prepare(is, in, true, p);
+    if (st) return st;
+    return launched(lop::launch_pyr_reduce(p, static_cast<cudaStream_t>(cuda_stream)), "pyramid reduce launch");
+}
+
+lop_status lop_pyramid_expand_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                      const lop_image *addend, float sign, void *cuda_stream)
+{
+    lop::PyrParams p;
+    lop_status st = pyr_prepare(is, in, false, p);
+    if (st) return st;
+    if (!std::isfinite(sign)) return fail(LOP_ERR_INVALID, "sign is not finite");
+    p.sign = sign;
+    if (addend) {
+        st = pyr_check_level(*addend, "addend");
+        if (st) return st;
+        const lop_image &oi = is->image;
+        if (addend->width != oi.width || addend->height != oi.height || addend->batch != oi.batch)
+            return fail(LOP_ERR_INVALID, "addend %d x %d x %d differs from the output %d x %d x %d",
+                        addend->width, addend->height, addend->batch, oi.width, oi.height, oi.batch);
+        const bool same = addend->data == oi.data && addend->stride_bytes == oi.stride_bytes &&
+                          (oi.batch == 1 || addend->batch_stride_bytes == oi.batch_stride_bytes);
+        if (!same) {
+            st = check_disjoint(*addend, oi);
+            if (st) return fail(LOP_ERR_INVALID, "addend must be the output itself or disjoint from it");
+        }
+        st = check_disjoint(in->bc->image, *addend);
+        if (st) return st;
+        p.add = static_cast<const char *>(addend->data);
+        p.add_stride = addend->stride_bytes;
+        p.add_bstride = addend->batch > 1 ? addend->batch_stride_bytes : 0;
+    }
+    return launched(lop::launch_pyr_expand(p, static_cast<cudaStream_t>(cuda_stream)), "pyramid expand launch");
+}
+
+lop_status lop_multires_workspace_bytes(int32_t width, int32_t height, int32_t batch, int32_t levels,
+                                        int64_t *bytes)
+{
+    if (!bytes) return fail(LOP_ERR_INVALID, "bytes is NULL");
+    if (width <= 0 || height <= 0 || batch <= 0) return fail(LOP_ERR_INVALID, "empty image");
+    if (levels < 1 || levels > kMaxLevels) return fail(LOP_ERR_INVALID, "levels %d outside 1..%d", levels, kMaxLevels);
+    PyrLevel lv[kMaxLevels];
+    int64_t goff[kMaxLevels], foff[kMaxLevels], t0;
+    *bytes = multires_layout(width, height, batch, levels, lv, goff, &t0, foff);
+    return LOP_OK;
+}
+
+lop_status lop_multires_bilateral_execute(const lop_iteration_space *is, const lop_accessor *in,
+                                          int32_t levels, float sigma_d, const float *sigma_r,
+                                          void *d_workspace, int64_t workspace_bytes,
+                                          void *cuda_stream)
+{
+    if (!is || !in || !in->bc) return fail(LOP_ERR_INVALID, "iteration space / accessor is NULL");
+    if (levels < 1 || levels > kMaxLevels) return fail(LOP_ERR_INVALID, "levels %d outside 1..%d", levels, kMaxLevels);
+    if (!sigma_r) return fail(LOP_ERR_INVALID, "sigma_r is NULL");
+    if (!(sigma_d > 0.0f) || !std::isfinite(sigma_d)) return fail(LOP_ERR_INVALID, "sigma_d must be > 0");
+    for (int l = 0; l < levels; ++l)
+        if (!std::isfinite(sigma_r[l])) return fail(LOP_ERR_INVALID, "sigma_r[%d] is not finite", l);
+    const lop_boundary_condition &bc = *in->bc;
+    const lop_image &ii = bc.image, &oi = is->image;
+    lop_status st = pyr_check_level(ii, "input");
+    if (st) return st;
+    st = pyr_check_level(oi, "output");
+    if (st) return st;
+    if (ii.width != oi.width || ii.height != oi.height || ii.batch != oi.batch)
+        return fail(LOP_ERR_INVALID, "input and output differ in size or batch");
+    if (bc.mode < LOP_CLAMP || bc.mode > LOP_CONSTANT)
+        return fail(LOP_ERR_INVALID, "multiresolution mode %d: CLAMP, REPEAT, MIRROR or CONSTANT", bc.mode);
+    if (in->offset_x || in->offset_y) return fail(LOP_ERR_INVALID, "the multiresolution accessor takes no offset");
+    if (is->x0 || is->y0 || (is->width && is->width != oi.width) || (is->height && is->height != oi.height))
+        return fail(LOP_ERR_INVALID, "the multiresolution filter is computed whole (no ROI)");
+    st = check_disjoint(ii, oi);
+    if (st) return st;
+    PyrLevel lv[kMaxLevels];
+    int64_t goff[kMaxLevels], foff[kMaxLevels], t0off;
+    const int64_t need = multires_layout(oi.width, oi.height, oi.batch, levels, lv, goff, &t0off, foff);
+    if (need > 0 && (!d_workspace || workspace_bytes < need))
+        return fail(LOP_ERR_INVALID, "workspace of %lld bytes needed (%lld given)", (long long)need,
+                    (long long)workspace_bytes);
+    if (reinterpret_cast<uintptr_t>(d_workspace) & 15) return fail(LOP_ERR_INVALID, "workspace not 16-B aligned");
+    const cudaStream_t stream = static_cast<cudaStream_t>(cuda_stream);
+    char *ws = static_cast<char *>(d_workspace);
+    const int32_t B = oi.batch;
+    lop_image G[kMaxLevels], F[kMaxLevels];
+    G[0] = ii;
+    for (int l = 1; l < levels; ++l) G[l] = pyr_view(ws + goff[l], lv[l], B);
+    const lop_image T0 = pyr_view(ws + t0off, lv[0], B);
+
+    auto bcond = [&](const lop_image &im, int sx, int sy, double cval) {
+        lop_boundary_condition c;
+        c.image = im;
+        c.mode = bc.mode;
+        c.size_x = sx;
+        c.size_y = sy;
+        c.constant = cval;
+        return c;
+    };
+    auto space = [](const lop_image &im) {
+        lop_iteration_space s;
+        std::memset(&s, 0, sizeof s);
+        s.image = im;
+        return s;
+    };
+    // 1. Gaussian levels
+    for (int l = 0; l + 1 < levels; ++l) {
+        const lop_boundary_condition c = bcond(G[l], 5, 5, bc.constant);
+        const lop_accessor a{&c, 0, 0};
+        const lop_iteration_space s = space(G[l + 1]);
+        st = lop_pyramid_reduce_execute(&s, &a, cuda_stream);
+        if (st) return st;
+    }
+    // 2. band-pass levels: B_0 -> T0, B_l (l >= 1) in place of G_l
+    lop_image Bv[kMaxLevels];
+    for (int l = 0; l + 1 < levels; ++l) {
+        Bv[l] = l == 0 ? T0 : G[l];
+        const lop_boundary_condition c = bcond(G[l + 1], 5, 5, bc.constant);
+        const lop_accessor a{&c, 0, 0};
+        const lop_iteration_space s = space(Bv[l]);
+        st = lop_pyramid_expand_execute(&s, &a, &G[l], -1.0f, cuda_stream);
+        if (st) return st;
+    }
+    Bv[levels - 1] = G[levels - 1];
+    // 3. filtered levels: F_0 -> out; F_l (l >= 1) -> T0's sub-buffers, after F_0
+    for (int l = 0; l < levels; ++l) {
+        const double cval = l == levels - 1 ? bc.constant : 0.0;   // band-pass levels read 0
+        lop_image dst = l == 0 ? oi : pyr_view(ws + foff[l], lv[l], B);
+        if (sigma_r[l] > 0.0f) {
+            const lop_boundary_condition c = bcond(Bv[l], bc.size_x, bc.size_y, cval);
+            const lop_accessor a{&c, 0, 0};
+            const lop_iteration_space s = space(dst);
+            st = lop_bilateral_execute(&s, &a, nullptr, sigma_d, sigma_r[l], cuda_stream);
+            if (st) return fail(st, "level %d bilateral: %s", l, lop_last_error());
+            F[l] = dst;
+        } else if (l == 0) {                                        // unfiltered level 0: copy to out
+            for (int b = 0; b < B; ++b) {
+                const cudaError_t e = cudaMemcpy2DAsync(
+                    static_cast<char *>(oi.data) + (int64_t)b * (B > 1 ? oi.batch_stride_bytes : 0), oi.stride_bytes,
+                    static_cast<const char *>(Bv[0].data) + (int64_t)b * (B > 1 ? Bv[0].batch_stride_bytes : 0),
+                    Bv[0].stride_bytes, (size_t)oi.width * 4, oi.height, cudaMemcpyDeviceToDevice, stream);
+                if (e != cudaSuccess) return cuda_fail(e, "level 0 copy");
+            }
+            F[0] = oi;
+        } else {
+            F[l] = Bv[l];
+        }
+    }
+    // 4. reconstruction, coarse to fine, in place on F_l (F_0 = out)
+    for (int l = levels - 2; l >= 0; --l) {
+        const lop_boundary_condition c = bcond(F[l + 1], 5, 5, bc.constant);
+        const lop_accessor a{&c, 0, 0};
+        const lop_iteration_space s = space(F[l]);
+        st = lop_pyramid_expand_execute(&s, &a, &F[l], 1.0f, cuda_stream);
+        if (st) return st;
+    }
+    return LOP_OK;
+}
+
+}  // extern "C"

@@ -207,4 +207,16 @@ struct LocalParams {
     } m;
 };
 
+// Laplacian-pyramid REDUCE / EXPAND (pyramid.cu, reading c28).
+struct PyrParams {
+    Geom in;                     // level read (whole image, no band)
+    OutGeom out;                 // level written
+    const char *add;             // EXPAND: addend image (may alias out) or nullptr
+    int64_t add_stride, add_bstride;
+    float sign;                  // EXPAND: out = add + sign * E
+    int32_t mode;
+    float cval;
+    int32_t batch;
+};
+
 }  // namespace lop

@@ -26,7 +26,9 @@ def test_header_declares_expected_entry_points():
     for s in ("lop_bilateral_execute", "lop_convolve_execute", "lop_mask_closeness",
               "lop_mask_gaussian", "lop_mask_sobel", "lop_last_error", "lop_pipeline_create",
               "lop_convolve_chain_execute", "lop_reduce_execute", "lop_convolve2_execute",
-              "lop_pipeline_bilateral_frames"):
+              "lop_pipeline_bilateral_frames", "lop_local_execute_point",
+              "lop_pyramid_reduce_execute", "lop_pyramid_expand_execute",
+              "lop_multires_workspace_bytes", "lop_multires_bilateral_execute"):
         assert s in syms
 
 
