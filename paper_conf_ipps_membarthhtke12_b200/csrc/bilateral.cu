@@ -660,7 +660,7 @@ __device__ __forceinline__ void pair_issue_row(const Common &c, int b, int iy, i
 // the row (may alias src: each lane reads its chunk before writing it), the
 // first half of its interleaved slot and the second half of the previous
 // row's interleaved slot.
-template <int SW>
+template <int SW, bool PLAIN = true>
 __device__ __forceinline__ void pair_put_row(const Common &c, int iy, int ix0, float alpha,
                                              const float4 *src, float4 *plain, float2 *first,
                                              float2 *second, const int *cm, int lane, bool vec_ok)
@@ -683,7 +683,7 @@ __device__ __forceinline__ void pair_put_row(const Common &c, int iy, int ix0, f
         }
         q.x = __fmul_rn(q.x, alpha); q.y = __fmul_rn(q.y, alpha);
         q.z = __fmul_rn(q.z, alpha); q.w = __fmul_rn(q.w, alpha);
-        plain[k] = q;
+        if (PLAIN) plain[k] = q;
         // interleaved slot, swizzled: float4 i of a slot lives at i ^ ((i >> 3) & 1),
         // so the LDS.128 of 8 lanes reading float4 2L + k (2 x 16 B apart) hit 8
         // distinct 16-B bank groups (no 2-way conflict); columns 4k..4k+3 are
@@ -842,6 +842,239 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
     }
 }
 
+// ------------------------- pair-sharing kernel, partner ring in TMEM
+// Same arithmetic, order and results as bilateral_pair_kernel (bit-identical,
+// tested), with two storage changes that free registers and shared memory so
+// that 16 warps fit on an SM instead of 12 (the kernel is latency-bound:
+// ncu "wait" / MIO stalls with 3 warps per scheduler):
+//  * the per-row partner accumulators D/P[1..R] (8(R+1) floats per thread,
+//    the largest live register set) live in tensor memory: TMEM lane
+//    32 (warp % 4) + lane, 8 columns per ring slot (D[0..3], P[0..3]), the
+//    slot of row s is s mod (R+1), so the per-step ring shift of the
+//    register version becomes an index rotation.  Each row pair loads its two
+//    partner slots (tcgen05.ld 32x32b.x8), folds, and stores them back
+//    (tcgen05.st); the own row's slot is loaded once per step.  One warp of
+//    the CTA allocates 64 columns (<= 8 CTAs per SM: 512 columns).
+//  * no plain (non-interleaved) row ring: the own row dy = 0 and the odd last
+//    row are read as the .x halves of the interleaved row-pair slots.
+#ifndef LOP_PAIR_TM_MAXREG
+#define LOP_PAIR_TM_MAXREG 128
+#endif
+namespace pair {
+constexpr int kTmemCols = 64;                          // per CTA; >= 8 (R + 1) for R <= 7
+constexpr int kTmemMinSmem = 25600;                    // dynamic smem floor: <= 8 CTAs / SM
+template <int R> struct ShapeTM {
+    static constexpr int WARP_FLOATS = Shape<R>::RING2 + 2 * Shape<R>::SW;   // ring2, staging, column map
+};
+}  // namespace pair
+
+__device__ __forceinline__ void tm_ld8(uint32_t ta, float v[8])
+{
+    asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+                 : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]),
+                   "=f"(v[7])
+                 : "r"(ta));
+}
+// wait for the outstanding tcgen05.ld; the values become valid here (the
+// registers are in/out operands so no use is scheduled above the wait)
+__device__ __forceinline__ void tm_wait_ld8(float v[8])
+{
+    asm volatile("tcgen05.wait::ld.sync.aligned;"
+                 : "+f"(v[0]), "+f"(v[1]), "+f"(v[2]), "+f"(v[3]), "+f"(v[4]), "+f"(v[5]), "+f"(v[6]),
+                   "+f"(v[7]));
+}
+__device__ __forceinline__ void tm_wait_ld16(float a[8], float b[8])
+{
+    asm volatile("tcgen05.wait::ld.sync.aligned;"
+                 : "+f"(a[0]), "+f"(a[1]), "+f"(a[2]), "+f"(a[3]), "+f"(a[4]), "+f"(a[5]), "+f"(a[6]),
+                   "+f"(a[7]), "+f"(b[0]), "+f"(b[1]), "+f"(b[2]), "+f"(b[3]), "+f"(b[4]), "+f"(b[5]),
+                   "+f"(b[6]), "+f"(b[7]));
+}
+__device__ __forceinline__ void tm_st8(uint32_t ta, const float v[8])
+{
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};"
+                 ::"r"(ta), "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]),
+                   "f"(v[7]));
+}
+__device__ __forceinline__ void tm_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+
+// The .x halves (row r) of this lane's 4 NV columns of an interleaved slot.
+template <int NV>
+__device__ __forceinline__ void load_row_x(const float2 *slot, int lane, float *u)
+{
+    const float4 *src = reinterpret_cast<const float4 *>(slot);
+#pragma unroll
+    for (int k = 0; k < 2 * NV; ++k) {
+        const int i = 2 * lane + k;                          // swizzled (pair_put_row)
+        const float4 q = src[i ^ ((i >> 3) & 1)];
+        u[2 * k] = q.x;
+        u[2 * k + 1] = q.z;
+    }
+}
+
+template <int R>
+__global__ void __maxnreg__(LOP_PAIR_TM_MAXREG) bilateral_pair_tm_kernel(const __grid_constant__ BilateralSep p)
+{
+    using S = pair::Shape<R>;
+    constexpr int SW = S::SW, NV = S::NV, NR = S::NR, PAD = S::PAD, HLN = S::HLN;
+    constexpr int NT = R + 1;                                    // TMEM ring slots
+    const Common &c = p.c;
+    const Geom &g = c.in;
+    extern __shared__ float4 smem4[];
+    __shared__ uint32_t tm_base_sh;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    float *wbase = reinterpret_cast<float *>(smem4) + warp * pair::ShapeTM<R>::WARP_FLOATS;
+    float2 *ring2 = reinterpret_cast<float2 *>(wbase);                    // NR x SW pairs
+    float4 *stg = reinterpret_cast<float4 *>(wbase + S::RING2);           // SW
+    int *cm = reinterpret_cast<int *>(wbase + S::RING2 + SW);             // SW
+    if (warp == 0) {
+        asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;"
+                     ::"r"(smem_addr(&tm_base_sh)), "n"(pair::kTmemCols) : "memory");
+        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+    const uint32_t tbase = tm_base_sh + ((uint32_t)(32 * (warp & 3)) << 16);
+    const int b = blockIdx.z;
+    const int ox0 = (c.roi_x0 & ~3) + blockIdx.x * S::OW;
+    const int T = p.pair_rows;
+    const int y0 = c.roi_y0 + (blockIdx.y * pair::NW + warp) * T;
+    const int roi_y1 = c.roi_y0 + c.roi_h;
+    if (y0 < roi_y1) {                                           // warp-uniform
+        const int yend = min(y0 + T, roi_y1);
+        const int ix0 = ox0 - S::HL + c.off_x - PAD;
+        const bool vec_ok = ((ix0 & 3) == 0) && ((g.stride & 15) == 0) &&
+                            ((reinterpret_cast<uintptr_t>(g.data + (int64_t)b * g.bstride) & 15) == 0);
+        pair_colmap<SW>(c, ix0, cm, lane);
+        __syncwarp();
+        // rows y0-R .. y0 -> interleaved slots 0..R; raw row r is fetched into
+        // the storage of slot r + 1 (not written until row r + 1 is put)
+        for (int r = 0; r <= R; ++r)
+            pair_issue_row<SW>(c, b, y0 - R + r + c.off_y, ix0, reinterpret_cast<float4 *>(ring2 + (r + 1) * SW),
+                               cm, lane, vec_ok);
+        asm volatile("cp.async.wait_all;" ::: "memory");
+        for (int r = 0; r <= R; ++r) {
+            pair_put_row<SW, false>(c, y0 - R + r + c.off_y, ix0, p.alpha,
+                                    reinterpret_cast<const float4 *>(ring2 + (r + 1) * SW), nullptr,
+                                    ring2 + r * SW, r > 0 ? ring2 + (r - 1) * SW : nullptr, cm, lane, vec_ok);
+            __syncwarp();
+        }
+        const float zero8[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+#pragma unroll
+        for (int k = 0; k < NT; ++k) tm_st8(tbase + 8 * k, zero8);
+        const int x_out = ox0 + 4 * (lane - HLN);
+        const bool store_lane = lane >= HLN && lane < 32 - HLN && x_out < c.roi_x0 + c.roi_w &&
+                                x_out + 3 >= c.roi_x0;
+        int slot0 = 0, ts0 = 0;                                  // ring slot / TMEM slot of row s
+#pragma unroll 1
+        for (int s = y0 - R; s < yend; ++s) {
+            const bool pre = s + 1 < yend;
+            if (pre) pair_issue_row<SW>(c, b, s + R + 1 + c.off_y, ix0, stg, cm, lane, vec_ok);
+            const int kmin = y0 - s;
+            float u[4 * NV];
+            load_row_x<NV>(ring2 + slot0 * SW, lane, u);
+            const float cen[4] = {u[PAD], u[PAD + 1], u[PAD + 2], u[PAD + 3]};
+            tm_wait_st();                                        // last step's stores have landed
+            float DP[8];                                         // row s: D[0..3], P[0..3]
+            tm_ld8(tbase + 8 * ts0, DP);
+            tm_wait_ld8(DP);
+            float *D0 = DP, *P0 = DP + 4;
+            if (kmin <= 0) {                                     // dy = 0: own row (scalar)
+                float rd[4], rp[4], qd[4], qp[4];
+                pair_row1<R, PAD, true>(u, cen, p.lx, p.nk, rd, rp, qd, qp);
+                const float cy = p.cy[R];
+                fold4(cy, rd, rp, D0, P0);
+                fold4(cy, qd, qp, D0, P0);
+            }
+#pragma unroll 1
+            for (int dy = 1; dy + 1 <= R; dy += 2) {             // row pairs (dy, dy+1): packed
+                if (dy + 1 < kmin) continue;
+                const int sl = slot0 + dy >= NR ? slot0 + dy - NR : slot0 + dy;
+                float2 v[4 * NV];
+                {
+                    const float4 *src = reinterpret_cast<const float4 *>(ring2 + sl * SW);
+#pragma unroll
+                    for (int k = 0; k < 2 * NV; ++k) {
+                        const int i = 2 * lane + k;
+                        const float4 q = src[i ^ ((i >> 3) & 1)];
+                        v[2 * k] = make_float2(q.x, q.y);
+                        v[2 * k + 1] = make_float2(q.z, q.w);
+                    }
+                }
+                float2 rd[4], rp[4], qd[4], qp[4];
+                pair_row2<R, PAD>(v, cen, p.lx, rd, rp, qd, qp);
+                const float cya = p.cy[dy + R], cyb = p.cy[dy + 1 + R];
+                float ta[4], tb[4], sa[4], sb[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) { ta[j] = rd[j].x; sa[j] = rp[j].x; tb[j] = rd[j].y; sb[j] = rp[j].y; }
+                fold4(cya, ta, sa, D0, P0);
+                fold4(cyb, tb, sb, D0, P0);
+#pragma unroll
+                for (int j = 0; j < 4; ++j) { ta[j] = qd[j].x; sa[j] = qp[j].x; tb[j] = qd[j].y; sb[j] = qp[j].y; }
+                const int ka = ts0 + dy >= NT ? ts0 + dy - NT : ts0 + dy;
+                const int kb = ka + 1 >= NT ? ka + 1 - NT : ka + 1;
+                float A[8], B[8];                                // partner rows s+dy, s+dy+1
+                tm_ld8(tbase + 8 * ka, A);
+                tm_ld8(tbase + 8 * kb, B);
+                tm_wait_ld16(A, B);
+                fold4(cya, ta, sa, A, A + 4);
+                fold4(cyb, tb, sb, B, B + 4);
+                tm_st8(tbase + 8 * ka, A);
+                tm_st8(tbase + 8 * kb, B);
+            }
+            if constexpr (R % 2 == 1) {                          // odd R: last row dy = R (scalar)
+                const int sl = slot0 + R >= NR ? slot0 + R - NR : slot0 + R;
+                float v[4 * NV];
+                load_row_x<NV>(ring2 + sl * SW, lane, v);
+                float rd[4], rp[4], qd[4], qp[4];
+                pair_row1<R, PAD, false>(v, cen, p.lx, p.nk, rd, rp, qd, qp);
+                const float cy = p.cy[2 * R];
+                fold4(cy, rd, rp, D0, P0);
+                const int kr = ts0 + R >= NT ? ts0 + R - NT : ts0 + R;
+                float A[8];
+                tm_ld8(tbase + 8 * kr, A);
+                tm_wait_ld8(A);
+                fold4(cy, qd, qp, A, A + 4);
+                tm_st8(tbase + 8 * kr, A);
+            }
+            if (s >= y0 && store_lane) {
+                float res[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) res[j] = bilateral_finish_scaled(D0[j], P0[j], p.inv_alpha);
+                if (x_out >= c.roi_x0) {
+                    store4(c, b, s, x_out, res);
+                } else {
+                    float *orow = reinterpret_cast<float *>(c.out.data + (int64_t)b * c.out.bstride +
+                                                            (int64_t)s * c.out.stride);
+#pragma unroll
+                    for (int j = 0; j < 4; ++j)
+                        if (x_out + j >= c.roi_x0 && x_out + j < c.roi_x0 + c.roi_w) orow[x_out + j] = res[j];
+                }
+            }
+            tm_st8(tbase + 8 * ts0, zero8);                      // the slot now serves row s + R + 1
+            if (pre) {
+                const int sn = slot0 + R + 1 >= NR ? slot0 + R + 1 - NR : slot0 + R + 1;
+                const int sp = slot0 + R >= NR ? slot0 + R - NR : slot0 + R;
+                asm volatile("cp.async.wait_all;" ::: "memory");
+                pair_put_row<SW, false>(c, s + R + 1 + c.off_y, ix0, p.alpha, stg, nullptr, ring2 + sn * SW,
+                                        ring2 + sp * SW, cm, lane, vec_ok);
+            }
+            __syncwarp();
+            slot0 = slot0 + 1 == NR ? 0 : slot0 + 1;
+            ts0 = ts0 + 1 == NT ? 0 : ts0 + 1;
+        }
+        tm_wait_st();
+    }
+    asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+    __syncthreads();
+    if (warp == 0) {
+        asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tm_base_sh),
+                     "n"(pair::kTmemCols) : "memory");
+    }
+}
+
 // ------------------------------------------------------------- launchers
 template <typename P, typename K>
 static cudaError_t launch_tiled(K kernel, const P &p, size_t smem, cudaStream_t stream,
@@ -901,17 +1134,34 @@ int bilateral_sep_max_npoly(int rx) { return rx >= 4 ? 1 : 0; }
 // Alg. 2 idea -- pick the configuration from occupancy -- on B200 terms):
 // cost(T) = waves(T) * (T + warm-up), waves = ceil(CTAs / resident CTAs);
 // LOP_PAIR_ROWS overrides.
+#ifndef LOP_PAIR_TMEM
+#define LOP_PAIR_TMEM 1       // default kernel: 1 = partner ring in TMEM (bilateral_pair_tm_kernel)
+#endif
+static bool pair_tmem_enabled()
+{
+    static const int v = [] {
+        const char *env = std::getenv("LOP_PAIR_TMEM");
+        return env ? std::atoi(env) : LOP_PAIR_TMEM;
+    }();
+    return v != 0;
+}
+
 template <int R>
 static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
 {
     using S = pair::Shape<R>;
-    static PerDevice smem_set, resident_cache;
-    const size_t smem = (size_t)pair::NW * S::WARP_FLOATS * sizeof(float);
+    const bool tm = pair_tmem_enabled();
+    static PerDevice smem_set, resident_cache, smem_set_tm, resident_cache_tm;
+    const size_t smem = tm ? std::max((size_t)pair::NW * pair::ShapeTM<R>::WARP_FLOATS * sizeof(float),
+                                      (size_t)pair::kTmemMinSmem)
+                           : (size_t)pair::NW * S::WARP_FLOATS * sizeof(float);
+    auto kern = tm ? bilateral_pair_tm_kernel<R> : bilateral_pair_kernel<R>;
     cudaError_t e;
-    const int64_t resident = resident_ctas(bilateral_pair_kernel<R>, pair::NW * 32, smem, smem_set,
-                                           resident_cache, e);
+    const int64_t resident =
+        tm ? resident_ctas_tmem(kern, pair::NW * 32, smem, pair::kTmemCols, smem_set_tm, resident_cache_tm, e)
+           : resident_ctas(kern, pair::NW * 32, smem, smem_set, resident_cache, e);
     if (e != cudaSuccess) return e;
-    e = ensure_smem(bilateral_pair_kernel<R>, smem, smem_set);
+    e = ensure_smem(kern, smem, tm ? smem_set_tm : smem_set);
     if (e != cudaSuccess) return e;
     BilateralSep p = p0;
     const int64_t strips = ((p.c.roi_x0 & 3) + p.c.roi_w + S::OW - 1) / S::OW;
@@ -920,7 +1170,7 @@ static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
     static thread_local int64_t memo_key[4] = {-1, -1, -1, -1};
     static thread_local int memo_T = 0;
     if (T <= 0 && memo_key[0] == p.c.roi_h && memo_key[1] == strips && memo_key[2] == p.c.batch &&
-        memo_key[3] == resident)
+        memo_key[3] == resident * 2 + tm)
         T = memo_T;
     if (T <= 0) {
         // every T from 1 to the ROI height: waves of resident CTAs x rows per warp
@@ -937,13 +1187,13 @@ static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
             if (T == 0 || cost < best) { best = cost; T = t; }
             if (segs == 1) break;
         }
-        memo_key[0] = p.c.roi_h; memo_key[1] = strips; memo_key[2] = p.c.batch; memo_key[3] = resident;
+        memo_key[0] = p.c.roi_h; memo_key[1] = strips; memo_key[2] = p.c.batch; memo_key[3] = resident * 2 + tm;
         memo_T = T;
     }
     p.pair_rows = T;
     const int64_t segs = (p.c.roi_h + T - 1) / T;
     dim3 grid((unsigned)strips, (unsigned)((segs + pair::NW - 1) / pair::NW), p.c.batch);
-    bilateral_pair_kernel<R><<<grid, pair::NW * 32, smem, stream>>>(p);
+    kern<<<grid, pair::NW * 32, smem, stream>>>(p);
     return cudaGetLastError();
 }
 
