@@ -409,7 +409,8 @@ def sfu_roofline(peaks, px_per_launch, launch_ms):
     achieved_168 = taps * px_per_launch / (launch_ms / 1000.0) / 1e12
     peak = sfu_peak_tex2(peaks)
     return {"bound": "alu",
-            "kernel": "lop::bilateral_pair_kernel<6>" if pair else "lop::bilateral_sep_kernel<6>",
+            "kernel": ("lop::bilateral_pair_tm_kernel<6>" if os.environ.get("LOP_PAIR_TMEM", "1") != "0"
+                       else "lop::bilateral_pair_kernel<6>") if pair else "lop::bilateral_sep_kernel<6>",
             "achieved": round(achieved, 4), "peak": round(peak, 4), "unit": "Tex2/s",
             "frac": round(achieved / peak, 4),
             "work_per_launch": "%d ex2 (= %d distinct per px x %d px)" % (ex2_per_launch, ex2_px,
@@ -526,7 +527,8 @@ def run_lop(args, dist, peaks):
     # DRAM traffic is not measurable inside this process (no profiler); the ncu
     # capture of the same kernel is committed under profiles/ 
     roofline["traffic"] = None
-    roofline["traffic_note"] = "dram bytes per launch: see profiles/r02_*ncu_full_bilateral_pair*.md"
+    roofline["traffic_note"] = ("dram bytes per launch (ncu --set full of the same kernel and "
+                                "config): profiles/r02/ncu_full_bilateral_pair_tm.md")
     result = dict(metric=BASELINE_METRIC, value=round(value, 2), unit="Mpixel/s",
                   n_gpus=dist.world, steps=K, warmup=W, ms_per_step=round(total_ms / K, 5),
                   higher_is_better=True, scaling=wl["scaling"], vs_baseline=None, dtype="f32",

@@ -24,6 +24,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 #include <type_traits>
@@ -540,7 +541,10 @@ template <typename T, typename TO, int R, int SWAR, int TS, int NBUF>
 cudaError_t launch_cfg(const ConvSep &s, cudaStream_t stream)
 {
     using S = TileShape<T>;
-    const size_t smem = (size_t)NBUF * (TS + 2 * R) * S::ROW_BYTES;
+    size_t smem = (size_t)NBUF * (TS + 2 * R) * S::ROW_BYTES;
+    // LOP_CONV_SMEM_PAD (exploration): extra dynamic shared memory per CTA, which caps
+    // the co-resident CTAs (more, staggered waves instead of one lock-step wave)
+    if (const char *env = std::getenv("LOP_CONV_SMEM_PAD")) smem += (size_t)std::max(0, std::atoi(env));
     static PerDevice smem_set, resident;
     cudaError_t e;
     int64_t grid_max = resident_ctas(conv_sep_kernel<T, TO, R, SWAR, TS, NBUF>, convt::NT, smem,

@@ -68,7 +68,7 @@ __global__ void __launch_bounds__(pyr::RW * pyr::RWARPS) pyr_reduce_kernel(const
     char *ob = p.out.data + (int64_t)b * p.out.bstride;
     const bool ovec = cx + 1 < p.out.W && (p.out.stride & 7) == 0 && (reinterpret_cast<uintptr_t>(ob) & 7) == 0;
     constexpr int NF = 2 * pyr::RROWS + 3;                            // fine rows per warp
-    // all of the warp's row loads are issued before any is used (11 x 512 B in
+    // all of the warp's row loads are issued before any is used (7 x 512 B in
     // flight per warp; a load-use chain per row left the kernel latency-bound)
     float4 qs[NF];
     if (inside) {
