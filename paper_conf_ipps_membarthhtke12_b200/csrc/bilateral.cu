@@ -1150,7 +1150,12 @@ template <int R>
 static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
 {
     using S = pair::Shape<R>;
-    const bool tm = pair_tmem_enabled();
+    // TMEM kernel for launches of at least 1024^2 pixels: below that the launch is
+    // latency-bound and the TMEM allocation / barriers / ring clearing cost more
+    // than the occupancy buys (config 1, 256^2 3x3: 4.5 -> 6.1 us per launch).
+    // Both kernels give the same bits, so the choice is free to depend on size.
+    const bool tm = pair_tmem_enabled() &&
+                    (double)p0.c.in.W * (double)p0.c.in.GH * (double)p0.c.batch >= 1024.0 * 1024.0;
     static PerDevice smem_set, resident_cache, smem_set_tm, resident_cache_tm;
     const size_t smem = tm ? std::max((size_t)pair::NW * pair::ShapeTM<R>::WARP_FLOATS * sizeof(float),
                                       (size_t)pair::kTmemMinSmem)
