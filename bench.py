@@ -739,7 +739,12 @@ def conv_extras(lop, synthetic, dev, stream, hbm, img, timed):
                                 out=f_out[k], stream=s), 12),
         ("local_2acc_max_absdiff_u8_i32",
          lambda k, s: lop.local([u_in[k], u_in_b[k]], [np.ones((3, 3), np.int32)] * 2, "max",
-                                "absdiff", "clamp", out=i_out[k], stream=s), 6)]
+                                "absdiff", "clamp", out=i_out[k], stream=s), 6),
+        # the same f32 operator with a point-operator prologue on both accessors (N3,
+        # reading c27: window/level a I + b applied once per staged element)
+        ("local_2acc_sum_product_f32_point_prologue",
+         lambda k, s: lop.local([f_in[k], f_in_b[k]], [m5, m3], "sum", "product", "clamp",
+                                out=f_out[k], stream=s, point=[(1.5, -0.25), (-1.0, 1.0)]), 12)]
     # global operator (sum of all pixels, deterministic two-level reduction)
     gres = torch.empty(1, dtype=torch.float64, device=dev)
     gwork = torch.zeros(1025, dtype=torch.float64, device=dev)     # LOP_GLOBAL_WORK_DOUBLES
@@ -747,7 +752,11 @@ def conv_extras(lop, synthetic, dev, stream, hbm, img, timed):
         ("global_sum_f32", lambda k, s: lop.global_reduce(f_in[k], "sum", out=gres, work=gwork,
                                                           stream=s), 4),
         ("global_max_u8", lambda k, s: lop.global_reduce(u_in[k], "max", out=gres, work=gwork,
-                                                         stream=s), 1)]
+                                                         stream=s), 1),
+        ("global_sumsq_f32", lambda k, s: lop.global_reduce(f_in[k], "sumsq", out=gres, work=gwork,
+                                                            stream=s), 4),
+        ("global_sumsq_u8", lambda k, s: lop.global_reduce(u_in[k], "sumsq", out=gres, work=gwork,
+                                                           stream=s), 1)]
     # Laplacian-pyramid steps of the multiresolution filter (N4, reading c28):
     # REDUCE 4096^2 -> 2048^2 (4 B read per fine pixel + 4 B per coarse = 5 B / fine px),
     # band-pass EXPAND with the fine addend (coarse 1 B + addend 4 B + out 4 B = 9 B / fine px)
