@@ -258,6 +258,20 @@ struct ConvTile {
     int b, tx0, ty0, nrows;
 };
 
+// Tile (blockIdx.x, blockIdx.y) of frame blockIdx.z (one tile per CTA): no
+// integer division (the linear form below costs two division sequences per warp).
+template <typename T, int TS>
+__device__ __forceinline__ ConvTile conv_tile_grid(const Common &c)
+{
+    using S = TileShape<T>;
+    ConvTile ct;
+    ct.b = blockIdx.z;
+    ct.tx0 = c.roi_x0 + (int)blockIdx.x * S::TWE;
+    ct.ty0 = c.roi_y0 + (int)blockIdx.y * TS;
+    ct.nrows = min(TS, c.roi_y0 + c.roi_h - ct.ty0);
+    return ct;
+}
+
 template <typename T, int TS>
 __device__ __forceinline__ ConvTile conv_tile_at(const Common &c, int t)
 {
@@ -456,15 +470,16 @@ __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_consta
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
-    int t = blockIdx.x;
-    if (t < ntiles) conv_stage<T, R>(c, conv_tile_at<T, TS>(c, t), buf0, &bar[0]);
-    if (NBUF == 1) {
-        if (t >= ntiles) return;
+    if constexpr (NBUF == 1) {                      // 3D grid: one tile per CTA
+        const ConvTile ct = conv_tile_grid<T, TS>(c);
+        conv_stage<T, R>(c, ct, buf0, &bar[0]);
         __syncthreads();
         mbar_wait(&bar[0], 0);
-        conv_compute<T, TO, R, SWAR, TS>(p, conv_tile_at<T, TS>(c, t), buf0);
+        conv_compute<T, TO, R, SWAR, TS>(p, ct, buf0);
         return;
     }
+    int t = blockIdx.x;
+    if (t < ntiles) conv_stage<T, R>(c, conv_tile_at<T, TS>(c, t), buf0, &bar[0]);
     for (int it = 0; t < ntiles; t += gridDim.x, ++it) {
         const int cur = it & 1;
         __syncthreads();        // tile it-1 fully consumed; element fills of tile it visible
@@ -563,7 +578,11 @@ cudaError_t launch_cfg(const ConvSep &s, cudaStream_t stream)
     }
     const long ntiles = (long)((s.c.roi_w + S::TWE - 1) / S::TWE) * ((s.c.roi_h + TS - 1) / TS) *
                         s.c.batch;
-    const int grid = NBUF == 1 ? (int)ntiles : (int)(ntiles < grid_max ? ntiles : grid_max);
+    dim3 grid;
+    if (NBUF == 1)
+        grid = dim3((s.c.roi_w + S::TWE - 1) / S::TWE, (s.c.roi_h + TS - 1) / TS, s.c.batch);
+    else
+        grid = dim3((unsigned)(ntiles < grid_max ? ntiles : grid_max));
     conv_sep_kernel<T, TO, R, SWAR, TS, NBUF><<<grid, convt::NT, smem, stream>>>(s);
     return cudaGetLastError();
 }
