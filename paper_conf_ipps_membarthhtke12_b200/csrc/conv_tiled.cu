@@ -77,7 +77,10 @@ template <typename T> struct TileShape {
 // (a + e) + 4 (b + d) + 6 c -- two adds, a shift-add and one IMAD.
 enum { SW_ON = 1, SW_SYM = 2, SW_SH8 = 4, SW_I32 = 8, SW_BIN5 = 16 };
 
-template <int R, int TS, int MODE>
+// FULL: the tile has all TS + 2R staged rows (every tile but a partial last
+// one), so the unrolled row loop carries no per-row bound check (the check made
+// the compiler wrap every row in a divergence region).
+template <int R, int TS, int MODE, bool FULL>
 __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tcol, int srows,
                                              char *orow0, int64_t ostride, int ox0, int roi_x1,
                                              bool ovec)
@@ -94,7 +97,7 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
     uint32_t h[2 * R + 1][4];                     // pairs (0,2) (1,3) (4,6) (5,7)
 #pragma unroll
     for (int k = 0; k < TS + 2 * R; ++k) {
-        if (k >= srows) break;
+        if (!FULL && k >= srows) break;
         const uint8_t *rp = tcol + k * SWE;
         const uint2 cv = *reinterpret_cast<const uint2 *>(rp);
         const uint32_t W[4] = {*reinterpret_cast<const uint32_t *>(rp - 4), cv.x, cv.y,
@@ -164,7 +167,8 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
                 v[px] = quantize_shift((int)(q4[jj] & 0xFFFFu) - p.sw_off, p.shift);
                 v[px + 2] = quantize_shift((int)(q4[jj] >> 16) - p.sw_off, p.shift);
             }
-            int32_t *op = reinterpret_cast<int32_t *>(orow0 + (int64_t)o * ostride) + ox0;
+            int32_t *op = reinterpret_cast<int32_t *>(orow0) + ox0;   // output row o (running pointer)
+            orow0 += ostride;
             if (ovec) {
                 *reinterpret_cast<int4 *>(op) = make_int4(v[0], v[1], v[2], v[3]);
                 *reinterpret_cast<int4 *>(op + 4) = make_int4(v[4], v[5], v[6], v[7]);
@@ -178,7 +182,8 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
         // lo = pixels 0..3 = lanes of q4[0] (0, 2) and q4[1] (1, 3); hi likewise
         const uint32_t lo = SH8 ? __byte_perm(q4[0], q4[1], 0x7351) : __byte_perm(q4[0], q4[1], 0x6240);
         const uint32_t hi = SH8 ? __byte_perm(q4[2], q4[3], 0x7351) : __byte_perm(q4[2], q4[3], 0x6240);
-        uint8_t *op = reinterpret_cast<uint8_t *>(orow0 + (int64_t)o * ostride) + ox0;
+        uint8_t *op = reinterpret_cast<uint8_t *>(orow0) + ox0;    // output row o (running pointer)
+        orow0 += ostride;
         if (ovec) {
             *reinterpret_cast<uint2 *>(op) = make_uint2(lo, hi);
         } else {
@@ -195,7 +200,7 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
 // FFMA2 per tap with the coefficient as a broadcast pair.  Each lane performs
 // exactly the scalar operation of its column (same operands, same order,
 // round-to-nearest), so the result is the scalar kernel's bit for bit.
-template <int R, int TS>
+template <int R, int TS, bool FULL>
 __device__ __forceinline__ void conv_f32_packed(const ConvSep &p, const float *tcol, int srows,
                                                 char *orow0, int64_t ostride, int ox0, int roi_x1,
                                                 bool ovec)
@@ -205,7 +210,7 @@ __device__ __forceinline__ void conv_f32_packed(const ConvSep &p, const float *t
     float2 h[P][2];                                                 // (h0,h1), (h2,h3) ring
 #pragma unroll
     for (int k = 0; k < TS + 2 * R; ++k) {
-        if (k >= srows) break;
+        if (!FULL && k >= srows) break;
         const float *rp = tcol + k * SWE;
         float v[4 + 2 * R];
         const float4 cv = *reinterpret_cast<const float4 *>(rp);
@@ -241,7 +246,8 @@ __device__ __forceinline__ void conv_f32_packed(const ConvSep &p, const float *t
                 a = __ffma2_rn(h[(o + t) % P][q], make_float2(p.cf[t], p.cf[t]), a);
             out[q] = a;
         }
-        float *op = reinterpret_cast<float *>(orow0 + (int64_t)o * ostride) + ox0;
+        float *op = reinterpret_cast<float *>(orow0) + ox0;        // output row o (running pointer)
+        orow0 += ostride;
         if (ovec) {
             *reinterpret_cast<float4 *>(op) = make_float4(out[0].x, out[0].y, out[1].x, out[1].y);
         } else {
@@ -304,7 +310,7 @@ __device__ __forceinline__ void conv_stage(const Common &c, const ConvTile &ct, 
 
 
 // Filter one staged tile: each thread streams its PX columns down the tile.
-template <typename T, typename TO, int R, int SWAR, int TS>
+template <typename T, typename TO, int R, int SWAR, int TS, bool FULL>
 __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &ct, const T *tile)
 {
     constexpr int RX = R, RY = R;
@@ -325,19 +331,20 @@ __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &c
     const T *tcol = tile + PADE + threadIdx.x * PX;              // this thread's centre column
     if constexpr (SWAR != 0) {
         static_assert(SWAR == 0 || sizeof(T) == 1, "SWAR is for u8 inputs");
-        conv_u8_swar<R, TS, SWAR>(p, reinterpret_cast<const uint8_t *>(tcol), srows,
-                        obase + (int64_t)ty0 * c.out.stride, c.out.stride, ox0, roi_x1, ovec);
+        char *orow0 = obase + (int64_t)ty0 * c.out.stride;
+        conv_u8_swar<R, TS, SWAR, FULL>(p, reinterpret_cast<const uint8_t *>(tcol), srows, orow0,
+                                        c.out.stride, ox0, roi_x1, ovec);
         return;
     }
     if constexpr (F) {
-        conv_f32_packed<R, TS>(p, reinterpret_cast<const float *>(tcol), srows,
+        conv_f32_packed<R, TS, FULL>(p, reinterpret_cast<const float *>(tcol), srows,
                                obase + (int64_t)ty0 * c.out.stride, c.out.stride, ox0, roi_x1, ovec);
         return;
     }
     A h[2 * RY + 1][PX];                                          // horizontal sums, ring
 #pragma unroll
     for (int k = 0; k < TS + 2 * RY; ++k) {
-        if (k >= srows) break;
+        if (!FULL && k >= srows) break;
         // ---- gather PX + 2RX values of staged row k
         A v[PX + 2 * RX];
         const T *rp = tcol + k * SWE;
@@ -475,7 +482,9 @@ __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_consta
         conv_stage<T, R>(c, ct, buf0, &bar[0]);
         __syncthreads();
         mbar_wait(&bar[0], 0);
-        conv_compute<T, TO, R, SWAR, TS>(p, ct, buf0);
+        // full tiles (all but a partial last row of tiles) without per-row bound checks
+        if (ct.nrows == TS) conv_compute<T, TO, R, SWAR, TS, true>(p, ct, buf0);
+        else conv_compute<T, TO, R, SWAR, TS, false>(p, ct, buf0);
         return;
     }
     int t = blockIdx.x;
@@ -487,7 +496,7 @@ __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_consta
         if (tn < ntiles)
             conv_stage<T, R>(c, conv_tile_at<T, TS>(c, tn), cur ? buf0 : buf1, &bar[cur ^ 1]);
         mbar_wait(&bar[cur], (it >> 1) & 1);
-        conv_compute<T, TO, R, SWAR, TS>(p, conv_tile_at<T, TS>(c, t), cur ? buf1 : buf0);
+        conv_compute<T, TO, R, SWAR, TS, false>(p, conv_tile_at<T, TS>(c, t), cur ? buf1 : buf0);
     }
 }
 
