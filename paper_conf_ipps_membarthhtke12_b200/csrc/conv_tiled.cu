@@ -80,7 +80,7 @@ enum { SW_ON = 1, SW_SYM = 2, SW_SH8 = 4, SW_I32 = 8, SW_BIN5 = 16 };
 // FULL: the tile has all TS + 2R staged rows (every tile but a partial last
 // one), so the unrolled row loop carries no per-row bound check (the check made
 // the compiler wrap every row in a divergence region).
-template <int R, int TS, int MODE, bool FULL>
+template <int R, int TS, int MODE, bool FULL, bool VEC>
 __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tcol, int srows,
                                              char *orow0, int64_t ostride, int ox0, int roi_x1,
                                              bool ovec)
@@ -169,7 +169,7 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
             }
             int32_t *op = reinterpret_cast<int32_t *>(orow0) + ox0;   // output row o (running pointer)
             orow0 += ostride;
-            if (ovec) {
+            if (VEC || ovec) {
                 *reinterpret_cast<int4 *>(op) = make_int4(v[0], v[1], v[2], v[3]);
                 *reinterpret_cast<int4 *>(op + 4) = make_int4(v[4], v[5], v[6], v[7]);
             } else {
@@ -184,7 +184,7 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
         const uint32_t hi = SH8 ? __byte_perm(q4[2], q4[3], 0x7351) : __byte_perm(q4[2], q4[3], 0x6240);
         uint8_t *op = reinterpret_cast<uint8_t *>(orow0) + ox0;    // output row o (running pointer)
         orow0 += ostride;
-        if (ovec) {
+        if (VEC || ovec) {
             *reinterpret_cast<uint2 *>(op) = make_uint2(lo, hi);
         } else {
 #pragma unroll
@@ -332,8 +332,16 @@ __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &c
     if constexpr (SWAR != 0) {
         static_assert(SWAR == 0 || sizeof(T) == 1, "SWAR is for u8 inputs");
         char *orow0 = obase + (int64_t)ty0 * c.out.stride;
-        conv_u8_swar<R, TS, SWAR, FULL>(p, reinterpret_cast<const uint8_t *>(tcol), srows, orow0,
-                                        c.out.stride, ox0, roi_x1, ovec);
+        // VEC: the whole tile row is inside the iteration space and 16-B aligned, so
+        // every thread stores whole vectors (no per-row divergent store branch)
+        const bool cta_vec = ct.tx0 + S::TWE <= roi_x1 && (ct.tx0 % PX) == 0 &&
+                             ((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) % 16) == 0;
+        if (cta_vec)
+            conv_u8_swar<R, TS, SWAR, FULL, true>(p, reinterpret_cast<const uint8_t *>(tcol), srows, orow0,
+                                                  c.out.stride, ox0, roi_x1, ovec);
+        else
+            conv_u8_swar<R, TS, SWAR, FULL, false>(p, reinterpret_cast<const uint8_t *>(tcol), srows, orow0,
+                                                   c.out.stride, ox0, roi_x1, ovec);
         return;
     }
     if constexpr (F) {
