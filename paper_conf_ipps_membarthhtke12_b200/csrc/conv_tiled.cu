@@ -608,7 +608,9 @@ cudaError_t launch_cfg(const ConvSep &s, cudaStream_t stream)
 // else the default measured best on B200.  The sweep space is
 // instantiated for radii 1 and 2 (Sobel 3x3, Gaussian 5x5); other radii use
 // the default.
-constexpr int kDefTS = 8, kDefTSSwar = 16, kDefNBUF = 1;   // tools/tune_conv.py on B200, round 1
+// f32 / other: 8 rows per tile (round 1); 4 rows for radii <= 2 (f32 Gaussian 5x5 23.8 -> 22.4 us
+// at 4096^2 once the full-tile instances dropped the per-row checks, tools/time_conv_all.py)
+constexpr int kDefTS = 8, kDefTSSmallR = 4, kDefTSSwar = 16, kDefNBUF = 1;
 // u8 -> i32 (Sobel): 4 rows per tile -- a 4096^2 image is then 4096 tiles (~2 waves), so
 // CTAs in their store phase overlap CTAs in their load phase (0.0180 vs 0.0192 ms at 8
 // rows; profiles/r01_tune_conv.jsonl)
@@ -617,7 +619,7 @@ constexpr int kDefTSI32 = 4;
 template <typename T, typename TO, int R, int SWAR = 0>
 cudaError_t launch_sep(const ConvSep &s, cudaStream_t stream)
 {
-    int ts = SWAR ? kDefTSSwar : (sizeof(T) == 1 && sizeof(TO) == 4 ? kDefTSI32 : kDefTS);
+    int ts = SWAR ? kDefTSSwar : (sizeof(T) == 1 && sizeof(TO) == 4 ? kDefTSI32 : (R <= 2 ? kDefTSSmallR : kDefTS));
     int nbuf = kDefNBUF;
     if (const char *env = std::getenv("LOP_CONV_CFG")) std::sscanf(env, "%d:%d", &ts, &nbuf);
     if constexpr (R == 1 || R == 2) {
