@@ -63,35 +63,17 @@ template <int OP, int N> __device__ __forceinline__ uint32_t red_n(const uint32_
     return m;
 }
 
-template <typename T, int OP, int R, int TS_>
-__global__ void __launch_bounds__(red::NT) reduce_tiled_kernel(const __grid_constant__ ReduceParams p)
+// Filter one staged tile (thread: PX columns streamed down the tile).  FULL:
+// all TS + 2R staged rows present (no per-row bound check); VEC: the CTA's
+// whole tile row is inside the iteration space and aligned (every thread
+// stores whole vectors, no per-row divergent store branch).  Output rows are
+// addressed by a running pointer.
+template <typename T, int OP, int R, int TS_, bool FULL, bool VEC>
+__device__ __forceinline__ void reduce_compute(const Common &c, const T *tile, int srows, char *obase,
+                                               int ox0, int roi_x1, bool ovec)
 {
     using S = red::Shape<T, TS_>;
     constexpr int PX = S::PX, SWE = S::SWE, PADE = S::PADE, TS = S::TS, P = 2 * R + 1;
-    static_assert(R >= 1 && R <= 4, "halo must fit the 16-B pad");
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    __shared__ __align__(8) uint64_t bar;
-    T *tile = reinterpret_cast<T *>(smem_raw);
-    const Common &c = p.c;
-    const int b = blockIdx.z;
-    const int tx0 = c.roi_x0 + blockIdx.x * S::TWE, ty0 = c.roi_y0 + blockIdx.y * TS;
-    const int roi_x1 = c.roi_x0 + c.roi_w;
-    const int nrows = min(TS, c.roi_y0 + c.roi_h - ty0), srows = nrows + 2 * R;
-    if (threadIdx.x == 0) {
-        asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&bar)));
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
-    stage_rows<T, SWE, red::NT>(c, b, tx0 + c.off_x - PADE, ty0 + c.off_y - R, srows, tile, &bar);
-    __syncthreads();
-    mbar_wait(&bar, 0);
-
-    const int ox0 = tx0 + threadIdx.x * PX;
-    if (ox0 >= roi_x1) return;
-    char *obase = c.out.data + (int64_t)b * c.out.bstride + (int64_t)ty0 * c.out.stride;
-    const bool ovec = (ox0 + PX <= roi_x1) && (ox0 % PX == 0) &&
-                      (((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) %
-                        (sizeof(T) * PX)) == 0);
     const T *tcol = tile + PADE + threadIdx.x * PX;
     if constexpr (sizeof(T) == 1) {
         // staged words W0..W3 = bytes -4..11 of this thread's 8 columns; sources
@@ -99,7 +81,7 @@ __global__ void __launch_bounds__(red::NT) reduce_tiled_kernel(const __grid_cons
         uint32_t h[P][4];                                        // lanes (0,2) (1,3) (4,6) (5,7)
 #pragma unroll
         for (int k = 0; k < TS + 2 * R; ++k) {
-            if (k >= srows) break;
+            if (!FULL && k >= srows) break;
             const uint8_t *rp = reinterpret_cast<const uint8_t *>(tcol) + k * SWE;
             const uint2 cv = *reinterpret_cast<const uint2 *>(rp);
             const uint32_t W[4] = {*reinterpret_cast<const uint32_t *>(rp - 4), cv.x, cv.y,
@@ -133,8 +115,9 @@ __global__ void __launch_bounds__(red::NT) reduce_tiled_kernel(const __grid_cons
                 q4[jj] = red_n<OP, P>(col);
             }
             const uint32_t lo = __byte_perm(q4[0], q4[1], 0x6240), hi = __byte_perm(q4[2], q4[3], 0x6240);
-            uint8_t *op = reinterpret_cast<uint8_t *>(obase + (int64_t)o * c.out.stride) + ox0;
-            if (ovec) {
+            uint8_t *op = reinterpret_cast<uint8_t *>(obase) + ox0;
+            obase += c.out.stride;
+            if (VEC || ovec) {
                 *reinterpret_cast<uint2 *>(op) = make_uint2(lo, hi);
             } else {
 #pragma unroll
@@ -146,7 +129,7 @@ __global__ void __launch_bounds__(red::NT) reduce_tiled_kernel(const __grid_cons
         float h[P][PX];
 #pragma unroll
         for (int k = 0; k < TS + 2 * R; ++k) {
-            if (k >= srows) break;
+            if (!FULL && k >= srows) break;
             const float *rp = reinterpret_cast<const float *>(tcol) + k * SWE;
             const float4 cv = *reinterpret_cast<const float4 *>(rp);
             const float4 l = *reinterpret_cast<const float4 *>(rp - 4);
@@ -169,8 +152,9 @@ __global__ void __launch_bounds__(red::NT) reduce_tiled_kernel(const __grid_cons
                 for (int t = 1; t < P; ++t) m = red_f<OP>(m, h[(o + t) % P][j]);
                 q[j] = m;
             }
-            float *op = reinterpret_cast<float *>(obase + (int64_t)o * c.out.stride) + ox0;
-            if (ovec) {
+            float *op = reinterpret_cast<float *>(obase) + ox0;
+            obase += c.out.stride;
+            if (VEC || ovec) {
                 *reinterpret_cast<float4 *>(op) = make_float4(q[0], q[1], q[2], q[3]);
             } else {
 #pragma unroll
@@ -179,6 +163,43 @@ __global__ void __launch_bounds__(red::NT) reduce_tiled_kernel(const __grid_cons
             }
         }
     }
+}
+
+template <typename T, int OP, int R, int TS_>
+__global__ void __launch_bounds__(red::NT) reduce_tiled_kernel(const __grid_constant__ ReduceParams p)
+{
+    using S = red::Shape<T, TS_>;
+    constexpr int PX = S::PX, SWE = S::SWE, PADE = S::PADE, TS = S::TS;
+    static_assert(R >= 1 && R <= 4, "halo must fit the 16-B pad");
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ __align__(8) uint64_t bar;
+    T *tile = reinterpret_cast<T *>(smem_raw);
+    const Common &c = p.c;
+    const int b = blockIdx.z;
+    const int tx0 = c.roi_x0 + blockIdx.x * S::TWE, ty0 = c.roi_y0 + blockIdx.y * TS;
+    const int roi_x1 = c.roi_x0 + c.roi_w;
+    const int nrows = min(TS, c.roi_y0 + c.roi_h - ty0), srows = nrows + 2 * R;
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&bar)));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    stage_rows<T, SWE, red::NT>(c, b, tx0 + c.off_x - PADE, ty0 + c.off_y - R, srows, tile, &bar);
+    __syncthreads();
+    mbar_wait(&bar, 0);
+
+    const int ox0 = tx0 + threadIdx.x * PX;
+    if (ox0 >= roi_x1) return;
+    char *obase = c.out.data + (int64_t)b * c.out.bstride + (int64_t)ty0 * c.out.stride;
+    const bool ovec = (ox0 + PX <= roi_x1) && (ox0 % PX == 0) &&
+                      (((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) %
+                        (sizeof(T) * PX)) == 0);
+    const bool full = srows == TS + 2 * R;
+    const bool cta_vec = tx0 + S::TWE <= roi_x1 &&
+                         ((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) % 16) == 0;
+    if (full && cta_vec) reduce_compute<T, OP, R, TS_, true, true>(c, tile, srows, obase, ox0, roi_x1, ovec);
+    else if (full) reduce_compute<T, OP, R, TS_, true, false>(c, tile, srows, obase, ox0, roi_x1, ovec);
+    else reduce_compute<T, OP, R, TS_, false, false>(c, tile, srows, obase, ox0, roi_x1, ovec);
 }
 
 template <int OP>
