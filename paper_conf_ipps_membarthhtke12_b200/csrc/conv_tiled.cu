@@ -200,7 +200,7 @@ __device__ __forceinline__ void conv_u8_swar(const ConvSep &p, const uint8_t *tc
 // FFMA2 per tap with the coefficient as a broadcast pair.  Each lane performs
 // exactly the scalar operation of its column (same operands, same order,
 // round-to-nearest), so the result is the scalar kernel's bit for bit.
-template <int R, int TS, bool FULL>
+template <int R, int TS, bool FULL, bool VEC>
 __device__ __forceinline__ void conv_f32_packed(const ConvSep &p, const float *tcol, int srows,
                                                 char *orow0, int64_t ostride, int ox0, int roi_x1,
                                                 bool ovec)
@@ -248,7 +248,7 @@ __device__ __forceinline__ void conv_f32_packed(const ConvSep &p, const float *t
         }
         float *op = reinterpret_cast<float *>(orow0) + ox0;        // output row o (running pointer)
         orow0 += ostride;
-        if (ovec) {
+        if (VEC || ovec) {
             *reinterpret_cast<float4 *>(op) = make_float4(out[0].x, out[0].y, out[1].x, out[1].y);
         } else {
             const float w[4] = {out[0].x, out[0].y, out[1].x, out[1].y};
@@ -310,14 +310,20 @@ __device__ __forceinline__ void conv_stage(const Common &c, const ConvTile &ct, 
 
 
 // Filter one staged tile: each thread streams its PX columns down the tile.
-template <typename T, typename TO, int R, int SWAR, int TS, bool FULL>
+template <typename T, typename TO, int R, int TS, bool FULL, bool VEC>
+__device__ __forceinline__ void conv_scalar(const ConvSep &p, const T *tcol, int srows, char *obase, int ty0,
+                                            int ox0, int roi_x1, bool ovec);
+
+// FULL: all TS + 2R staged rows present; VEC: the CTA's whole tile row lies in
+// the iteration space and the output is 16-B aligned (whole-vector stores by
+// every thread, no per-row divergent store branch).
+template <typename T, typename TO, int R, int SWAR, int TS, bool FULL, bool VEC>
 __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &ct, const T *tile)
 {
-    constexpr int RX = R, RY = R;
+    constexpr int RY = R;
     using S = TileShape<T>;
-    constexpr int PX = S::PX, SWE = S::SWE, PADE = S::PADE;
+    constexpr int PX = S::PX, PADE = S::PADE;
     constexpr bool F = sizeof(T) == 4;
-    using A = typename std::conditional<F, float, int>::type;   // accumulator type
     const Common &c = p.c;
     const int b = ct.b, ty0 = ct.ty0;
     const int srows = ct.nrows + 2 * RY;
@@ -332,23 +338,29 @@ __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &c
     if constexpr (SWAR != 0) {
         static_assert(SWAR == 0 || sizeof(T) == 1, "SWAR is for u8 inputs");
         char *orow0 = obase + (int64_t)ty0 * c.out.stride;
-        // VEC: the whole tile row is inside the iteration space and 16-B aligned, so
-        // every thread stores whole vectors (no per-row divergent store branch)
-        const bool cta_vec = ct.tx0 + S::TWE <= roi_x1 && (ct.tx0 % PX) == 0 &&
-                             ((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) % 16) == 0;
-        if (cta_vec)
-            conv_u8_swar<R, TS, SWAR, FULL, true>(p, reinterpret_cast<const uint8_t *>(tcol), srows, orow0,
-                                                  c.out.stride, ox0, roi_x1, ovec);
-        else
-            conv_u8_swar<R, TS, SWAR, FULL, false>(p, reinterpret_cast<const uint8_t *>(tcol), srows, orow0,
-                                                   c.out.stride, ox0, roi_x1, ovec);
+        conv_u8_swar<R, TS, SWAR, FULL, VEC>(p, reinterpret_cast<const uint8_t *>(tcol), srows, orow0,
+                                             c.out.stride, ox0, roi_x1, ovec);
         return;
     }
     if constexpr (F) {
-        conv_f32_packed<R, TS, FULL>(p, reinterpret_cast<const float *>(tcol), srows,
+        conv_f32_packed<R, TS, FULL, VEC>(p, reinterpret_cast<const float *>(tcol), srows,
                                obase + (int64_t)ty0 * c.out.stride, c.out.stride, ox0, roi_x1, ovec);
         return;
     }
+    if constexpr (SWAR == 0 && !F) conv_scalar<T, TO, R, TS, FULL, VEC>(p, tcol, srows, obase, ty0, ox0, roi_x1, ovec);
+}
+
+// Scalar (unpacked integer) path: u8 -> u8 without SWAR, u8 -> i32.
+template <typename T, typename TO, int R, int TS, bool FULL, bool VEC>
+__device__ __forceinline__ void conv_scalar(const ConvSep &p, const T *tcol, int srows, char *obase, int ty0,
+                                            int ox0, int roi_x1, bool ovec)
+{
+    constexpr int RX = R, RY = R;
+    using S = TileShape<T>;
+    constexpr int PX = S::PX, SWE = S::SWE;
+    constexpr bool F = sizeof(T) == 4;
+    using A = typename std::conditional<F, float, int>::type;   // accumulator type
+    const Common &c = p.c;
     A h[2 * RY + 1][PX];                                          // horizontal sums, ring
 #pragma unroll
     for (int k = 0; k < TS + 2 * RY; ++k) {
@@ -422,7 +434,7 @@ __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &c
         char *orow = obase + (int64_t)(ty0 + o) * c.out.stride;
         if constexpr (F) {
             float *op = reinterpret_cast<float *>(orow) + ox0;
-            if (ovec) {
+            if (VEC || ovec) {
                 *reinterpret_cast<float4 *>(op) = make_float4(out[0], out[1], out[2], out[3]);
             } else {
 #pragma unroll
@@ -437,7 +449,7 @@ __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &c
                 w[j >> 2] |= (uint32_t)q << (8 * (j & 3));
             }
             uint8_t *op = reinterpret_cast<uint8_t *>(orow) + ox0;
-            if (ovec) {
+            if (VEC || ovec) {
                 *reinterpret_cast<uint2 *>(op) = make_uint2(w[0], w[1]);
             } else {
 #pragma unroll
@@ -449,7 +461,7 @@ __device__ __forceinline__ void conv_compute(const ConvSep &p, const ConvTile &c
             int q[PX];
 #pragma unroll
             for (int j = 0; j < PX; ++j) q[j] = quantize_shift(out[j], p.shift);
-            if (ovec) {
+            if (VEC || ovec) {
                 *reinterpret_cast<int4 *>(op) = make_int4(q[0], q[1], q[2], q[3]);
                 *reinterpret_cast<int4 *>(op + 4) = make_int4(q[4], q[5], q[6], q[7]);
             } else {
@@ -490,9 +502,15 @@ __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_consta
         conv_stage<T, R>(c, ct, buf0, &bar[0]);
         __syncthreads();
         mbar_wait(&bar[0], 0);
-        // full tiles (all but a partial last row of tiles) without per-row bound checks
-        if (ct.nrows == TS) conv_compute<T, TO, R, SWAR, TS, true>(p, ct, buf0);
-        else conv_compute<T, TO, R, SWAR, TS, false>(p, ct, buf0);
+        // full tiles (all but a partial last row of tiles) without per-row bound checks;
+        // whole-vector stores when the tile row lies in the iteration space, aligned
+        using S = TileShape<T>;
+        const char *ob = c.out.data + (int64_t)ct.b * c.out.bstride;
+        const bool cta_vec = ct.tx0 + S::TWE <= c.roi_x0 + c.roi_w && (ct.tx0 % S::PX) == 0 &&
+                             ((reinterpret_cast<uintptr_t>(ob) | (uintptr_t)c.out.stride) % 16) == 0;
+        if (ct.nrows == TS && cta_vec) conv_compute<T, TO, R, SWAR, TS, true, true>(p, ct, buf0);
+        else if (ct.nrows == TS) conv_compute<T, TO, R, SWAR, TS, true, false>(p, ct, buf0);
+        else conv_compute<T, TO, R, SWAR, TS, false, false>(p, ct, buf0);
         return;
     }
     int t = blockIdx.x;
@@ -504,7 +522,7 @@ __global__ void __launch_bounds__(convt::NT) conv_sep_kernel(const __grid_consta
         if (tn < ntiles)
             conv_stage<T, R>(c, conv_tile_at<T, TS>(c, tn), cur ? buf0 : buf1, &bar[cur ^ 1]);
         mbar_wait(&bar[cur], (it >> 1) & 1);
-        conv_compute<T, TO, R, SWAR, TS, false>(p, conv_tile_at<T, TS>(c, t), cur ? buf1 : buf0);
+        conv_compute<T, TO, R, SWAR, TS, false, false>(p, conv_tile_at<T, TS>(c, t), cur ? buf1 : buf0);
     }
 }
 
