@@ -23,7 +23,9 @@ cases = {"gaussian5x5_f32": lambda k, s: lop.gaussian(fi[k], 5, "clamp", out=fo[
          "gaussian5x5_u8": lambda k, s: lop.gaussian(ui[k], 5, "clamp", out=uo[k], stream=s),
          "gaussian3x3_u8": lambda k, s: lop.gaussian(ui[k], 3, "clamp", out=uo[k], stream=s),
          "sobel3x3_u8_i32": lambda k, s: lop.sobel(ui[k], 0, "clamp", out=io_[k], stream=s),
-         "erode5x5_u8": lambda k, s: lop.erode(ui[k], 5, "clamp", out=uo[k], stream=s)}
+         "erode5x5_u8": lambda k, s: lop.erode(ui[k], 5, "clamp", out=uo[k], stream=s),
+         "sobel_magnitude_l2_f32": lambda k, s: lop.sobel_magnitude(fi[k], "clamp", out=fo[k], stream=s),
+         "sobel_magnitude_l1_u8_i32": lambda k, s: lop.sobel_magnitude(ui[k], "clamp", out=io_[k], stream=s)}
 res = {}
 for name, fn in cases.items():
     s2 = torch.cuda.Stream()
