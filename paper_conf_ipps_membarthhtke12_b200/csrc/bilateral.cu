@@ -1154,7 +1154,9 @@ static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
     // latency-bound and the TMEM allocation / barriers / ring clearing cost more
     // than the occupancy buys (config 1, 256^2 3x3: 4.5 -> 6.1 us per launch).
     // Both kernels give the same bits, so the choice is free to depend on size.
-    const bool tm = pair_tmem_enabled() &&
+    // and windows of 9 x 9 and up: for 3 x 3 the register kernel is faster (4096^2: 82 vs
+    // 98 us), 5 x 5 / 7 x 7 tie (profiles/r02/sweep_bilateral_pair_vs_sep_tm.jsonl)
+    const bool tm = pair_tmem_enabled() && R >= 4 &&
                     (double)p0.c.in.W * (double)p0.c.in.GH * (double)p0.c.batch >= 1024.0 * 1024.0;
     static PerDevice smem_set, resident_cache, smem_set_tm, resident_cache_tm;
     const size_t smem = tm ? std::max((size_t)pair::NW * pair::ShapeTM<R>::WARP_FLOATS * sizeof(float),
