@@ -365,10 +365,10 @@ __global__ void __launch_bounds__(256) local_small_kernel(const __grid_constant_
         const int ix0 = tx0 + a.off_x - HX, iy0 = ty0 + a.off_y - a.ry;
         const int sh = rows + 2 * a.ry;                                 // fetched rows
         if (bulk_ok(a, ix0, iy0, sh)) {
-            if (tid == 0) {
+            {                                                        // rows spread over the threads
                 const char *src = a.in.data + (int64_t)b * a.in.bstride + (int64_t)iy0 * a.in.stride +
                                   (int64_t)ix0 * 4;
-                for (int r = 0; r < sh; ++r)
+                for (int r = tid; r < sh; r += blockDim.x * blockDim.y)
                     asm volatile(
                         "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                         ::"r"(smem_addr(sm + base + r * pitch)), "l"(src + (int64_t)r * a.in.stride),
