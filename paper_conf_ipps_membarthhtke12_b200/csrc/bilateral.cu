@@ -495,9 +495,11 @@ __device__ __forceinline__ float lane_shift(float x, int o)
 // One window row dy of the half window for this lane's 4 owners (scalar; DY0:
 // dy = 0, own side dx = 0..R with the centre, partner side dx = 1..R): own
 // sums (rd, rp) and partner sums (qd, qp) of the receiving columns.
+// wc: the centre tap's weight ex2(lx[R]) (difference exactly 0), computed once
+// per thread instead of per pixel -- the same bits as evaluating it here.
 template <int R, int PAD, bool DY0>
 __device__ __forceinline__ void pair_row1(const float *v, const float cen[4], const float *lx, float nk,
-                                          float rd[4], float rp[4], float qd[4], float qp[4])
+                                          float wc, float rd[4], float rp[4], float qd[4], float qp[4])
 {
     constexpr int dx0 = DY0 ? 0 : -R;             // own side: first dx of this row
     constexpr int px0 = DY0 ? 1 : -R;             // partner side: first dx of this row
@@ -508,7 +510,7 @@ __device__ __forceinline__ void pair_row1(const float *v, const float cen[4], co
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
             const float jq = v[PAD + j + dx];
-            w[j] = bilateral_weight<false, true>(jq, cen[j], lx[dx + R], nk);
+            w[j] = DY0 && dx == 0 ? wc : bilateral_weight<false, true>(jq, cen[j], lx[dx + R], nk);
             if (dx == dx0) { rd[j] = w[j]; rp[j] = __fmul_rn(w[j], jq); }
             else { rd[j] = __fadd_rn(rd[j], w[j]); rp[j] = __fmaf_rn(w[j], jq, rp[j]); }
         }
@@ -718,6 +720,7 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
     // independent of the iteration space (owner push groups by lane)
     const int ox0 = (c.roi_x0 & ~3) + blockIdx.x * S::OW;        // first output column of the warp
     const int T = p.pair_rows;
+    const float wc = ex2_approx(p.lx[R]);                        // centre weight (see pair_row1)
     const int y0 = c.roi_y0 + (blockIdx.y * pair::NW + warp) * T;
     const int roi_y1 = c.roi_y0 + c.roi_h;
     if (y0 >= roi_y1) return;                                    // warp-uniform; warps are independent
@@ -757,7 +760,7 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
         if (kmin <= 0) {                                         // dy = 0: own row (scalar)
             float rd[4], rp[4], qd[4], qp[4];
 #pragma unroll
-            pair_row1<R, PAD, true>(u, cen, p.lx, p.nk, rd, rp, qd, qp);
+            pair_row1<R, PAD, true>(u, cen, p.lx, p.nk, wc, rd, rp, qd, qp);
             const float cy = p.cy[R];
             fold4(cy, rd, rp, D[0], P[0]);
             fold4(cy, qd, qp, D[0], P[0]);
@@ -799,7 +802,7 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
             float v[4 * NV];
             load_row<NV>(ring1 + sl * SW4 + lane, v);
             float rd[4], rp[4], qd[4], qp[4];
-            pair_row1<R, PAD, false>(v, cen, p.lx, p.nk, rd, rp, qd, qp);
+            pair_row1<R, PAD, false>(v, cen, p.lx, p.nk, wc, rd, rp, qd, qp);
             const float cy = p.cy[2 * R];
             fold4(cy, rd, rp, D[0], P[0]);
             fold4(cy, qd, qp, D[R], P[R]);
@@ -939,6 +942,7 @@ __global__ void __maxnreg__(LOP_PAIR_TM_MAXREG) bilateral_pair_tm_kernel(const _
     const int b = blockIdx.z;
     const int ox0 = (c.roi_x0 & ~3) + blockIdx.x * S::OW;
     const int T = p.pair_rows;
+    const float wc = ex2_approx(p.lx[R]);                        // centre weight (see pair_row1)
     const int y0 = c.roi_y0 + (blockIdx.y * pair::NW + warp) * T;
     const int roi_y1 = c.roi_y0 + c.roi_h;
     if (y0 < roi_y1) {                                           // warp-uniform
@@ -982,7 +986,7 @@ __global__ void __maxnreg__(LOP_PAIR_TM_MAXREG) bilateral_pair_tm_kernel(const _
             float *D0 = DP, *P0 = DP + 4;
             if (kmin <= 0) {                                     // dy = 0: own row (scalar)
                 float rd[4], rp[4], qd[4], qp[4];
-                pair_row1<R, PAD, true>(u, cen, p.lx, p.nk, rd, rp, qd, qp);
+                pair_row1<R, PAD, true>(u, cen, p.lx, p.nk, wc, rd, rp, qd, qp);
                 const float cy = p.cy[R];
                 fold4(cy, rd, rp, D0, P0);
                 fold4(cy, qd, qp, D0, P0);
@@ -1028,7 +1032,7 @@ __global__ void __maxnreg__(LOP_PAIR_TM_MAXREG) bilateral_pair_tm_kernel(const _
                 float v[4 * NV];
                 load_row_x<NV>(ring2 + sl * SW, lane, v);
                 float rd[4], rp[4], qd[4], qp[4];
-                pair_row1<R, PAD, false>(v, cen, p.lx, p.nk, rd, rp, qd, qp);
+                pair_row1<R, PAD, false>(v, cen, p.lx, p.nk, wc, rd, rp, qd, qp);
                 const float cy = p.cy[2 * R];
                 fold4(cy, rd, rp, D0, P0);
                 const int kr = ts0 + R >= NT ? ts0 + R - NT : ts0 + R;
