@@ -173,6 +173,41 @@ __global__ void __launch_bounds__(glob::NT) global_partial_kernel(const __grid_c
         return t;                                                 // same bits in every thread
     };
     const double part = cta_reduce(acc);
+    if constexpr (OP == RED_MIN || OP == RED_MAX) {
+        // MIN / MAX are order-independent: each CTA folds its part into one word
+        // with an integer atomic (an order-preserving encoding, identity 0, in the
+        // high half of work[kGlobalCounter]); the last CTA decodes it -- no
+        // 512-part read and tree at the end.  Same value as the tree, any order.
+        __shared__ bool lastm;
+        unsigned int *count = reinterpret_cast<unsigned int *>(p.work + kGlobalCounter);
+        if (threadIdx.x == 0) {
+            uint32_t enc;
+            if constexpr (F) {
+                const uint32_t bits = __float_as_uint((float)part);
+                const uint32_t ord = (bits >> 31) ? ~bits : (bits | 0x80000000u);   // monotone in the value
+                enc = OP == RED_MAX ? ord : ~ord;
+            } else {
+                enc = OP == RED_MAX ? (uint32_t)part : 255u - (uint32_t)part;
+            }
+            atomicMax(count + 1, enc);
+            __threadfence();
+            lastm = atomicAdd(count, 1u) == kGlobalParts - 1;
+        }
+        __syncthreads();
+        if (!lastm || threadIdx.x != 0) return;
+        __threadfence();
+        const uint32_t enc = atomicExch(count + 1, 0u);                // read and reset
+        double total;
+        if constexpr (F) {
+            const uint32_t ord = OP == RED_MAX ? enc : ~enc;
+            total = (double)__uint_as_float((ord & 0x80000000u) ? (ord ^ 0x80000000u) : ~ord);
+        } else {
+            total = (double)(OP == RED_MAX ? enc : 255u - enc);
+        }
+        *p.result = total;
+        *count = 0u;
+        return;
+    }
     // The last CTA to finish combines the parts (fixed tree over the part index,
     // so the result does not depend on which CTA is last); the arrival counter
     // lives in work[kGlobalCounter] and is reset for the next call.
