@@ -341,7 +341,9 @@ lop_status lop_pyramid_expand_execute(const lop_iteration_space *is, const lop_a
  * levels: 1 .. 16 (1 = the bilateral filter itself); sigma_r: `levels` host
  * floats.  d_workspace: device memory of at least
  * lop_multires_workspace_bytes() bytes (16-B aligned), owned by the caller.
- * At most 4 * levels kernel launches on cuda_stream, nothing synchronised. */
+ * At most 4 * levels kernel launches on cuda_stream, nothing synchronised; if a
+ * launch fails part of the sequence may already be enqueued (the status says
+ * which level failed) and the output is unspecified. */
 lop_status lop_multires_workspace_bytes(int32_t width, int32_t height, int32_t batch,
                                         int32_t levels, int64_t *bytes);
 lop_status lop_multires_bilateral_execute(const lop_iteration_space *is, const lop_accessor *in,
