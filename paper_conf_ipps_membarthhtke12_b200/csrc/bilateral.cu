@@ -863,8 +863,12 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
 #ifndef LOP_PAIR_TM_MAXREG
 #define LOP_PAIR_TM_MAXREG 128
 #endif
+#ifndef LOP_PAIR_TM_DY_UNROLL
+#define LOP_PAIR_TM_DY_UNROLL 1   // packed row-pair loop of the TMEM kernel (1: rolled)
+#endif
 namespace pair {
 constexpr int kTmemCols = 64;                          // per CTA; >= 8 (R + 1) for R <= 7
+constexpr int kTmDyUnroll = LOP_PAIR_TM_DY_UNROLL;
 constexpr int kTmemMinSmem = 25600;                    // dynamic smem floor: <= 8 CTAs / SM
 template <int R> struct ShapeTM {
     static constexpr int WARP_FLOATS = Shape<R>::RING2 + 2 * Shape<R>::SW;   // ring2, staging, column map
@@ -991,7 +995,7 @@ __global__ void __maxnreg__(LOP_PAIR_TM_MAXREG) bilateral_pair_tm_kernel(const _
                 fold4(cy, rd, rp, D0, P0);
                 fold4(cy, qd, qp, D0, P0);
             }
-#pragma unroll 1
+#pragma unroll pair::kTmDyUnroll
             for (int dy = 1; dy + 1 <= R; dy += 2) {             // row pairs (dy, dy+1): packed
                 if (dy + 1 < kmin) continue;
                 const int sl = slot0 + dy >= NR ? slot0 + dy - NR : slot0 + dy;
