@@ -727,13 +727,149 @@ int swar_mode(const ConvSep &s)
     return bin5 ? (SW_ON | SW_SYM | SW_SH8 | SW_BIN5) : (SW_ON | SW_SYM | SW_SH8);
 }
 
+// u8 Gaussian 5x5 (SW_BIN5), 16 pixels per thread: the SWAR arithmetic of
+// conv_u8_swar<2, ., BIN5> (same integer operations per pixel, so the same
+// bytes) on four staged words per thread and row instead of two, which halves
+// the per-pixel share of the halo words, their unpacking and the per-warp
+// set-up.  A CTA (128 threads) owns 2048 columns x TS16 rows.
+namespace conv16 {
+constexpr int NT = 128, PX = 16, TWE = NT * PX, PADE = 16, SWE = TWE + 2 * PADE;
+}
+
+template <int TS, bool FULL, bool VEC>
+__device__ __forceinline__ void conv_u8_bin5_x16_rows(const uint8_t *tcol, int srows, char *orow, int64_t ostride,
+                                                      int ox0, int roi_x1, bool ovec)
+{
+    constexpr int SWE = conv16::SWE, R = 2;
+    constexpr uint32_t rnd = 0x00800080u;                       // 2^7 per lane (shift 8)
+    uint32_t h[2 * R + 1][8];                                   // lanes (q, q+2), q in J
+    constexpr int J[8] = {0, 1, 4, 5, 8, 9, 12, 13};
+#pragma unroll
+    for (int k = 0; k < TS + 2 * R; ++k) {
+        if (!FULL && k >= srows) break;
+        const uint8_t *rp = tcol + k * SWE;
+        const uint4 cv = *reinterpret_cast<const uint4 *>(rp);
+        const uint32_t W[6] = {*reinterpret_cast<const uint32_t *>(rp - 4), cv.x, cv.y, cv.z, cv.w,
+                               *reinterpret_cast<const uint32_t *>(rp + 16)};
+        uint32_t E[6], O[6];
+#pragma unroll
+        for (int i = 0; i < 6; ++i) {
+            E[i] = __byte_perm(W[i], 0u, 0x4240);                // bytes 0, 2 -> lanes
+            O[i] = __byte_perm(W[i], 0u, 0x4341);                // bytes 1, 3 -> lanes
+        }
+        uint32_t S[14 + 2 * R];                                 // S[q + R] = lanes (q, q+2), q in [-R, 13+R]
+#pragma unroll
+        for (int q = -R; q <= 13 + R; ++q) {
+            const int wi = (q + 4) >> 2, sh = (q + 4) & 3;
+            if (sh == 0) S[q + R] = E[wi];
+            else if (sh == 1) S[q + R] = O[wi];
+            else if (sh == 2) S[q + R] = __byte_perm(E[wi], E[wi + 1], 0x5412);
+            else S[q + R] = __byte_perm(O[wi], O[wi + 1], 0x5412);
+        }
+        uint32_t *hk = h[k % (2 * R + 1)];
+#pragma unroll
+        for (int jj = 0; jj < 8; ++jj) {
+            const uint32_t *x = S + J[jj];
+            hk[jj] = (x[0] + x[4]) + ((x[1] + x[3]) << 2) + 6u * x[2];
+        }
+        const int o = k - 2 * R;
+        if (o < 0) continue;
+        uint32_t q8[8];
+#pragma unroll
+        for (int jj = 0; jj < 8; ++jj) {
+            const uint32_t h0 = h[o % 5][jj], h1 = h[(o + 1) % 5][jj], h2 = h[(o + 2) % 5][jj],
+                           h3 = h[(o + 3) % 5][jj], h4 = h[(o + 4) % 5][jj];
+            q8[jj] = (h0 + h4 + rnd) + ((h1 + h3) << 2) + 6u * h2;
+        }
+        const uint4 outw = make_uint4(__byte_perm(q8[0], q8[1], 0x7351), __byte_perm(q8[2], q8[3], 0x7351),
+                                      __byte_perm(q8[4], q8[5], 0x7351), __byte_perm(q8[6], q8[7], 0x7351));
+        uint8_t *op = reinterpret_cast<uint8_t *>(orow) + ox0;      // output row o (running pointer)
+        orow += ostride;
+        if (VEC || ovec) {
+            *reinterpret_cast<uint4 *>(op) = outw;
+        } else {
+            const uint32_t w4[4] = {outw.x, outw.y, outw.z, outw.w};
+#pragma unroll
+            for (int j = 0; j < 16; ++j)
+                if (ox0 + j < roi_x1) op[j] = (uint8_t)(w4[j >> 2] >> (8 * (j & 3)));
+        }
+    }
+}
+
+template <int TS>
+__global__ void __launch_bounds__(conv16::NT) conv_u8_bin5_x16_kernel(const __grid_constant__ ConvSep p)
+{
+    constexpr int R = 2, SWE = conv16::SWE;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    __shared__ __align__(8) uint64_t bar;
+    uint8_t *tile = smem_raw;
+    const Common &c = p.c;
+    const int b = blockIdx.z;
+    const int tx0 = c.roi_x0 + (int)blockIdx.x * conv16::TWE, ty0 = c.roi_y0 + (int)blockIdx.y * TS;
+    const int nrows = min(TS, c.roi_y0 + c.roi_h - ty0), srows = nrows + 2 * R;
+    const int roi_x1 = c.roi_x0 + c.roi_w;
+    if (threadIdx.x == 0) {
+        asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&bar)));
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    stage_rows<uint8_t, SWE, conv16::NT>(c, b, tx0 + c.off_x - conv16::PADE, ty0 + c.off_y - R, srows, tile, &bar);
+    __syncthreads();
+    mbar_wait(&bar, 0);
+    const int ox0 = tx0 + threadIdx.x * conv16::PX;
+    if (ox0 >= roi_x1) return;
+    char *obase = c.out.data + (int64_t)b * c.out.bstride;
+    const bool ovec = ox0 + conv16::PX <= roi_x1 && (ox0 % 16) == 0 &&
+                      ((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) % 16) == 0;
+    const bool cta_vec = tx0 + conv16::TWE <= roi_x1 && (tx0 % 16) == 0 &&
+                         ((reinterpret_cast<uintptr_t>(obase) | (uintptr_t)c.out.stride) % 16) == 0;
+    const uint8_t *tcol = tile + conv16::PADE + threadIdx.x * conv16::PX;
+    char *orow = obase + (int64_t)ty0 * c.out.stride;
+    if (nrows == TS && cta_vec)
+        conv_u8_bin5_x16_rows<TS, true, true>(tcol, srows, orow, c.out.stride, ox0, roi_x1, ovec);
+    else if (nrows == TS)
+        conv_u8_bin5_x16_rows<TS, true, false>(tcol, srows, orow, c.out.stride, ox0, roi_x1, ovec);
+    else
+        conv_u8_bin5_x16_rows<TS, false, false>(tcol, srows, orow, c.out.stride, ox0, roi_x1, ovec);
+}
+
+template <int TS>
+cudaError_t launch_bin5_x16(const ConvSep &s, cudaStream_t stream)
+{
+    const size_t smem = (size_t)(TS + 4) * conv16::SWE;
+    static PerDevice smem_set;
+    cudaError_t e = ensure_smem(conv_u8_bin5_x16_kernel<TS>, smem, smem_set);
+    if (e != cudaSuccess) return e;
+    dim3 grid((s.c.roi_w + conv16::TWE - 1) / conv16::TWE, (s.c.roi_h + TS - 1) / TS, s.c.batch);
+    conv_u8_bin5_x16_kernel<TS><<<grid, conv16::NT, smem, stream>>>(s);
+    return cudaGetLastError();
+}
+
+// LOP_CONV_X16: 0 = the 8-pixel kernel; 4 / 8 / 16 = the 16-pixel kernel with that many rows
+// per tile.  4096^2 (tools/time_conv_all.py): 8-pixel kernel 11.15 us; 16 pixels x 4 / 8 / 16
+// rows 11.6 / 10.8 / 11.6 us -- 8 rows (1024 CTAs) is the default.
+static int bin5_x16_rows()
+{
+    static const int v = [] {
+        const char *env = std::getenv("LOP_CONV_X16");
+        return env ? std::atoi(env) : 8;
+    }();
+    return v;
+}
+
 template <int R>
 cudaError_t dispatch_swar_r(const ConvSep &s, cudaStream_t stream)
 {
     const int mode = swar_mode(s);
     if constexpr (R == 2) {
-        if (mode == (SW_ON | SW_SYM | SW_SH8 | SW_BIN5))
+        if (mode == (SW_ON | SW_SYM | SW_SH8 | SW_BIN5)) {
+            if (!std::getenv("LOP_CONV_CFG")) {                 // (a tile-config sweep keeps the 8-px kernel)
+                if (bin5_x16_rows() == 16) return launch_bin5_x16<16>(s, stream);
+                if (bin5_x16_rows() == 8) return launch_bin5_x16<8>(s, stream);
+                if (bin5_x16_rows() == 4) return launch_bin5_x16<4>(s, stream);
+            }
             return launch_sep<uint8_t, uint8_t, R, SW_ON | SW_SYM | SW_SH8 | SW_BIN5>(s, stream);
+        }
     }
     if (mode & SW_SH8)
         return launch_sep<uint8_t, uint8_t, R, SW_ON | SW_SYM | SW_SH8>(s, stream);
