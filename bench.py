@@ -620,10 +620,13 @@ def extras(lop, synthetic, dev, stream, peaks):
         return statistics.median(ts)
 
     modes = {}
-    for mode in ("undefined", "clamp", "repeat", "mirror", "constant"):
-        ms = timed(lambda: lop.bilateral(img, 3.0, 5.0, mode, size=13, out=res, stream=stream),
-                   10, False)
-        modes[mode] = round(H * Wd / ms / 1e3, 1)
+    # two passes over the modes, the better median per mode (one slow sample of a mode -- a
+    # clock dip, another process -- must not read as a mode effect)
+    for _ in range(2):
+        for mode in ("undefined", "clamp", "repeat", "mirror", "constant"):
+            ms = timed(lambda: lop.bilateral(img, 3.0, 5.0, mode, size=13, out=res, stream=stream),
+                       10, False)
+            modes[mode] = max(modes.get(mode, 0.0), round(H * Wd / ms / 1e3, 1))
     out["bilateral_13x13_4096_f32_Mpx_s"] = modes
     v = list(modes.values())
     out["bilateral_mode_spread"] = round(max(v) / min(v) - 1.0, 4)
