@@ -44,8 +44,8 @@ __device__ __forceinline__ bool pyr_vec_ok(const Geom &g, int b)
 // REDUCE.  Lane t of a warp owns coarse columns 2t, 2t + 1 of the warp's 64
 // (fine columns 4t .. 4t + 3: one 16-byte load per fine row, a warp reads 512
 // contiguous bytes) and streams 7 fine rows for 2 coarse rows; the two fine
-// columns left and the one right of its quad come from the neighbouring lanes
-// (SHFL; the warp's edge lanes load them).  Per fine row the horizontal sums
+// columns left and the one right of its quad are loaded by the lane too (L1
+// hits), every load issued before the first use.  Per fine row the horizontal sums
 // at the two even columns enter a 5-row register window; a coarse row is
 // complete every second fine row.  CTAs whose footprint leaves the image (or
 // an unaligned view) read every element through the boundary mode (Table I).
@@ -70,10 +70,20 @@ __global__ void __launch_bounds__(pyr::RW * pyr::RWARPS) pyr_reduce_kernel(const
     constexpr int NF = 2 * pyr::RROWS + 3;                            // fine rows per warp
     // all of the warp's row loads are issued before any is used (7 x 512 B in
     // flight per warp; a load-use chain per row left the kernel latency-bound)
+    // the two columns left and the one right of the quad are loaded by every lane
+    // as well (L1 hits: the neighbouring lanes' quads), all before the first use --
+    // the edge lanes' loads are no longer a dependent round trip per row
     float4 qs[NF];
+    float2 ls[NF];
+    float rs[NF];
     if (inside) {
 #pragma unroll
-        for (int i = 0; i < NF; ++i) qs[i] = __ldg(reinterpret_cast<const float4 *>(row_ptr<float>(g, b, fy0 + i) + fx));
+        for (int i = 0; i < NF; ++i) {
+            const float *rp = row_ptr<float>(g, b, fy0 + i) + fx;
+            qs[i] = __ldg(reinterpret_cast<const float4 *>(rp));
+            ls[i] = __ldg(reinterpret_cast<const float2 *>(rp - 2));
+            rs[i] = __ldg(rp + 4);
+        }
     }
     // border CTAs: the 7 columns of the lane resolved once (Table I; -1 = the
     // CONSTANT value), each row resolved once per row
@@ -88,13 +98,8 @@ __global__ void __launch_bounds__(pyr::RW * pyr::RWARPS) pyr_reduce_kernel(const
         const int fy = fy0 + i;
         float f[7];                                                    // fine columns fx - 2 .. fx + 4
         if (inside) {
-            const float *rp = row_ptr<float>(g, b, fy) + fx;
             const float4 q = qs[i];
-            float l2 = __shfl_up_sync(0xffffffffu, q.z, 1), l1 = __shfl_up_sync(0xffffffffu, q.w, 1);
-            float r1 = __shfl_down_sync(0xffffffffu, q.x, 1);
-            if (lane == 0) { l2 = __ldg(rp - 2); l1 = __ldg(rp - 1); }
-            if (lane == 31) r1 = __ldg(rp + 4);
-            f[0] = l2; f[1] = l1; f[2] = q.x; f[3] = q.y; f[4] = q.z; f[5] = q.w; f[6] = r1;
+            f[0] = ls[i].x; f[1] = ls[i].y; f[2] = q.x; f[3] = q.y; f[4] = q.z; f[5] = q.w; f[6] = rs[i];
         } else {
             int row;
             const bool row_ok = resolve_row(fy, g, p.mode, row);
