@@ -187,6 +187,36 @@ __device__ __forceinline__ void local_stage(const LocalAcc &a, int b, int ix0, i
             return;
         }
     }
+    if (U8 && interior && vec && pitch <= 256) {
+        // u8 interior, rows up to 256 bytes: each lane fetches its words of 4 rows
+        // before storing any (8 independent loads in flight per lane; one row per
+        // iteration made every row a dependent DRAM round trip of the warp)
+        for (int r0 = r_lo + warp; r0 < r_hi; r0 += 4 * nwarps) {
+            uint32_t w[4][2];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const int r = r0 + u * nwarps;
+                const char *rp = fb + (int64_t)(iy0 + r) * a.in.stride + ix0;
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    const int x = 4 * lane + 128 * h;
+                    w[u][h] = r < r_hi && x < pitch ? __ldg(reinterpret_cast<const uint32_t *>(rp + x)) : 0u;
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                const int r = r0 + u * nwarps;
+#pragma unroll
+                for (int h = 0; h < 2; ++h) {
+                    const int x = 4 * lane + 128 * h;
+                    if (r < r_hi && x < pitch)
+                        *reinterpret_cast<int4 *>(t + r * pitch + x) =
+                            make_int4(w[u][h] & 0xFF, (w[u][h] >> 8) & 0xFF, (w[u][h] >> 16) & 0xFF, w[u][h] >> 24);
+                }
+            }
+        }
+        return;
+    }
     for (int r = r_lo + warp; r < r_hi; r += nwarps) {
         V *trow = t + r * pitch;
         if (interior) {
