@@ -239,6 +239,20 @@ __device__ __forceinline__ void store4(const Common &c, int b, int oy, int x_out
     }
 }
 
+// Store the outputs of lane columns x_out .. x_out + 3 that lie in [xs0, xs1).
+__device__ __forceinline__ void pair_store_span(const Common &c, int b, int s, int x_out, int xs0, int xs1,
+                                                const float res[4])
+{
+    if (xs0 == x_out && xs1 == x_out + 4) {
+        store4(c, b, s, x_out, res);
+        return;
+    }
+    float *orow = reinterpret_cast<float *>(c.out.data + (int64_t)b * c.out.bstride + (int64_t)s * c.out.stride);
+#pragma unroll
+    for (int j = 0; j < 4; ++j)
+        if (x_out + j >= xs0 && x_out + j < xs1) orow[x_out + j] = res[j];
+}
+
 template <int NV>
 __device__ __forceinline__ void load_row(const float4 *rowv, float *v)
 {
@@ -461,6 +475,11 @@ template <int R> struct Shape {
     static constexpr int HLN = (R + 3) / 4;            // halo lanes each side
     static constexpr int HL = 4 * HLN;                 // halo columns each side
     static constexpr int OW = 128 - 2 * HL;            // output columns per warp
+    // the TMEM kernel's TIGHT geometry: frame columns [R, R + OWT) are complete
+    // (every partner of them is owned inside the frame); OWT a multiple of 4 so
+    // frame starts stay at x = 0 mod 4; lanes straddling the output edge store
+    // their inner columns (13x13: 116 of 128 columns instead of 112)
+    static constexpr int OWT = (128 - 2 * R) & ~3;
     static constexpr int PAD = HL;                     // smem columns left of frame column 0
     static constexpr int SW = 128 + 2 * PAD;           // smem row (floats)
     static constexpr int NV = PAD / 2 + 1;             // float4 per lane per row: 4L-PAD .. 4L+3+PAD
@@ -759,7 +778,6 @@ __global__ void __maxnreg__(LOP_PAIR_MAXREG) bilateral_pair_kernel(const __grid_
         const float cen[4] = {u[PAD], u[PAD + 1], u[PAD + 2], u[PAD + 3]};
         if (kmin <= 0) {                                         // dy = 0: own row (scalar)
             float rd[4], rp[4], qd[4], qp[4];
-#pragma unroll
             pair_row1<R, PAD, true>(u, cen, p.lx, p.nk, wc, rd, rp, qd, qp);
             const float cy = p.cy[R];
             fold4(cy, rd, rp, D[0], P[0]);
@@ -919,11 +937,15 @@ __device__ __forceinline__ void load_row_x(const float2 *slot, int lane, float *
     }
 }
 
-template <int R>
+// TIGHT: frames of OWT output columns (launches that span several waves, where
+// fewer frames mean fewer waves); otherwise the lane-aligned OW of the register
+// kernel (its simpler store path measured faster within one wave).  The frame
+// geometry never changes a result: every pixel's order depends on x mod 4 only.
+template <int R, bool TIGHT>
 __global__ void __maxnreg__(LOP_PAIR_TM_MAXREG) bilateral_pair_tm_kernel(const __grid_constant__ BilateralSep p)
 {
     using S = pair::Shape<R>;
-    constexpr int SW = S::SW, NV = S::NV, NR = S::NR, PAD = S::PAD, HLN = S::HLN;
+    constexpr int SW = S::SW, NV = S::NV, NR = S::NR, PAD = S::PAD;
     constexpr int NT = R + 1;                                    // TMEM ring slots
     const Common &c = p.c;
     const Geom &g = c.in;
@@ -944,14 +966,15 @@ __global__ void __maxnreg__(LOP_PAIR_TM_MAXREG) bilateral_pair_tm_kernel(const _
     asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
     const uint32_t tbase = tm_base_sh + ((uint32_t)(32 * (warp & 3)) << 16);
     const int b = blockIdx.z;
-    const int ox0 = (c.roi_x0 & ~3) + blockIdx.x * S::OW;
+    const int ox0 = TIGHT ? ((c.roi_x0 - R) & ~3) + blockIdx.x * S::OWT + R   // frame start + R
+                          : (c.roi_x0 & ~3) + blockIdx.x * S::OW;             // frame start + HL
     const int T = p.pair_rows;
     const float wc = ex2_approx(p.lx[R]);                        // centre weight (see pair_row1)
     const int y0 = c.roi_y0 + (blockIdx.y * pair::NW + warp) * T;
     const int roi_y1 = c.roi_y0 + c.roi_h;
     if (y0 < roi_y1) {                                           // warp-uniform
         const int yend = min(y0 + T, roi_y1);
-        const int ix0 = ox0 - S::HL + c.off_x - PAD;
+        const int ix0 = ox0 - (TIGHT ? R : S::HL) + c.off_x - PAD;
         const bool vec_ok = ((ix0 & 3) == 0) && ((g.stride & 15) == 0) &&
                             ((reinterpret_cast<uintptr_t>(g.data + (int64_t)b * g.bstride) & 15) == 0);
         pair_colmap<SW>(c, ix0, cm, lane);
@@ -971,9 +994,19 @@ __global__ void __maxnreg__(LOP_PAIR_TM_MAXREG) bilateral_pair_tm_kernel(const _
         const float zero8[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
 #pragma unroll
         for (int k = 0; k < NT; ++k) tm_st8(tbase + 8 * k, zero8);
-        const int x_out = ox0 + 4 * (lane - HLN);
-        const bool store_lane = lane >= HLN && lane < 32 - HLN && x_out < c.roi_x0 + c.roi_w &&
-                                x_out + 3 >= c.roi_x0;
+        // this lane's stored columns [xs0, xs1): TIGHT frames store the frame columns
+        // [R, R + OWT) (straddling lanes partly); aligned frames whole lanes
+        // [HLN, 32 - HLN) (the register kernel's store path)
+        const int x_out = TIGHT ? ox0 - R + 4 * lane : ox0 + 4 * (lane - S::HLN);
+        int xs0 = 0, xs1 = 0;
+        bool store_lane;
+        if constexpr (TIGHT) {
+            xs0 = max(x_out, max(ox0, c.roi_x0));
+            xs1 = min(x_out + 4, min(ox0 + S::OWT, c.roi_x0 + c.roi_w));
+            store_lane = xs1 > xs0;
+        } else {
+            store_lane = lane >= S::HLN && lane < 32 - S::HLN && x_out < c.roi_x0 + c.roi_w && x_out + 3 >= c.roi_x0;
+        }
         int slot0 = 0, ts0 = 0;                                  // ring slot / TMEM slot of row s
 #pragma unroll 1
         for (int s = y0 - R; s < yend; ++s) {
@@ -1050,7 +1083,9 @@ __global__ void __maxnreg__(LOP_PAIR_TM_MAXREG) bilateral_pair_tm_kernel(const _
                 float res[4];
 #pragma unroll
                 for (int j = 0; j < 4; ++j) res[j] = bilateral_finish_scaled(D0[j], P0[j], p.inv_alpha);
-                if (x_out >= c.roi_x0) {
+                if (TIGHT) {
+                    pair_store_span(c, b, s, x_out, xs0, xs1, res);
+                } else if (x_out >= c.roi_x0) {
                     store4(c, b, s, x_out, res);
                 } else {
                     float *orow = reinterpret_cast<float *>(c.out.data + (int64_t)b * c.out.bstride +
@@ -1170,7 +1205,7 @@ static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
     const size_t smem = tm ? std::max((size_t)pair::NW * pair::ShapeTM<R>::WARP_FLOATS * sizeof(float),
                                       (size_t)pair::kTmemMinSmem)
                            : (size_t)pair::NW * S::WARP_FLOATS * sizeof(float);
-    auto kern = tm ? bilateral_pair_tm_kernel<R> : bilateral_pair_kernel<R>;
+    auto kern = tm ? bilateral_pair_tm_kernel<R, false> : bilateral_pair_kernel<R>;
     cudaError_t e;
     const int64_t resident =
         tm ? resident_ctas_tmem(kern, pair::NW * 32, smem, pair::kTmemCols, smem_set_tm, resident_cache_tm, e)
@@ -1179,21 +1214,10 @@ static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
     e = ensure_smem(kern, smem, tm ? smem_set_tm : smem_set);
     if (e != cudaSuccess) return e;
     BilateralSep p = p0;
-    const int64_t strips = ((p.c.roi_x0 & 3) + p.c.roi_w + S::OW - 1) / S::OW;
-    int T = 0;
-    if (const char *env = std::getenv("LOP_PAIR_ROWS")) T = std::atoi(env);
-    static thread_local int64_t memo_key[4] = {-1, -1, -1, -1};
-    static thread_local int memo_T = 0;
-    if (T <= 0 && memo_key[0] == p.c.roi_h && memo_key[1] == strips && memo_key[2] == p.c.batch &&
-        memo_key[3] == resident * 2 + tm)
-        T = memo_T;
-    if (T <= 0) {
-        // every T from 1 to the ROI height: waves of resident CTAs x rows per warp
-        // (+ warm-up); a partial wave costs a full one (few warps per SM
-        // cannot saturate the SFU).  Small images take small T: the row steps of
-        // a warp are serial (one global row fetch each), so a launch that fits
-        // in one wave is latency-bound by T + R steps (config 1: T = 1).
-        double best = 0;
+    // rows per warp T from the wave model, for a frame geometry of `strips` frames
+    auto plan = [&](int64_t strips, double &best) {
+        int T = 0;
+        best = 0;
         const int tmax = std::max(1, p.c.roi_h);
         for (int t = 1; t <= tmax; ++t) {
             const int64_t segs = (p.c.roi_h + t - 1) / t;
@@ -1202,12 +1226,47 @@ static cudaError_t launch_pair_r(const BilateralSep &p0, cudaStream_t stream)
             if (T == 0 || cost < best) { best = cost; T = t; }
             if (segs == 1) break;
         }
-        memo_key[0] = p.c.roi_h; memo_key[1] = strips; memo_key[2] = p.c.batch; memo_key[3] = resident * 2 + tm;
+        return T;
+    };
+    // lane-aligned frames of OW output columns, or (TMEM kernel) TIGHT frames of OWT
+    const int64_t strips_a = ((p.c.roi_x0 & 3) + p.c.roi_w + S::OW - 1) / S::OW;
+    const int64_t first_t = ((p.c.roi_x0 - R) & ~3) + R;
+    const int64_t strips_t = (p.c.roi_x0 + p.c.roi_w - first_t + S::OWT - 1) / S::OWT;
+    int T = 0;
+    if (const char *env = std::getenv("LOP_PAIR_ROWS")) T = std::atoi(env);
+    static thread_local int64_t memo_key[4] = {-1, -1, -1, -1};
+    static thread_local int memo_T = 0, memo_tight = 0;
+    int tight = 0;
+    if (T <= 0 && memo_key[0] == p.c.roi_h && memo_key[1] == strips_a * 4096 + p.c.roi_w % 4096 &&
+        memo_key[2] == p.c.batch && memo_key[3] == resident * 2 + tm) {
+        T = memo_T;
+        tight = memo_tight;
+    } else if (T <= 0) {
+        // every T from 1 to the ROI height: waves of resident CTAs x rows per warp
+        // (+ warm-up); a partial wave costs a full one (few warps per SM
+        // cannot saturate the SFU).  Small images take small T: the row steps of
+        // a warp are serial (one global row fetch each), so a launch that fits
+        // in one wave is latency-bound by T + R steps (config 1: T = 1).
+        // TIGHT frames when they cut the modelled time by more than the ~2 % their
+        // store path costs (launches spanning several waves: config 4's 1024-column
+        // frames, config 5's 32768-column bands); same results either way.
+        double cost_a = 0, cost_t = 0;
+        T = plan(strips_a, cost_a);
+        if (tm) {
+            const int Tt = plan(strips_t, cost_t);
+            if (cost_t < 0.97 * cost_a) { T = Tt; tight = 1; }
+        }
+        memo_key[0] = p.c.roi_h; memo_key[1] = strips_a * 4096 + p.c.roi_w % 4096;
+        memo_key[2] = p.c.batch; memo_key[3] = resident * 2 + tm;
         memo_T = T;
+        memo_tight = tight;
     }
+    if (const char *env = std::getenv("LOP_PAIR_TIGHT")) tight = tm && std::atoi(env) != 0;   // A/B
     p.pair_rows = T;
+    const int64_t strips = tight ? strips_t : strips_a;
     const int64_t segs = (p.c.roi_h + T - 1) / T;
     dim3 grid((unsigned)strips, (unsigned)((segs + pair::NW - 1) / pair::NW), p.c.batch);
+    if (tight) kern = bilateral_pair_tm_kernel<R, true>;
     kern<<<grid, pair::NW * 32, smem, stream>>>(p);
     return cudaGetLastError();
 }
