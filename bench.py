@@ -528,7 +528,7 @@ def run_lop(args, dist, peaks):
     # capture of the same kernel is committed under profiles/ 
     roofline["traffic"] = None
     roofline["traffic_note"] = ("dram bytes per launch (ncu --set full of the same kernel and "
-                                "config): profiles/r02/ncu_full_bilateral_pair_tm_s7.md")
+                                "config): profiles/r02/ncu_full_bilateral_pair_tm_s10.md")
     result = dict(metric=BASELINE_METRIC, value=round(value, 2), unit="Mpixel/s",
                   n_gpus=dist.world, steps=K, warmup=W, ms_per_step=round(total_ms / K, 5),
                   higher_is_better=True, scaling=wl["scaling"], vs_baseline=None, dtype="f32",
