@@ -76,3 +76,24 @@ def test_tm_kernel_roi_offset_frames(lop, monkeypatch):
         ref, _ = oracle.bilateral_f32_points(img, 3.0, 0.1, "mirror", xs + 2, ys - 3)
         got = out[f].cpu().numpy()[ys, xs]
         assert float(np.abs(got - ref).max()) <= 1e-5
+
+
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("win", [9, 13])
+def test_tight_frames_bit_identical(lop, monkeypatch, mode, win):
+    """TIGHT frames (frame columns [R, R + OWT)) and lane-aligned frames give the
+    same bits: the summation order depends on x mod 4 only.  ROI with an odd
+    start, accessor offset, two frames."""
+    monkeypatch.setenv("LOP_BILATERAL_PAIR", "1")
+    frames = torch.stack([synthetic.angio(1030, 1057, seed=s) for s in (3, 4)]).cuda()
+    roi = (13, 9, 1001, 1000)
+    outs = []
+    for tight in ("0", "1"):
+        monkeypatch.setenv("LOP_PAIR_TIGHT", tight)
+        o = torch.zeros_like(frames)
+        lop.bilateral(frames, (win - 1) / 4.0, 0.1, mode, constant=0.3, size=win, out=o, roi=roi,
+                      offset=(1, -2))
+        outs.append(o)
+    assert torch.equal(outs[0], outs[1])
+    x0, y0, w, h = roi
+    assert float(outs[1][:, :, x0 + w:].abs().max()) == 0.0    # nothing stored past the ROI
