@@ -364,10 +364,12 @@ __global__ void __launch_bounds__(256) local_small_kernel(const __grid_constant_
     const int rows = min(th, roi_y1 - ty0);
     const int tid = threadIdx.y * blockDim.x + threadIdx.x;
     // f32 interior footprints: one cp.async.bulk per staged row (TMA bulk
-    // engine, issued by one thread, completing on `sbar`); the rest element-wise
-    __shared__ __align__(8) uint64_t sbar;
+    // engine, rows spread over the threads), completing on the accessor's own
+    // mbarrier, so accessor k's taps start as soon as its rows have landed while
+    // the later accessors' rows are still in flight; the rest element-wise
+    __shared__ __align__(8) uint64_t sbar[kLocalMaxAcc];
     if (tid == 0) {
-        asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&sbar)));
+        for (int k = 0; k < p.n; ++k) asm volatile("mbarrier.init.shared.b64 [%0], 1;" ::"r"(smem_addr(&sbar[k])));
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
@@ -379,14 +381,13 @@ __global__ void __launch_bounds__(256) local_small_kernel(const __grid_constant_
                (a.in.stride & 15) == 0 && (reinterpret_cast<uintptr_t>(fb) & 15) == 0;
     };
     if (tid == 0) {
-        uint32_t nbytes = 0;
         for (int k = 0; k < p.n; ++k) {
             const LocalAcc &a = p.acc[k];
             const int ix0 = tx0 + a.off_x - HX, iy0 = ty0 + a.off_y - a.ry, sh = rows + 2 * a.ry;
-            if (bulk_ok(a, ix0, iy0, sh)) nbytes += (uint32_t)(sh * pitch * 4);
+            const uint32_t nbytes = bulk_ok(a, ix0, iy0, sh) ? (uint32_t)(sh * pitch * 4) : 0u;
+            asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;" ::"r"(smem_addr(&sbar[k])),
+                         "r"(nbytes) : "memory");
         }
-        asm volatile("mbarrier.arrive.expect_tx.shared.b64 _, [%0], %1;" ::"r"(smem_addr(&sbar)), "r"(nbytes)
-                     : "memory");
     }
     int base = 0;
 #pragma unroll 1
@@ -402,7 +403,7 @@ __global__ void __launch_bounds__(256) local_small_kernel(const __grid_constant_
                     asm volatile(
                         "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                         ::"r"(smem_addr(sm + base + r * pitch)), "l"(src + (int64_t)r * a.in.stride),
-                          "r"(pitch * 4), "r"(smem_addr(&sbar))
+                          "r"(pitch * 4), "r"(smem_addr(&sbar[k]))
                         : "memory");
             }
         } else {
@@ -415,9 +416,9 @@ __global__ void __launch_bounds__(256) local_small_kernel(const __grid_constant_
             sm[base + i] = (V)0;
         base += (th + 2 * a.ry) * pitch;
     }
-    mbar_wait(&sbar, 0);
-    __syncthreads();
+    __syncthreads();                                       // element-wise staging visible
     if (p.any_point) {                                     // point-operator prologue
+        for (int k = 0; k < p.n; ++k) mbar_wait(&sbar[k], 0);
         base = 0;
         for (int k = 0; k < p.n; ++k) {
             const LocalAcc &a = p.acc[k];
@@ -441,6 +442,7 @@ __global__ void __launch_bounds__(256) local_small_kernel(const __grid_constant_
     for (int k = 0; k < p.n; ++k) {
         const LocalAcc &a = p.acc[k];
         const int rx = a.rx, ry = a.ry;
+        mbar_wait(&sbar[k], 0);                             // accessor k's bulk rows have landed
         const V *t = sm + base + c0;                        // column c0 - HX of the input
         const V *mk = (const V *)(U8 ? (const void *)p.ms.i[k] : (const void *)p.ms.f[k]);
         V cen[OY][SX];
