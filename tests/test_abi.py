@@ -182,3 +182,50 @@ def test_chain_rejects_bad_masks_before_launch():
     st = lop.lib.lop_convolve_chain_execute(ctypes.byref(is_), ctypes.byref(acc), None,
                                             ctypes.byref(m1), None)
     assert st == _lib.LOP_ERR_INVALID
+
+
+def test_session5_entry_points_validate_before_launch():
+    """The point prologue, SUMSQ, pyramid and multiresolution entry points reject
+    bad arguments (host pointers, unknown ops, wrong sizes) without launching;
+    the multiresolution workspace size is a pure host function."""
+    lib = lop.lib
+    before = lop.launch_count()
+    host = np.zeros((8, 16), np.float32)
+    bc, acc, is_ = _views(data=host.ctypes.data)
+    accs = (ctypes.POINTER(_lib.lop_accessor) * 1)(ctypes.pointer(acc))
+    m = _lib.lop_mask()
+    ms = (ctypes.POINTER(_lib.lop_mask) * 1)(ctypes.pointer(m))
+    sc = (ctypes.c_double * 1)(2.0)
+    of = (ctypes.c_double * 1)(0.5)
+    assert lib.lop_local_execute_point(ctypes.byref(is_), accs, ms, 1, 0, 0, sc, of, None) == \
+        _lib.LOP_ERR_INVALID
+    assert lib.lop_global_reduce_execute(ctypes.byref(is_), 9, None, None, None) == _lib.LOP_ERR_INVALID
+    assert b"SUMSQ" in lib.lop_last_error()
+    bc.size_x = bc.size_y = 5
+    assert lib.lop_pyramid_reduce_execute(ctypes.byref(is_), ctypes.byref(acc), None) == \
+        _lib.LOP_ERR_INVALID
+    assert lib.lop_pyramid_expand_execute(ctypes.byref(is_), ctypes.byref(acc), None, 1.0, None) == \
+        _lib.LOP_ERR_INVALID
+    srs = (ctypes.c_float * 2)(0.1, 0.1)
+    assert lib.lop_multires_bilateral_execute(ctypes.byref(is_), ctypes.byref(acc), 0, 1.0, srs, None,
+                                              0, None) == _lib.LOP_ERR_INVALID
+    assert b"levels" in lib.lop_last_error()
+    assert lib.lop_multires_bilateral_execute(ctypes.byref(is_), ctypes.byref(acc), 2, 1.0, srs, None,
+                                              0, None) == _lib.LOP_ERR_INVALID
+    assert lop.launch_count() == before
+    # workspace: the Gaussian levels 1..L-1 plus one full-size level (B_0, later the
+    # filtered coarse levels), 256-B rounded; 1 level needs none
+    n = ctypes.c_int64(-1)
+    assert lib.lop_multires_workspace_bytes(4096, 4096, 1, 1, ctypes.byref(n)) == 0 and n.value == 0
+    sizes = []
+    for L in (2, 3, 4, 8):
+        assert lib.lop_multires_workspace_bytes(4096, 4096, 1, L, ctypes.byref(n)) == 0
+        sizes.append(n.value)
+    full = 4096 * 4096 * 4
+    assert sizes[0] == full + full // 4
+    assert all(a < b for a, b in zip(sizes, sizes[1:]))
+    assert sizes[-1] < full * 4 // 3 + full + 8 * 256
+    assert lib.lop_multires_workspace_bytes(4096, 4096, 2, 3, ctypes.byref(n)) == 0
+    assert n.value >= 2 * (full + full // 4)
+    assert lib.lop_multires_workspace_bytes(0, 4096, 1, 3, ctypes.byref(n)) == _lib.LOP_ERR_INVALID
+    assert lib.lop_multires_workspace_bytes(64, 64, 1, 17, ctypes.byref(n)) == _lib.LOP_ERR_INVALID
